@@ -1,0 +1,150 @@
+"""Seeded, counter-based synthetic input generators.
+
+This module is shared by the CUDA path's tests/bench AND by the oracle side
+(DESIGN.md "Input recipe").  It deliberately holds none of the method's
+arithmetic: no RMT, no kernel definitions -- only "element i of stream `seed`"
+= splitmix64(seed, i), mapped to the value distributions of the paper's
+workloads (AMD APP SDK-style random inputs, "input sizes were
+scaled to the maximum size ...").  Because every value is a pure function of
+(seed, global index), a shard [off, off+n) on any rank reproduces exactly the
+same numbers as the corresponding slice of the 1-GPU input.
+
+All functions return numpy arrays on the host; callers copy them to the GPU.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+_GOLDEN = np.uint64(0x9E3779B97F4A7C15)
+_M1 = np.uint64(0xBF58476D1CE4E5B9)
+_M2 = np.uint64(0x94D049BB133111EB)
+_CHUNK = 1 << 24
+
+
+def _mix(z: np.ndarray) -> np.ndarray:
+    z = (z ^ (z >> np.uint64(30))) * _M1
+    z = (z ^ (z >> np.uint64(27))) * _M2
+    return z ^ (z >> np.uint64(31))
+
+
+def u64(seed: int, n: int, offset: int = 0, stream: int = 0) -> np.ndarray:
+    """uint64 stream: splitmix64 of (seed, stream) keyed counter, element offset+i."""
+    key = _mix(np.array([(seed * 0x100000001B3 + stream * 0x1000193 + 1) & (2**64 - 1)],
+                        dtype=np.uint64))[0]
+    out = np.empty(n, dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        for s in range(0, n, _CHUNK):
+            e = min(n, s + _CHUNK)
+            idx = np.arange(offset + s, offset + e, dtype=np.uint64)
+            out[s:e] = _mix(idx * _GOLDEN + key)
+    return out
+
+
+def u32(seed: int, n: int, offset: int = 0, stream: int = 0) -> np.ndarray:
+    return (u64(seed, n, offset, stream) >> np.uint64(32)).astype(np.uint32)
+
+
+def uniform_f32(seed: int, n: int, offset: int = 0, stream: int = 0) -> np.ndarray:
+    """U[0,1) with 24 random bits: every value k*2^-24 is exact in fp32."""
+    k = (u64(seed, n, offset, stream) >> np.uint64(40)).astype(np.float64)
+    return (k * (2.0 ** -24)).astype(np.float32)
+
+
+# --------------------------------------------------------------------------
+# Per-workload recipes (SURVEY.md 8(d) synthetic inputs)
+# --------------------------------------------------------------------------
+
+def blackscholes_r(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """One U[0,1) draw per option (APP-SDK style; the kernel maps r -> S,K,T,R,sigma)."""
+    return uniform_f32(seed, n, offset)
+
+
+def binarysearch_inputs(seed: int, N: int, Q: int, q_offset: int = 0):
+    """Sorted, strictly increasing u32 A[N] spread over the full u32 range, and
+    uniform u32 queries q[Q].  A[i] = i*stride + (h(i) mod stride) (no prefix sum
+    needed to make it sorted)."""
+    stride = (1 << 32) // N
+    if stride < 1:
+        raise ValueError("N too large for u32 keys")
+    h = u32(seed, N, 0, stream=1).astype(np.uint64)
+    A = (np.arange(N, dtype=np.uint64) * np.uint64(stride) + h % np.uint64(stride)).astype(np.uint32)
+    q = u32(seed, Q, q_offset, stream=2)
+    return A, q
+
+
+def fwt_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """U[-1,1) fp32 (exact: 2*k*2^-24 - 1)."""
+    return (uniform_f32(seed, n, offset) * np.float32(2.0) - np.float32(1.0)).astype(np.float32)
+
+
+def fwt_ternary(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """x in {-1,0,1} (exact-integer pin input for the FWT)."""
+    return ((u32(seed, n, offset, stream=3) % np.uint32(3)).astype(np.int64) - 1).astype(np.float32)
+
+
+def prefixsum_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """u32 U{0..255}."""
+    return (u32(seed, n, offset, stream=4) & np.uint32(0xFF)).astype(np.uint32)
+
+
+def reduction_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """u32 U{0..2^16-1}."""
+    return (u32(seed, n, offset, stream=5) & np.uint32(0xFFFF)).astype(np.uint32)
+
+
+def transpose_a(seed: int, H: int, W: int, row_offset: int = 0) -> np.ndarray:
+    """f32 U[0,1), H x W row-major."""
+    return uniform_f32(seed, H * W, row_offset * W, stream=6).reshape(H, W)
+
+
+def sobel_image(seed: int, H: int, W: int, row_offset: int = 0) -> np.ndarray:
+    """uchar4 image (H, W, 4): 64x64 checker blocks (edges) + diagonal ramp + 4-bit noise."""
+    y = np.arange(row_offset, row_offset + H, dtype=np.int64)[:, None, None]
+    x = np.arange(W, dtype=np.int64)[None, :, None]
+    c = np.arange(4, dtype=np.int64)[None, None, :]
+    block = (((x // 64) + (y // 64)) % 2) * 96
+    ramp = (x % 64) + (y % 64) + 8 * c
+    noise = (u32(seed, H * W * 4, row_offset * W * 4, stream=7).astype(np.int64)
+             & 15).reshape(H, W, 4)
+    return np.minimum(block + ramp + noise, 255).astype(np.uint8)
+
+
+def floydwarshall_w(seed: int, n: int) -> np.ndarray:
+    """Complete digraph, u32 weights U{1..200}, zero diagonal."""
+    w = (u32(seed, n * n, 0, stream=8) % np.uint32(200) + np.uint32(1)).reshape(n, n)
+    np.fill_diagonal(w, 0)
+    return w.astype(np.uint32)
+
+
+def dct_x(seed: int, H: int, W: int, row_offset: int = 0) -> np.ndarray:
+    """f32 U[0,255)."""
+    return (uniform_f32(seed, H * W, row_offset * W, stream=9) * np.float32(255.0)).reshape(H, W)
+
+
+def f32_to_bf16_bits(x: np.ndarray) -> np.ndarray:
+    """Round-to-nearest-even fp32 -> bf16, returned as uint16 bit patterns."""
+    b = np.ascontiguousarray(x, dtype=np.float32).view(np.uint32).astype(np.uint64)
+    b = b + np.uint64(0x7FFF) + ((b >> np.uint64(16)) & np.uint64(1))
+    return (b >> np.uint64(16)).astype(np.uint16)
+
+
+def bf16_bits_to_f32(b: np.ndarray) -> np.ndarray:
+    return (b.astype(np.uint32) << np.uint32(16)).view(np.float32)
+
+
+def matmul_bf16_normal(seed: int, rows: int, cols: int, stream: int, row_offset: int = 0) -> np.ndarray:
+    """bf16 N(0,1) (Box-Muller on two counter streams), returned as uint16 bits."""
+    n = rows * cols
+    off = row_offset * cols
+    u1 = (u64(seed, n, off, stream=stream) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+    u2 = (u64(seed, n, off, stream=stream + 1) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+    g = np.sqrt(-2.0 * np.log1p(-u1)) * np.cos(2.0 * np.pi * u2)
+    return f32_to_bf16_bits(g.astype(np.float32)).reshape(rows, cols)
+
+
+def matmul_bf16_int(seed: int, rows: int, cols: int, stream: int, lo: int = -4, hi: int = 4,
+                    row_offset: int = 0) -> np.ndarray:
+    """Integer-valued bf16 in [lo, hi] (exactness pin input), uint16 bits."""
+    n = rows * cols
+    v = (u32(seed, n, row_offset * cols, stream=stream) % np.uint32(hi - lo + 1)).astype(np.int64) + lo
+    return f32_to_bf16_bits(v.astype(np.float32)).reshape(rows, cols)

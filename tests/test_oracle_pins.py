@@ -1,0 +1,363 @@
+"""Pins for the CPU oracle (-m "not gpu").
+
+Each test checks the oracle against something other than itself: a closed
+form, an invariant, brute force on a tiny input, an independent algorithm or
+a library routine the definition reduces to.  A
+plausible mistake anywhere in oracle.c (dropped term, wrong sign or index,
+transposed operand) must fail one of these.
+"""
+import itertools
+import math
+
+import numpy as np
+import pytest
+import scipy.fft
+import scipy.ndimage
+
+import oracle
+from paper_conf_isca_waddenlgss14_b200 import inputs
+
+# ---------------------------------------------------------------- BlackScholes
+
+
+def test_cnd_matches_erfc_within_as_bound():
+    # A&S 26.2.17 has |error| < 7.5e-8 against the exact normal CDF.
+    for x in np.linspace(-8, 8, 4001):
+        exact = 0.5 * math.erfc(-x / math.sqrt(2.0))
+        assert abs(oracle.cnd(x) - exact) < 7.5e-8, x
+
+
+def test_cnd_symmetry():
+    # N(-x) = 1 - N(x) holds by construction for x != 0; at 0 the polynomial
+    # itself is off by its A&S error (5e-10).
+    for x in np.linspace(-5, 5, 100):
+        assert abs(oracle.cnd(x) + oracle.cnd(-x) - 1.0) < 1e-15
+    assert abs(oracle.cnd(0.0) - 0.5) < 7.5e-8
+
+
+def test_bs_textbook_point():
+    # Hull, Options Futures & Other Derivatives: S=K=100, T=1, r=5%, sigma=20%
+    c, p = oracle.bs_price(100.0, 100.0, 1.0, 0.05, 0.2)
+    assert abs(c - 10.45058) < 1e-4
+    assert abs(p - 5.57353) < 1e-4
+
+
+def _bs_exact(S, K, T, R, V):
+    N = lambda x: 0.5 * math.erfc(-x / math.sqrt(2.0))
+    d1 = (math.log(S / K) + (R + V * V / 2) * T) / (V * math.sqrt(T))
+    d2 = d1 - V * math.sqrt(T)
+    return S * N(d1) - K * math.exp(-R * T) * N(d2), K * math.exp(-R * T) * N(-d2) - S * N(-d1)
+
+
+def test_bs_workload_mapping_and_exact_price():
+    # R-BS1 mapping at r=0 and r=1 and a sample of draws, against the exact-erfc
+    # price; the A&S error bound gives |dC| <= 2*7.5e-8*(S+K).
+    r = inputs.blackscholes_r(7, 2000)
+    r = np.concatenate([r, np.array([0.0, 1.0 - 2**-24], np.float32)])
+    call, put = oracle.blackscholes(r)
+    for i, ri in enumerate(r.astype(np.float64)):
+        S = 10 * ri + 100 * (1 - ri)
+        T = 1 * ri + 10 * (1 - ri)
+        R = 0.01 * ri + 0.05 * (1 - ri)
+        V = 0.01 * ri + 0.10 * (1 - ri)
+        ce, pe = _bs_exact(S, S, T, R, V)
+        assert abs(call[i] - ce) <= 3e-7 * S
+        assert abs(put[i] - pe) <= 3e-7 * S
+
+
+def test_bs_put_call_parity_and_bounds():
+    r = inputs.blackscholes_r(3, 1 << 16)
+    call, put = oracle.blackscholes(r)
+    rr = r.astype(np.float64)
+    S = 10 * rr + 100 * (1 - rr)
+    T = 1 * rr + 10 * (1 - rr)
+    R = 0.01 * rr + 0.05 * (1 - rr)
+    disc = S * np.exp(-R * T)
+    assert np.max(np.abs(call - put - (S - disc))) < 1e-10 * 100
+    assert np.all(call >= np.maximum(0, S - disc) - 1e-9) and np.all(call <= S)
+    assert np.all(put >= np.maximum(0, disc - S) - 1e-9) and np.all(put <= disc)
+
+
+# ---------------------------------------------------------------- BinarySearch
+
+
+def test_binarysearch_closed_form_odd_numbers():
+    N = 1 << 16
+    A = (2 * np.arange(N, dtype=np.uint64) + 1).astype(np.uint32)
+    q = np.concatenate([np.arange(0, 2 * N + 8, dtype=np.uint32),
+                        inputs.u32(1, 4096)])
+    idx = oracle.binarysearch(A, q)
+    expect = np.minimum(N, q.astype(np.uint64) // 2)
+    assert np.array_equal(idx.astype(np.uint64), expect)
+
+
+def test_binarysearch_brute_force_tiny():
+    for N in [1, 2, 3, 7, 64]:
+        A, q = inputs.binarysearch_inputs(11 + N, N, 300)
+        q = np.concatenate([q, A, A + 1, np.array([0, 2**32 - 1], np.uint32)])
+        idx = oracle.binarysearch(A, q)
+        brute = np.array([(A < k).sum() for k in q], np.uint32)
+        assert np.array_equal(idx, brute)
+
+
+def test_binarysearch_vs_searchsorted():
+    A, q = inputs.binarysearch_inputs(5, 1 << 18, 1 << 16)
+    assert np.all(A[1:] > A[:-1])
+    assert np.array_equal(oracle.binarysearch(A, q), np.searchsorted(A, q, side="left").astype(np.uint32))
+
+
+# ---------------------------------------------------------------- FastWalshTransform
+
+
+def _hadamard(N):
+    i = np.arange(N)
+    pc = np.vectorize(lambda v: bin(v).count("1"))(i[:, None] & i[None, :])
+    return np.where(pc % 2 == 0, 1, -1).astype(np.int64)
+
+
+def test_fwt_brute_force_matrix():
+    for N in [1, 2, 4, 64, 1024]:
+        x = inputs.fwt_x(2, N)
+        y = oracle.fwt_f64(x)
+        ref = _hadamard(N).astype(np.float64) @ x.astype(np.float64)
+        assert np.allclose(y, ref, rtol=0, atol=1e-9 * max(1, N))
+
+
+def test_fwt_exact_integer_pin_f32dag():
+    # x in {-1,0,1}: every partial sum is an integer of magnitude <= N <= 2^24,
+    # so the fp32 DAG is exact and equals the int64 transform bit for bit.
+    N = 4096
+    x = inputs.fwt_ternary(9, N)
+    y32 = oracle.fwt_f32dag(x)
+    ref = _hadamard(N) @ x.astype(np.int64)
+    assert np.array_equal(y32.astype(np.int64), ref)
+    # involution: H(H x) = N x (exact, integers)
+    yy = oracle.fwt_f32dag(y32)
+    assert np.array_equal(yy.astype(np.int64), N * x.astype(np.int64))
+
+
+def test_fwt_delta_and_parseval():
+    N = 1 << 12
+    j = 1234
+    x = np.zeros(N, np.float32)
+    x[j] = 1
+    y = oracle.fwt_f64(x)
+    expect = np.array([(-1) ** bin(i & j).count("1") for i in range(N)], np.float64)
+    assert np.array_equal(y, expect)
+    x = inputs.fwt_x(4, 1 << 16)
+    y = oracle.fwt_f64(x)
+    assert abs(np.sum(y * y) / (len(x) * np.sum(x.astype(np.float64) ** 2)) - 1) < 1e-12
+    # the fp32 DAG stays within fp32 rounding of the fp64 transform
+    y32 = oracle.fwt_f32dag(x).astype(np.float64)
+    assert np.max(np.abs(y32 - y)) <= 16 * 2.0**-24 * np.sum(np.abs(x))
+
+
+# ---------------------------------------------------------------- PrefixSum / Reduction
+
+
+def test_prefixsum_closed_forms():
+    n = 1 << 17
+    ones = np.ones(n, np.uint32)
+    assert np.array_equal(oracle.prefixsum_u32(ones), np.arange(1, n + 1, dtype=np.uint32))
+    i = np.arange(n, dtype=np.uint64)
+    y = oracle.prefixsum_u32(i.astype(np.uint32))
+    assert np.array_equal(y, ((i * (i + 1) // 2) % 2**32).astype(np.uint32))
+
+
+def test_prefixsum_differencing_and_library():
+    x = inputs.prefixsum_x(3, 100003)
+    y = oracle.prefixsum_u32(x)
+    d = np.diff(y.astype(np.int64)) % 2**32
+    assert np.array_equal(d, x[1:].astype(np.int64)) and y[0] == x[0]
+    assert np.array_equal(y, np.cumsum(x, dtype=np.uint32))
+
+
+def test_reduction_closed_forms():
+    n = (1 << 20) + 37
+    assert oracle.reduction_u32(np.full(n, 7, np.uint32)) == 7 * n
+    i = np.arange(n, dtype=np.uint64)
+    x = (i % 65536).astype(np.uint32)
+    full, rem = divmod(n, 65536)
+    expect = full * (65535 * 65536 // 2) + rem * (rem - 1) // 2
+    assert oracle.reduction_u32(x) == expect
+    x = inputs.reduction_x(2, n)
+    assert oracle.reduction_u32(x) == int(np.sum(x, dtype=np.uint64))
+    assert oracle.reduction_u32(x) % 2**32 == int(oracle.prefixsum_u32(x)[-1])
+    assert oracle.reduction_u32(np.zeros(0, np.uint32)) == 0
+
+
+# ---------------------------------------------------------------- Transpose
+
+
+def test_transpose_index_coded_and_involution():
+    H, W = 96, 200
+    A = np.arange(H * W, dtype=np.uint32).reshape(H, W)
+    B = oracle.transpose_u32(A)
+    jj, ii = np.meshgrid(np.arange(H), np.arange(W))
+    assert np.array_equal(B, (jj * W + ii).astype(np.uint32))
+    assert np.array_equal(oracle.transpose_u32(B), A)
+    X = inputs.transpose_a(1, 33, 65)
+    assert np.array_equal(oracle.transpose_u32(X), X.T)
+
+
+# ---------------------------------------------------------------- Sobel
+
+
+def _sobel_scipy(I):
+    # independent: scipy correlate with the two 3x3 masks (rows = dy, cols = dx)
+    kx = np.array([[1, 2, 1], [0, 0, 0], [-1, -2, -1]])
+    ky = np.array([[1, 0, -1], [2, 0, -2], [1, 0, -1]])
+    out = np.zeros_like(I)
+    for c in range(4):
+        ch = I[:, :, c].astype(np.int64)
+        gx = scipy.ndimage.correlate(ch, kx, mode="constant")
+        gy = scipy.ndimage.correlate(ch, ky, mode="constant")
+        m = np.floor(np.sqrt((gx * gx + gy * gy).astype(np.float64))).astype(np.int64) // 2
+        o = np.minimum(255, m)
+        o[0, :] = o[-1, :] = 0
+        o[:, 0] = o[:, -1] = 0
+        out[:, :, c] = o
+    return out
+
+
+def test_sobel_vs_scipy_correlate():
+    I = inputs.sobel_image(3, 70, 131)
+    assert np.array_equal(oracle.sobel(I), _sobel_scipy(I))
+    rnd = (inputs.u32(8, 40 * 50 * 4) & 255).astype(np.uint8).reshape(40, 50, 4)
+    assert np.array_equal(oracle.sobel(rnd), _sobel_scipy(rnd))
+
+
+def test_sobel_closed_forms():
+    H, W = 16, 24
+    assert not oracle.sobel(np.full((H, W, 4), 77, np.uint8)).any()
+    for a in [1, 3, 9]:
+        x = np.arange(W)
+        I = np.broadcast_to((a * x)[None, :, None], (H, W, 4)).astype(np.uint8)
+        O = oracle.sobel(I)
+        assert np.all(O[1:-1, 1:-1] == min(255, 4 * a))
+        assert not O[0].any() and not O[:, 0].any()
+    I = np.zeros((H, W, 4), np.uint8)
+    I[5, 7, 2] = 200
+    O = oracle.sobel(I)
+    # diagonal neighbour sees |Gx| = |Gy| = 200 -> floor(sqrt(2)*200)//2 = 141
+    assert O[6, 8, 2] == math.isqrt(2 * 200 * 200) // 2
+    # side neighbour sees one gradient of 2*200 -> 200
+    assert O[5, 8, 2] == 200
+    assert O[5, 7, 2] == 0 and not O[:, :, [0, 1, 3]].any()
+
+
+# ---------------------------------------------------------------- FloydWarshall
+
+
+def test_floydwarshall_vs_dijkstra_and_invariants():
+    n = 96
+    Wm = inputs.floydwarshall_w(4, n)
+    D, P = oracle.floydwarshall(Wm)
+    for s in [0, 5, 50, 95]:
+        assert np.array_equal(D[s], oracle.dijkstra_row(Wm, s))
+    assert not np.diag(D).any()
+    assert np.all(D <= Wm)
+    # path invariant: P[i][j] = i  =>  D = W ; else D[i][j] = D[i][p] + D[p][j]
+    for i in range(n):
+        for j in range(n):
+            p = P[i, j]
+            if p == i:
+                assert D[i, j] == Wm[i, j]
+            else:
+                assert D[i, j] == D[i, p] + D[p, j]
+    # triangle inequality
+    for i, j, k in itertools.product(range(0, n, 7), repeat=3):
+        assert D[i, j] <= D[i, k] + D[k, j]
+
+
+def test_floydwarshall_brute_force_paths_tiny():
+    n = 6
+    Wm = inputs.floydwarshall_w(12, n)
+    D, _ = oracle.floydwarshall(Wm)
+    for i in range(n):
+        for j in range(n):
+            best = int(Wm[i, j]) if i != j else 0
+            others = [v for v in range(n) if v not in (i, j)]
+            for L in range(1, len(others) + 1):
+                for mid in itertools.permutations(others, L):
+                    path = (i,) + mid + (j,)
+                    best = min(best, sum(int(Wm[a, b]) for a, b in zip(path, path[1:])))
+            assert D[i, j] == best
+
+
+def test_floydwarshall_pred_is_last_strict_improvement():
+    # strict '<': with all-equal weights nothing ever improves -> P stays i
+    n = 10
+    Wm = np.full((n, n), 5, np.uint32)
+    np.fill_diagonal(Wm, 0)
+    D, P = oracle.floydwarshall(Wm)
+    assert np.array_equal(D, Wm)
+    assert np.array_equal(P, np.repeat(np.arange(n, dtype=np.uint32)[:, None], n, axis=1))
+
+
+# ---------------------------------------------------------------- DCT
+
+
+def test_dct_vs_scipy_and_closed_forms():
+    X = inputs.dct_x(5, 32, 48)
+    Y = oracle.dct8x8(X)
+    for by in range(4):
+        for bx in range(6):
+            blk = X[by * 8:(by + 1) * 8, bx * 8:(bx + 1) * 8].astype(np.float64)
+            ref = scipy.fft.dctn(blk, type=2, norm="ortho")
+            got = Y[by * 8:(by + 1) * 8, bx * 8:(bx + 1) * 8]
+            assert np.allclose(got, ref, rtol=0, atol=1e-10)
+            assert abs(np.linalg.norm(got) - np.linalg.norm(blk)) < 1e-9  # Parseval
+    c = 3.5
+    Yc = oracle.dct8x8(np.full((8, 8), c, np.float32))
+    assert abs(Yc[0, 0] - 8 * c) < 1e-12 and np.max(np.abs(Yc.ravel()[1:])) < 1e-12
+    # basis: X = C[u]^T C[v] -> Y = e_uv
+    u, v = 3, 5
+    Cm = np.array([[(math.sqrt(1 / 8) if a == 0 else 0.5) * math.cos((2 * x + 1) * a * math.pi / 16)
+                    for x in range(8)] for a in range(8)])
+    Xb = np.outer(Cm[u], Cm[v]).astype(np.float32)
+    Yb = oracle.dct8x8(Xb)
+    E = np.zeros((8, 8))
+    E[u, v] = 1
+    assert np.allclose(Yb, E, atol=1e-6)
+    B = oracle.dct8x8_absbound(X)
+    assert np.all(B >= np.abs(Y) - 1e-9)
+
+
+# ---------------------------------------------------------------- MatrixMultiplication
+
+
+def test_matmul_integer_exact_vs_numpy():
+    M, N, K = 64, 48, 96
+    A = inputs.matmul_bf16_int(1, M, K, stream=20)
+    Bt = inputs.matmul_bf16_int(1, N, K, stream=21)
+    Af = inputs.bf16_bits_to_f32(A).astype(np.int64)
+    Bf = inputs.bf16_bits_to_f32(Bt).astype(np.int64)
+    C = oracle.matmul_bf16(A, Bt)
+    assert np.array_equal(C.astype(np.int64), Af @ Bf.T)
+
+
+def test_matmul_normal_vs_numpy_and_freivalds_and_samples():
+    M, N, K = 40, 56, 72
+    A = inputs.matmul_bf16_normal(2, M, K, stream=22)
+    Bt = inputs.matmul_bf16_normal(2, N, K, stream=24)
+    Af = inputs.bf16_bits_to_f32(A).astype(np.float64)
+    Bf = inputs.bf16_bits_to_f32(Bt).astype(np.float64)
+    C = oracle.matmul_bf16(A, Bt)
+    assert np.allclose(C, Af @ Bf.T, rtol=0, atol=1e-12)
+    r = inputs.uniform_f32(3, N).astype(np.float64)
+    assert np.allclose(C @ r, Af @ (Bf.T @ r), atol=1e-9)
+    rows = np.array([0, 5, 39, 17], np.int64)
+    cols = np.array([0, 55, 3, 28], np.int64)
+    s, sa = oracle.matmul_bf16_sampled(A, Bt, rows, cols)
+    assert np.allclose(s, C[rows, cols], atol=1e-12)
+    assert np.allclose(sa, np.abs(Af[rows] * Bf[cols]).sum(1))
+
+
+def test_bf16_rounding_is_rne():
+    x = np.array([1.0, 1.0 + 2**-8, 1.0 + 3 * 2**-9, -2.5, 3.0e38], np.float32)
+    b = inputs.f32_to_bf16_bits(x)
+    back = inputs.bf16_bits_to_f32(b)
+    assert back[0] == 1.0 and back[1] == 1.0  # tie -> even
+    assert back[2] == 1.0 + 2**-7  # above half -> up
+    assert back[3] == -2.5
