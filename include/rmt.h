@@ -1,0 +1,191 @@
+/*
+ * rmt.h -- C ABI of librmt.so: compiler-style software Redundant
+ * MultiThreading (RMT) for GPGPU kernels on B200 (sm_100a).
+ *
+ * Method: Wadden et al., "Real-World Design and Evaluation of Compiler-Managed
+ * GPU Redundant Multithreading", ISCA 2014.  "P:NNN" = line NNN of the paper
+ * text (/root/reference/PAPER.md, not shipped).
+ *
+ *   - Each work-item is replicated; replicas run on replicated input
+ *     ("input replication", "producer and consumer").
+ *   - Every value that leaves the sphere of replication (SoR) -- a global store
+ *     -- is sent by the producer to the consumer, which compares the store's
+ *     address and value with its private copy and executes the store only if
+ *     they agree ("communicate both the address and value operands
+ *     of the store ... If the values differ, we have detected an error").
+ *   - Detection only; recovery is orthogonal.  A mismatch suppresses the
+ *     store and adds 1 to a device error counter (reading R-RMT1).
+ *
+ * Variants (rmt_variant_t):
+ *   RMT_NONE        the unprotected kernel (the baseline every slowdown is
+ *                   normalised to, "normalized to the runtime of the
+ *                   original kernel").
+ *   RMT_INTRA_SMEM  Intra-Group RMT +LDS: each CTA
+ *                   has twice the threads; redundant pairs are lanes (2i, 2i+1)
+ *                   of one warp (low bit of the thread id = replica);
+ *                   kernel-written shared memory is duplicated per replica; the
+ *                   producer (odd lane) passes (address, value) through a
+ *                   shared-memory mailbox, the consumer (even lane, Fig. 8
+ *                   P:845) compares and stores.
+ *   RMT_INTRA_REG   as INTRA_SMEM, but the exchange is register-level
+ *                   __shfl_xor_sync(.., 1) -- the B200 form of the paper's
+ *                   "FAST" swizzle communication (Fig. 8).
+ *   RMT_INTER_GROUP Inter-Group RMT: twice the CTAs; each CTA takes
+ *                   a ticket from a global counter, pair = ticket>>1,
+ *                   even ticket = producer; the producer passes store records
+ *                   through a bounded global-memory queue with release/acquire
+ *                   flags ("two-tiered locking system"; L2-coherent
+ *                   reads); the consumer compares and stores.
+ *
+ * Thread-safety: launches on different streams must use different workspaces.
+ * The fault-injection and ablation state is process-global (test/bench use).
+ */
+#ifndef RMT_H
+#define RMT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    RMT_NONE = 0,
+    RMT_INTRA_SMEM = 1,
+    RMT_INTRA_REG = 2,
+    RMT_INTER_GROUP = 3
+} rmt_variant_t;
+
+/* The AMD APP SDK-style kernels the paper evaluates (Fig. 2 axis
+ * P:237-255) plus MatrixTranspose (BASELINE.json configs[1]). */
+typedef enum {
+    RMT_K_BLACKSCHOLES = 0,
+    RMT_K_BINARYSEARCH = 1,
+    RMT_K_FWT = 2,
+    RMT_K_PREFIXSUM = 3,
+    RMT_K_REDUCTION = 4,
+    RMT_K_TRANSPOSE = 5,
+    RMT_K_SOBEL = 6,
+    RMT_K_FLOYDWARSHALL = 7,
+    RMT_K_DCT = 8,
+    RMT_K_MATMUL = 9,
+    RMT_K_COUNT = 10
+} rmt_kernel_t;
+
+typedef enum { RMT_F32 = 0, RMT_U32 = 1, RMT_U64 = 2, RMT_U8X4 = 3, RMT_BF16 = 4 } rmt_dtype_t;
+
+/* One caller-owned buffer.  ptr: device pointer for rmt_launch, host pointer
+ * (ideally pinned) for the host side of rmt_run_host.  numel counts elements of
+ * `dtype` (RMT_U8X4: one element = one 4-channel pixel = 4 bytes).  ptr must be
+ * 16-byte aligned. */
+typedef struct {
+    void* ptr;
+    int32_t dtype;
+    int64_t numel;
+} rmt_buf_t;
+
+/* Buffer schema per kernel (n = logical units; dims as listed, others 0):
+ *   BLACKSCHOLES  buf {r:F32[n], call:F32[n], put:F32[n]}           n = options
+ *   BINARYSEARCH  buf {A:U32[N] sorted, q:U32[Q], idx:U32[Q]}       n = Q, dims {N, Q}
+ *   FWT           buf {x:F32[N], y:F32[N]}                          n = N = 2^m
+ *   PREFIXSUM     buf {x:U32[n], y:U32[n]}  inclusive, mod 2^32     n
+ *   REDUCTION     buf {x:U32[n], s:U64[1]}                          n
+ *   TRANSPOSE     buf {A:U32|F32[H*W], B:same[W*H]}                 n = H*W, dims {H, W}, H%4 = W%4 = 0
+ *   SOBEL         buf {I:U8X4[H*W], O:U8X4[H*W]}                    n = H*W, dims {H, W}, W%4 = 0
+ *   FLOYDWARSHALL buf {D:U32[n*n] in/out, P:U32[n*n] out}           n = nodes, n%4 = 0
+ *   DCT           buf {X:F32[H*W], Y:F32[H*W]}                      n = H*W, dims {H, W}, H%8 = W%8 = 0
+ *   MATMUL        buf {A:BF16[M*K], Bt:BF16[N*K], C:F32[M*N]}       n = M*N, dims {M, N, K}
+ *                 C = A * Bt^T (both operands K-major); M%128 = N%128 = 0, K%64 = 0
+ * Vector-committed buffers must have < 2^30 elements.
+ */
+typedef struct {
+    rmt_buf_t buf[6];
+    int32_t nbuf;
+    int64_t dims[4];
+} rmt_bufs_t;
+
+/* Return codes (0 = success).  A detected mismatch is NOT an error code: it is
+ * counted in *err_count and the store is not committed. */
+#define RMT_OK 0
+#define RMT_EINVAL (-1)       /* bad kernel/variant id, dtype, numel, alignment or dims */
+#define RMT_EUNSUPPORTED (-2) /* kernel x variant x mode combination not built */
+#define RMT_EWORKSPACE (-3)   /* workspace NULL or smaller than rmt_workspace_size() */
+#define RMT_ECUDA (-4)        /* CUDA launch/copy error; detail in rmt_last_error() */
+#define RMT_ENODEV (-5)       /* no sm_100 device */
+
+/*
+ * rmt_launch -- run kernel `kernel` under RMT variant `variant`, asynchronously
+ * on `stream` (a cudaStream_t, passed as void*; NULL = legacy default stream).
+ *   bufs       device buffers per the schema above (caller-owned, not freed).
+ *   n          logical units (see schema).
+ *   err_count  device pointer to one u64; the library ADDS the number of
+ *              mismatching commits (caller zeroes it).  Never NULL.
+ *   workspace  device scratch of >= rmt_workspace_size(...) bytes, ZERO-FILLED
+ *              once at allocation; the library leaves it zero-equivalent after
+ *              every successful launch (self-resetting inter-group tickets and
+ *              queue; per-launch scratch is cleared with cudaMemsetAsync).
+ *              May be NULL iff rmt_workspace_size() returned 0.
+ * Graph-capturable (no host synchronisation, no allocation).
+ * Returns RMT_OK or a negative code; never throws across the ABI.
+ */
+int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n,
+               unsigned long long* err_count, void* workspace, size_t ws_bytes, void* stream);
+
+/* Bytes of workspace rmt_launch needs for this kernel/variant/size (dims as in
+ * the schema; may be NULL for 1-D kernels).  0 = none needed. */
+size_t rmt_workspace_size(int kernel, int variant, int64_t n, const int64_t* dims);
+
+/*
+ * rmt_run_host -- the end-to-end call: copy the kernel's INPUT buffers from
+ * `host` to `dev` (host->device), rmt_launch, copy the OUTPUT buffers back
+ * (device->host) and the error count into *err_host, then synchronise
+ * `stream`.  host/dev follow the same schema; dev buffers, err_dev and
+ * workspace are caller-owned device memory.  Returns as rmt_launch, or
+ * RMT_ECUDA on a copy/sync failure.  *h2d_bytes / *d2h_bytes (nullable)
+ * receive the bytes copied.
+ */
+int rmt_run_host(int kernel, int variant, const rmt_bufs_t* host, const rmt_bufs_t* dev, int64_t n,
+                 unsigned long long* err_host, unsigned long long* err_dev, void* workspace,
+                 size_t ws_bytes, void* stream, int64_t* h2d_bytes, int64_t* d2h_bytes);
+
+/* Fault injection (BASELINE.json north_star item (4)): arm ONE single-bit flip
+ * for subsequent launches until rmt_clear_faults().
+ *   replica  0|1 (intra: 0 = even lane = consumer, 1 = odd lane = producer;
+ *            inter: 0 = even ticket = producer, 1 = odd ticket = consumer;
+ *            none: must be 0)
+ *   site     RMT_SITE_* below
+ *   bit      0..31, flipped in the 32-bit word at that site
+ *   elem     kernel-specific logical element; >= 0
+ * Launches while armed run the FAULT instantiation of the kernel (the timed
+ * path never contains fault code). */
+#define RMT_SITE_LOAD 0       /* first loaded input word of elem */
+#define RMT_SITE_COMPUTE 1    /* a kernel-specific intermediate of elem */
+#define RMT_SITE_SMEM 2       /* a value read back from kernel-written shared memory */
+#define RMT_SITE_STORE_VAL 3  /* the stored value (first output buffer) of elem */
+#define RMT_SITE_STORE_ADDR 4 /* the store address: bit of the (vector) index */
+int rmt_inject_fault(int replica, int site, int bit, int64_t elem);
+int rmt_clear_faults(void);
+
+/* Cost attribution "as the paper does": 0 = full RMT,
+ * 1 = NOCOMM (both replicas run, no exchange/compare; the consumer stores its
+ * own value), 2 = INFLATE (run RMT_NONE with its per-SM residency reduced to
+ * that of the RMT variant by padding dynamic shared memory). */
+#define RMT_ABL_FULL 0
+#define RMT_ABL_NOCOMM 1
+#define RMT_ABL_INFLATE 2
+int rmt_set_ablation(int mode);
+
+/* Kernel launches the last rmt_launch issued (for the bench's launch count). */
+int rmt_last_launch_count(void);
+
+const char* rmt_strerror(int code);
+const char* rmt_last_error(void); /* thread-local detail of the last failure */
+const char* rmt_kernel_name(int kernel);
+const char* rmt_variant_name(int variant);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* RMT_H */

@@ -1,0 +1,133 @@
+// k_blackscholes.cu -- BlackScholes (Fig. 2 "BlkSch"; P:621
+// Intra <10% on HD 7790; P:809 Inter ~2x) under every RMT variant.
+//
+// Logical thread = 4 options (one 16-B vector): r[i..i+3] -> call, put.
+// Stores leaving the SoR: 2 vector commits per logical thread (call, put).
+// Arithmetic: fp32 with explicit-rounding intrinsics only, so every variant
+// executes the identical operation sequence (bit-identity rule).
+// Readings R-BS1 (APP-SDK input mapping) and R-BS2 (A&S CND) in DESIGN.md.
+#include "rmt_host.cuh"
+
+namespace rmt {
+namespace {
+
+constexpr int BL = 256;  // logical threads per CTA
+constexpr int VEC = 4;
+
+struct BsArgs {
+  const float* r;
+  float* call;
+  float* put;
+  unsigned n;
+};
+
+// A&S 26.2.17: tail = phi(|x|) k (a1 + k(a2 + k(a3 + k(a4 + k a5)))),
+// k = 1/(1 + 0.2316419|x|);  N(x) = 1 - tail (x >= 0), tail (x < 0).
+__device__ __forceinline__ void cnd_pair(float x, float& nx, float& nmx) {
+  float ax = fabsf(x);
+  float k = __frcp_rn(__fadd_rn(1.0f, __fmul_rn(0.2316419f, ax)));
+  float poly = __fmaf_rn(k, 1.330274429f, -1.821255978f);
+  poly = __fmaf_rn(k, poly, 1.781477937f);
+  poly = __fmaf_rn(k, poly, -0.356563782f);
+  poly = __fmaf_rn(k, poly, 0.319381530f);
+  poly = __fmul_rn(k, poly);
+  float phi = __fmul_rn(0.398942280401432678f, __expf(__fmul_rn(-0.5f, __fmul_rn(ax, ax))));
+  float tail = __fmul_rn(phi, poly);
+  float body = __fsub_rn(1.0f, tail);
+  nx = x >= 0.0f ? body : tail;
+  nmx = x >= 0.0f ? tail : body;
+}
+
+template <int V, int M>
+__device__ __forceinline__ void bs_option(const Rep<V, M>& rep, float r, long long elem, float& call, float& put) {
+  // R-BS1: S = K = 10r + 100(1-r), T = r + 10(1-r), R = .01r + .05(1-r), sigma = .01r + .1(1-r)
+  float omr = __fsub_rn(1.0f, r);
+  float S = __fadd_rn(__fmul_rn(10.0f, r), __fmul_rn(100.0f, omr));
+  float K = __fadd_rn(__fmul_rn(10.0f, r), __fmul_rn(100.0f, omr));
+  float T = __fadd_rn(r, __fmul_rn(10.0f, omr));
+  float R = __fadd_rn(__fmul_rn(0.01f, r), __fmul_rn(0.05f, omr));
+  float sig = __fadd_rn(__fmul_rn(0.01f, r), __fmul_rn(0.10f, omr));
+  float sT = __fmul_rn(sig, __fsqrt_rn(T));
+  // d1 = (ln(S/K) + (R + sigma^2/2) T) / (sigma sqrt T), d2 = d1 - sigma sqrt T
+  float drift = __fmul_rn(__fadd_rn(R, __fmul_rn(0.5f, __fmul_rn(sig, sig))), T);
+  float d1 = __fdiv_rn(__fadd_rn(__logf(__fdiv_rn(S, K)), drift), sT);
+  d1 = rep.faultf(SITE_COMPUTE, elem, d1);
+  float d2 = __fsub_rn(d1, sT);
+  float disc = __fmul_rn(K, __expf(-__fmul_rn(R, T)));
+  float n1, nm1, n2, nm2;
+  cnd_pair(d1, n1, nm1);
+  cnd_pair(d2, n2, nm2);
+  call = __fsub_rn(__fmul_rn(S, n1), __fmul_rn(disc, n2));
+  put = __fsub_rn(__fmul_rn(disc, nm2), __fmul_rn(S, nm1));
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) bs_kernel(BsArgs a, Ctx c) {
+  __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const unsigned i0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * VEC;
+  float r4[VEC];
+  unsigned mask = 0;
+  if (i0 + VEC <= a.n) {  // input replication: each replica loads its own copy
+    float4 v = __ldcs(reinterpret_cast<const float4*>(a.r + i0));
+    r4[0] = v.x; r4[1] = v.y; r4[2] = v.z; r4[3] = v.w;
+    mask = 0xFu;
+  } else {
+#pragma unroll
+    for (int k = 0; k < VEC; ++k) {
+      bool in = i0 + k < a.n;
+      r4[k] = in ? a.r[i0 + k] : 0.5f;
+      mask |= (in ? 1u : 0u) << k;
+    }
+  }
+  unsigned cv[VEC], pv[VEC];
+#pragma unroll
+  for (int k = 0; k < VEC; ++k) {
+    float rk = rep.faultf(SITE_LOAD, (long long)i0 + k, r4[k]);
+    float cl, pt;
+    bs_option(rep, rk, (long long)i0 + k, cl, pt);
+    cv[k] = __float_as_uint(cl);
+    pv[k] = __float_as_uint(pt);
+  }
+  auto store_to = [](float* base) {
+    return [base](unsigned idx, unsigned m, const unsigned* v) {
+      if (m == 0xFu) {
+        __stcs(reinterpret_cast<float4*>(base + idx),
+               make_float4(__uint_as_float(v[0]), __uint_as_float(v[1]), __uint_as_float(v[2]), __uint_as_float(v[3])));
+      } else {
+#pragma unroll
+        for (int k = 0; k < VEC; ++k)
+          if ((m >> k) & 1u) base[idx + k] = __uint_as_float(v[k]);
+      }
+    };
+  };
+  rep.template commit<VEC, 0>(mask, i0, cv, a.n, store_to(a.call));
+  rep.template commit<VEC, 1>(mask, i0, pv, a.n, store_to(a.put));
+  rep.finish();
+}
+
+}  // namespace
+
+int blackscholes_validate(const rmt_bufs_t* b, int64_t n) {
+  if (b->nbuf < 3 || n < 0 || n >= (1LL << 30) || !buf_ok(b->buf[0], RMT_F32, n) ||
+      !buf_ok(b->buf[1], RMT_F32, n) || !buf_ok(b->buf[2], RMT_F32, n)) {
+    set_error("blackscholes: expected {r,call,put} F32[n], n < 2^30, 16-B aligned");
+    return RMT_EINVAL;
+  }
+  return RMT_OK;
+}
+size_t blackscholes_scratch(int64_t, const int64_t*) { return 0; }
+int blackscholes_inter_warps(int64_t, const int64_t*) { return BL / 32; }
+
+int blackscholes_run(Launch& L) {
+  BsArgs a{(const float*)L.bufs->buf[0].ptr, (float*)L.bufs->buf[1].ptr, (float*)L.bufs->buf[2].ptr,
+           (unsigned)L.n};
+  unsigned G = (unsigned)((L.n + BL * VEC - 1) / (BL * VEC));
+  return dispatch(L.variant, L.mode, [&](auto vm) {
+    constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+    return launch_std<V>(L, bs_kernel<V, M>, bs_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "blackscholes");
+  });
+}
+
+}  // namespace rmt

@@ -1,0 +1,137 @@
+// k_reduction.cu -- Reduction ("R"; memory-bound, P:571-575
+// comm >1/2 of Intra overhead; "ghost groups").  u32 inputs, exact u64
+// sum (reading R-RED1).  Two launches, both under the variant:
+//   pass 1: each logical CTA reduces a grid-strided share of x and commits ONE
+//           u64 partial (the only store leaving the SoR per CTA);
+//   pass 2: one logical CTA sums the partials and commits s.
+#include "rmt_host.cuh"
+
+namespace rmt {
+namespace {
+
+constexpr int BL = 256;      // logical threads per CTA
+constexpr int UNROLL = 4;    // 16-B loads in flight per thread per iteration
+constexpr unsigned G1 = 148u * 8u;  // pass-1 logical CTAs (8 per SM)
+
+struct RedArgs {
+  const unsigned* x;
+  unsigned long long* out;  // pass 1: partials[G1]; pass 2: s
+  const unsigned long long* partials;
+  unsigned n;               // pass 1: elements; pass 2: number of partials
+};
+
+// Block-wide u64 sum within one replica (logical warps + duplicated smem).
+template <int V, int M>
+__device__ __forceinline__ unsigned long long block_sum(const Rep<V, M>& rep, unsigned long long s,
+                                                        unsigned long long* sm_warp) {
+  constexpr int LW = Rep<V, M>::LW;
+  constexpr int NLW = BL / LW;
+#pragma unroll
+  for (int m = LW / 2; m >= 1; m >>= 1) s += rep.lshfl_xor64(s, m);
+  const int lw = rep.ltid / LW;
+  if (rep.llane == 0) rep.sm(sm_warp, lw) = s;
+  __syncthreads();
+  unsigned long long t = 0;
+  if (rep.warp == 0) {
+    t = rep.llane < NLW ? rep.sm(sm_warp, rep.llane) : 0ull;
+    t = (unsigned long long)rep.fault(SITE_SMEM, (long long)rep.lblock * NLW + rep.llane, (unsigned)t) |
+        (t & 0xffffffff00000000ull);
+#pragma unroll
+    for (int m = LW / 2; m >= 1; m >>= 1) t += rep.lshfl_xor64(t, m);
+  }
+  return t;
+}
+
+__device__ __forceinline__ void store_u64(unsigned long long* base, unsigned idx, unsigned m, const unsigned* v) {
+  if (m == 3u) base[idx / 2] = (unsigned long long)v[0] | ((unsigned long long)v[1] << 32);
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) red_partial_kernel(RedArgs a, Ctx c) {
+  constexpr int DUP = Geom<V>::DUP;
+  __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
+  __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * DUP];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const unsigned T = (unsigned)c.nblocks * BL;  // logical threads in the grid
+  const unsigned gt = (unsigned)rep.lblock * BL + rep.ltid;
+  unsigned long long s = 0;
+  const unsigned nvec = a.n / 4;
+  for (unsigned base = 0; base < nvec; base += T * UNROLL) {
+    uint4 v[UNROLL];
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      unsigned vi = base + u * T + gt;
+      v[u] = vi < nvec ? __ldcs(reinterpret_cast<const uint4*>(a.x) + vi) : make_uint4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      unsigned e = (base + u * T + gt) * 4;
+      if constexpr (M == M_FAULT) {
+        v[u].x = rep.fault(SITE_LOAD, (long long)e, v[u].x);
+        v[u].y = rep.fault(SITE_LOAD, (long long)e + 1, v[u].y);
+        v[u].z = rep.fault(SITE_LOAD, (long long)e + 2, v[u].z);
+        v[u].w = rep.fault(SITE_LOAD, (long long)e + 3, v[u].w);
+      }
+      s += (unsigned long long)v[u].x + v[u].y + (unsigned long long)v[u].z + v[u].w;
+    }
+  }
+  for (unsigned e = nvec * 4 + gt; e < a.n; e += T) s += rep.fault(SITE_LOAD, (long long)e, a.x[e]);  // ragged tail
+  s = (s & 0xffffffff00000000ull) | rep.fault(SITE_COMPUTE, (long long)gt, (unsigned)s);
+  unsigned long long t = block_sum(rep, s, sm_warp);
+  if (rep.warp == 0) {  // warp-uniform: only warp 0 holds the CTA's store (P:809 ghost warps)
+    unsigned v[2] = {(unsigned)t, (unsigned)(t >> 32)};
+    unsigned mask = rep.llane == 0 ? 3u : 0u;
+    rep.template commit<2, 0>(mask, 2u * (unsigned)rep.lblock, v, 2u * (unsigned)c.nblocks,
+                              [&](unsigned idx, unsigned m, const unsigned* w) { store_u64(a.out, idx, m, w); });
+  }
+  rep.finish();
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) red_final_kernel(RedArgs a, Ctx c) {
+  constexpr int DUP = Geom<V>::DUP;
+  __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
+  __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * DUP];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  unsigned long long s = 0;
+  for (unsigned i = rep.ltid; i < a.n; i += BL) s += a.partials[i];
+  unsigned long long t = block_sum(rep, s, sm_warp);
+  if (rep.warp == 0) {
+    unsigned v[2] = {(unsigned)t, (unsigned)(t >> 32)};
+    unsigned mask = rep.llane == 0 ? 3u : 0u;
+    rep.template commit<2, 1>(mask, 0u, v, 2u,
+                              [&](unsigned idx, unsigned m, const unsigned* w) { store_u64(a.out, idx, m, w); });
+  }
+  rep.finish();
+}
+
+}  // namespace
+
+int reduction_validate(const rmt_bufs_t* b, int64_t n) {
+  if (b->nbuf < 2 || n < 0 || n >= (1LL << 32) - 16 || !buf_ok(b->buf[0], RMT_U32, n) ||
+      !buf_ok(b->buf[1], RMT_U64, 1)) {
+    set_error("reduction: expected {x:U32[n], s:U64[1]}");
+    return RMT_EINVAL;
+  }
+  return RMT_OK;
+}
+size_t reduction_scratch(int64_t, const int64_t*) { return G1 * sizeof(unsigned long long); }
+int reduction_inter_warps(int64_t, const int64_t*) { return BL / 32; }
+
+int reduction_run(Launch& L) {
+  unsigned long long* partials = (unsigned long long*)L.scratch;
+  RedArgs a1{(const unsigned*)L.bufs->buf[0].ptr, partials, nullptr, (unsigned)L.n};
+  RedArgs a2{nullptr, (unsigned long long*)L.bufs->buf[1].ptr, partials, G1};
+  return dispatch(L.variant, L.mode, [&](auto vm) {
+    constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+    int rc = launch_std<V>(L, red_partial_kernel<V, M>, red_partial_kernel<V_NONE, M_NORMAL>, G1, BL, 0, a1,
+                           "reduction/partial");
+    if (rc) return rc;
+    return launch_std<V>(L, red_final_kernel<V, M>, red_final_kernel<V_NONE, M_NORMAL>, 1, BL, 0, a2,
+                         "reduction/final");
+  });
+}
+
+}  // namespace rmt

@@ -1,0 +1,235 @@
+// rmt_abi.cu -- the extern "C" boundary declared in include/rmt.h.
+// Validation, workspace layout, fault/ablation state, dispatch to the
+// per-kernel launchers, and the host-buffer end-to-end call.
+#include <cuda_runtime.h>
+#include <stdio.h>
+
+#include <string>
+
+#include "rmt_host.cuh"
+
+namespace rmt {
+
+namespace {
+thread_local std::string g_err;
+FaultDesc g_fault = {0, 0, 0, 0, 0};
+bool g_armed = false;
+int g_ablation = RMT_ABL_FULL;
+thread_local int g_last_launches = 0;
+
+struct KEntry {
+  const char* name;
+  int (*validate)(const rmt_bufs_t*, int64_t);
+  size_t (*scratch)(int64_t, const int64_t*);
+  int (*inter_warps)(int64_t, const int64_t*);
+  int (*run)(Launch&);
+  int nin, in[2], nout, out[2];  // buffer roles for rmt_run_host
+};
+
+#define KE(name, nin, i0, i1, nout, o0, o1) \
+  {#name, name##_validate, name##_scratch, name##_inter_warps, name##_run, nin, {i0, i1}, nout, {o0, o1}}
+
+const KEntry kTable[RMT_K_COUNT] = {
+    KE(blackscholes, 1, 0, 0, 2, 1, 2),
+    KE(binarysearch, 2, 0, 1, 1, 2, 0),
+    KE(fwt, 1, 0, 0, 1, 1, 0),
+    KE(prefixsum, 1, 0, 0, 1, 1, 0),
+    KE(reduction, 1, 0, 0, 1, 1, 0),
+    KE(transpose, 1, 0, 0, 1, 1, 0),
+    KE(sobel, 1, 0, 0, 1, 1, 0),
+    KE(floydwarshall, 1, 0, 0, 2, 0, 1),
+    KE(dct, 1, 0, 0, 1, 1, 0),
+    KE(matmul, 2, 0, 1, 1, 2, 0),
+};
+
+const char* kVariantNames[4] = {"none", "intra_smem", "intra_reg", "inter_group"};
+
+int check_device() {
+  static int ok_dev = -1;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) {
+    set_error("cudaGetDevice failed (no CUDA device?)");
+    return RMT_ENODEV;
+  }
+  if (ok_dev == dev) return RMT_OK;
+  int major = 0;
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+  if (major != 10) {
+    set_error("librmt is built for sm_100a only; device major=" + std::to_string(major));
+    return RMT_ENODEV;
+  }
+  ok_dev = dev;
+  return RMT_OK;
+}
+
+size_t dtype_bytes(int dt) { return dt == RMT_U64 ? 8 : dt == RMT_BF16 ? 2 : 4; }
+
+size_t ws_size(int kernel, int variant, int64_t n, const int64_t* dims, size_t* inter_part) {
+  const KEntry& e = kTable[kernel];
+  size_t ip = 0;
+  if (variant == RMT_INTER_GROUP) ip = align_up(inter_bytes(e.inter_warps(n, dims)), 256);
+  if (inter_part) *inter_part = ip;
+  return ip + align_up(e.scratch(n, dims), 256);
+}
+}  // namespace
+
+void set_error(const std::string& msg) { g_err = msg; }
+
+int cuda_check(cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return RMT_OK;
+  set_error(std::string(what) + ": " + cudaGetErrorString(e));
+  return RMT_ECUDA;
+}
+
+}  // namespace rmt
+
+using namespace rmt;
+
+extern "C" {
+
+int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsigned long long* err_count,
+               void* workspace, size_t ws_bytes, void* stream) {
+  g_last_launches = 0;
+  if (kernel < 0 || kernel >= RMT_K_COUNT) { set_error("bad kernel id"); return RMT_EINVAL; }
+  if (variant < 0 || variant > RMT_INTER_GROUP) { set_error("bad variant id"); return RMT_EINVAL; }
+  if (!bufs || !err_count) { set_error("bufs and err_count must be non-NULL"); return RMT_EINVAL; }
+  int rc = check_device();
+  if (rc) return rc;
+  const KEntry& e = kTable[kernel];
+  rc = e.validate(bufs, n);
+  if (rc) return rc;
+  size_t inter_part = 0;
+  size_t need = ws_size(kernel, variant, n, bufs->dims, &inter_part);
+  if (need > 0 && (workspace == nullptr || ws_bytes < need)) {
+    set_error("workspace too small: need " + std::to_string(need) + " bytes");
+    return RMT_EWORKSPACE;
+  }
+  if (g_armed && variant == RMT_NONE && g_fault.replica != 0) {
+    set_error("variant none has a single replica: fault replica must be 0");
+    return RMT_EINVAL;
+  }
+  Launch L{};
+  L.kernel = kernel;
+  L.variant = variant;
+  L.mode = g_armed ? M_FAULT : (g_ablation == RMT_ABL_NOCOMM && variant != RMT_NONE ? M_NOCOMM : M_NORMAL);
+  L.inflate = !g_armed && g_ablation == RMT_ABL_INFLATE && variant != RMT_NONE;
+  L.bufs = bufs;
+  L.n = n;
+  L.stream = (cudaStream_t)stream;
+  L.ctx.err = err_count;
+  L.ctx.f = g_fault;
+  char* ws = (char*)workspace;
+  if (variant == RMT_INTER_GROUP) {
+    int W = e.inter_warps(n, bufs->dims);
+    size_t slots = (size_t)INTER_R * W * INTER_S;
+    L.ctx.ctrl = (unsigned*)ws;
+    L.ctx.flags = (unsigned*)(ws + CTRL_BYTES);
+    L.ctx.payload = (unsigned*)(ws + CTRL_BYTES + slots * 4);
+    L.ctx.R = INTER_R;
+    L.ctx.W = W;
+    L.ctx.S = INTER_S;
+  }
+  L.scratch = ws ? ws + inter_part : nullptr;
+  L.scratch_bytes = need - inter_part;
+  rc = e.run(L);
+  g_last_launches = L.launches;
+  if (rc == RMT_OK) rc = cuda_check(cudaGetLastError(), "kernel launch");
+  return rc;
+}
+
+size_t rmt_workspace_size(int kernel, int variant, int64_t n, const int64_t* dims) {
+  if (kernel < 0 || kernel >= RMT_K_COUNT || variant < 0 || variant > RMT_INTER_GROUP) return 0;
+  int64_t zero[4] = {0, 0, 0, 0};
+  return ws_size(kernel, variant, n, dims ? dims : zero, nullptr);
+}
+
+int rmt_run_host(int kernel, int variant, const rmt_bufs_t* host, const rmt_bufs_t* dev, int64_t n,
+                 unsigned long long* err_host, unsigned long long* err_dev, void* workspace, size_t ws_bytes,
+                 void* stream, int64_t* h2d_bytes, int64_t* d2h_bytes) {
+  if (kernel < 0 || kernel >= RMT_K_COUNT || !host || !dev || !err_host || !err_dev) {
+    set_error("rmt_run_host: bad arguments");
+    return RMT_EINVAL;
+  }
+  const KEntry& e = kTable[kernel];
+  cudaStream_t s = (cudaStream_t)stream;
+  int64_t hb = 0, db = 0;
+  int rc;
+  for (int i = 0; i < e.nin; ++i) {
+    const rmt_buf_t& h = host->buf[e.in[i]];
+    const rmt_buf_t& d = dev->buf[e.in[i]];
+    if (!h.ptr || h.numel != d.numel || h.dtype != d.dtype) { set_error("host/dev schema mismatch"); return RMT_EINVAL; }
+    size_t bytes = (size_t)h.numel * dtype_bytes(h.dtype);
+    if ((rc = cuda_check(cudaMemcpyAsync(d.ptr, h.ptr, bytes, cudaMemcpyHostToDevice, s), "H2D"))) return rc;
+    hb += (int64_t)bytes;
+  }
+  if ((rc = cuda_check(cudaMemsetAsync(err_dev, 0, sizeof(unsigned long long), s), "memset err"))) return rc;
+  rc = rmt_launch(kernel, variant, dev, n, err_dev, workspace, ws_bytes, stream);
+  if (rc) return rc;
+  for (int i = 0; i < e.nout; ++i) {
+    const rmt_buf_t& h = host->buf[e.out[i]];
+    const rmt_buf_t& d = dev->buf[e.out[i]];
+    if (!h.ptr || h.numel != d.numel) { set_error("host/dev schema mismatch"); return RMT_EINVAL; }
+    size_t bytes = (size_t)h.numel * dtype_bytes(h.dtype);
+    if ((rc = cuda_check(cudaMemcpyAsync(h.ptr, d.ptr, bytes, cudaMemcpyDeviceToHost, s), "D2H"))) return rc;
+    db += (int64_t)bytes;
+  }
+  if ((rc = cuda_check(cudaMemcpyAsync(err_host, err_dev, 8, cudaMemcpyDeviceToHost, s), "D2H err"))) return rc;
+  db += 8;
+  if ((rc = cuda_check(cudaStreamSynchronize(s), "stream sync"))) return rc;
+  if (h2d_bytes) *h2d_bytes = hb;
+  if (d2h_bytes) *d2h_bytes = db;
+  return RMT_OK;
+}
+
+int rmt_inject_fault(int replica, int site, int bit, int64_t elem) {
+  if (replica < 0 || replica > 1 || site < RMT_SITE_LOAD || site > RMT_SITE_STORE_ADDR || bit < 0 || bit > 31 ||
+      elem < 0) {
+    set_error("rmt_inject_fault: bad arguments");
+    return RMT_EINVAL;
+  }
+  g_fault.replica = replica;
+  g_fault.site = site;
+  g_fault.bit = bit;
+  g_fault.sid = 0;
+  g_fault.elem = elem;
+  g_armed = true;
+  return RMT_OK;
+}
+
+int rmt_clear_faults(void) {
+  g_armed = false;
+  g_fault = FaultDesc{0, 0, 0, 0, 0};
+  return RMT_OK;
+}
+
+int rmt_set_ablation(int mode) {
+  if (mode < RMT_ABL_FULL || mode > RMT_ABL_INFLATE) { set_error("bad ablation mode"); return RMT_EINVAL; }
+  g_ablation = mode;
+  return RMT_OK;
+}
+
+int rmt_last_launch_count(void) { return g_last_launches; }
+
+const char* rmt_strerror(int code) {
+  switch (code) {
+    case RMT_OK: return "ok";
+    case RMT_EINVAL: return "invalid argument";
+    case RMT_EUNSUPPORTED: return "unsupported kernel/variant";
+    case RMT_EWORKSPACE: return "workspace too small";
+    case RMT_ECUDA: return "CUDA error";
+    case RMT_ENODEV: return "no sm_100 device";
+  }
+  return "unknown error";
+}
+
+const char* rmt_last_error(void) { return g_err.c_str(); }
+
+const char* rmt_kernel_name(int kernel) {
+  return (kernel >= 0 && kernel < RMT_K_COUNT) ? kTable[kernel].name : "?";
+}
+
+const char* rmt_variant_name(int variant) {
+  return (variant >= 0 && variant <= RMT_INTER_GROUP) ? kVariantNames[variant] : "?";
+}
+
+}  // extern "C"

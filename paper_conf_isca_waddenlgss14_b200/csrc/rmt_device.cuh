@@ -1,0 +1,383 @@
+// rmt_device.cuh -- device-side RMT policies for sm_100a.
+//
+// One kernel body is written once and instantiated per variant V and mode MODE:
+//   V    = V_NONE | V_INTRA_SMEM | V_INTRA_REG | V_INTER      (include/rmt.h)
+//   MODE = M_NORMAL | M_FAULT (single-bit fault hooks compiled in) | M_NOCOMM
+//          (ablation: replicas run, no exchange/compare)
+//
+// What this header implements, with the paper passage each piece follows
+// ("P:NNN" = line of /root/reference/PAPER.md):
+//   * replica identity (P:205-207 intra: mask the low bit of the work-item id and
+//     keep it as the producer/consumer flag; P:679-689 inter: a global counter
+//     hands out new group ids, pair = id>>1, flag = id&1);
+//   * duplicated kernel-written shared memory for the intra variants
+//     (+LDS);
+//   * the convergent predicated commit (the producer communicates
+//     the address and value of every store leaving the SoR, the consumer
+//     compares with its private copy and executes the store only if equal),
+//     over three transports:
+//       - INTRA_SMEM: per-warp shared-memory mailbox ("local memory
+//         communication buffer");
+//       - INTRA_REG : __shfl_xor_sync(.., 1) between lanes 2i/2i+1 (the B200
+//         form of the GCN swizzle, Fig. 8: even lanes receive);
+//       - INTER     : bounded per-(pair, warp) queue in global memory with
+//         release/acquire flags (P:691 two-tier locking, P:693 L2-coherent reads),
+//         region ownership handed over by a per-region turn counter;
+//   * warp-aggregated error counting (one atomicAdd per warp with mismatches).
+//
+// Determinism rule for bodies: everything that feeds a commit must be computed
+// identically in every variant.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace rmt {
+
+constexpr int V_NONE = 0, V_INTRA_SMEM = 1, V_INTRA_REG = 2, V_INTER = 3;
+constexpr int M_NORMAL = 0, M_FAULT = 1, M_NOCOMM = 2;
+constexpr int SITE_LOAD = 0, SITE_COMPUTE = 1, SITE_SMEM = 2, SITE_STORE_VAL = 3, SITE_STORE_ADDR = 4;
+constexpr int MAXW = 4;               // max value words per commit
+constexpr int RING_WORDS = 1 + MAXW;  // key + values per lane per record
+constexpr int MBOX_WORDS = RING_WORDS * 16;  // intra_smem mailbox words per warp
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int CTRL_TURN = 64;         // ctrl[64 ..) = per-region turn counters
+constexpr unsigned long long WATCHDOG_CYCLES = 1ull << 32;  // ~2 s at 2 GHz
+
+struct FaultDesc {
+  int replica, site, bit, sid;
+  long long elem;
+};
+
+// Passed by value to every kernel.
+struct Ctx {
+  unsigned long long* err;  // device u64 error counter (caller-owned)
+  unsigned* ctrl;           // inter: [0] ticket [1] done [2] watchdog flag, [64..64+R) turn
+  unsigned* flags;          // inter: R*W*S slot flags (0 free, 1 full)
+  unsigned* payload;        // inter: R*W*S records of RING_WORDS*32 words
+  int R, W, S;              // inter queue geometry (regions, warps per CTA, slots)
+  int nblocks;              // logical CTAs in this launch
+  FaultDesc f;
+};
+
+// ---------------------------------------------------------------- PTX helpers
+__device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned ld_relaxed(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(unsigned* p, unsigned v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(unsigned* p, unsigned v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_relaxed64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void keep_alive(unsigned v) { asm volatile("" ::"r"(v)); }
+
+// Streaming global loads/stores (16 B).
+__device__ __forceinline__ uint4 ldg4(const void* p) { return __ldg(reinterpret_cast<const uint4*>(p)); }
+__device__ __forceinline__ void stg4(void* p, uint4 v) { *reinterpret_cast<uint4*>(p) = v; }
+__device__ __forceinline__ uint4 ldcs4(const void* p) { return __ldcs(reinterpret_cast<const uint4*>(p)); }
+__device__ __forceinline__ void stcs4(void* p, uint4 v) { __stcs(reinterpret_cast<uint4*>(p), v); }
+
+// Spin until *p == want (acquire), with back-off and a watchdog that converts a
+// hang (a fault that desynchronised a pair) into err+1 and a sticky flag.
+__device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, const Ctx& c) {
+  if (ld_acquire(p) == want) return true;
+  unsigned long long t0 = clock64();
+  unsigned ns = 32;
+  while (true) {
+    __nanosleep(ns);
+    if (ld_acquire(p) == want) return true;
+    if (ns < 512) ns <<= 1;
+    if (clock64() - t0 > WATCHDOG_CYCLES) {
+      atomicAdd(c.err, 1ull);
+      atomicExch(c.ctrl + 2, 1u);
+      return false;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- replica state
+template <int V, int MODE>
+struct Rep {
+  static constexpr bool INTRA = (V == V_INTRA_SMEM || V == V_INTRA_REG);
+  static constexpr bool INTER = (V == V_INTER);
+  static constexpr int DUP = INTRA ? 2 : 1;  // physical threads per logical thread
+  static constexpr int LW = 32 / DUP;        // logical warp width
+  static constexpr bool FAULT = (MODE == M_FAULT);
+  static constexpr bool NOCOMM = (MODE == M_NOCOMM);
+
+  const Ctx& c;
+  int r;          // replica id 0/1 (fault targeting)
+  bool consumer;  // the replica that executes stores (none: always)
+  int ltid;       // logical thread id within the logical CTA
+  int lblock;     // logical CTA id
+  int lane, warp, llane;
+  unsigned j;     // records this warp has committed (inter)
+  unsigned region, epoch;
+  unsigned* mbox;  // intra_smem: this warp's mailbox
+
+  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), region(0), epoch(0), mbox(nullptr) {}
+
+  // Must be called by every thread of the CTA, first thing (may __syncthreads).
+  // mbox_smem: MBOX_WORDS * (blockDim/32) words of shared memory (intra_smem only).
+  __device__ __forceinline__ void init(unsigned* mbox_smem = nullptr) {
+    lane = threadIdx.x & 31;
+    warp = threadIdx.x >> 5;
+    if constexpr (INTRA) {
+      r = threadIdx.x & 1;  // low bit of the id = producer/consumer flag
+      consumer = (r == 0);  // Fig. 8: even lanes receive -> consumer
+      ltid = threadIdx.x >> 1;
+      llane = lane >> 1;
+      lblock = blockIdx.x;
+      if constexpr (V == V_INTRA_SMEM) mbox = mbox_smem + warp * MBOX_WORDS;
+    } else if constexpr (INTER) {
+      __shared__ unsigned s_ticket;
+      if (threadIdx.x == 0) s_ticket = atomicAdd(c.ctrl, 1u);  // P:679-681 global counter
+      __syncthreads();
+      unsigned t = s_ticket;
+      lblock = (int)(t >> 1);  // P:681 mask the low bit -> identical pair
+      r = (int)(t & 1u);
+      consumer = (r == 1);     // even ticket = producer (reading R-RMT2)
+      ltid = threadIdx.x;
+      llane = lane;
+      region = (unsigned)lblock % (unsigned)c.R;
+      epoch = (unsigned)lblock / (unsigned)c.R;
+      if constexpr (!NOCOMM) {
+        // Exclusive ownership of the queue region: wait until the pair that used
+        // it before (lblock - R) has fully drained it (both roles wait).
+        if (threadIdx.x == 0 && epoch != 0) spin_until(c.ctrl + CTRL_TURN + region, epoch, c);
+        __syncthreads();
+      }
+    } else {
+      r = 0;
+      consumer = true;
+      ltid = threadIdx.x;
+      llane = lane;
+      lblock = blockIdx.x;
+    }
+  }
+
+  // Must be called by every thread of the CTA, last thing.
+  __device__ __forceinline__ void finish() {
+    if constexpr (INTER) {
+      __shared__ unsigned s_last;
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        if (consumer && !NOCOMM) st_release(c.ctrl + CTRL_TURN + region, epoch + 1);
+        __threadfence();
+        unsigned d = atomicAdd(c.ctrl + 1, 1u);
+        s_last = (d == 2u * (unsigned)c.nblocks - 1u);
+      }
+      __syncthreads();
+      if (s_last) {  // self-reset: the next launch starts from zero
+        __threadfence();
+        for (int i = threadIdx.x; i < c.R; i += blockDim.x) c.ctrl[CTRL_TURN + i] = 0;
+        if (threadIdx.x == 0) {
+          c.ctrl[0] = 0;
+          c.ctrl[1] = 0;
+        }
+      }
+    }
+  }
+
+  // ---- duplicated shared memory (+LDS): replica r owns its interleaved copy
+  template <class T>
+  __device__ __forceinline__ T& sm(T* base, int i) const {
+    if constexpr (INTRA) return base[2 * i + r];
+    else return base[i];
+  }
+
+  // ---- logical-warp shuffles (replica-private: lanes keep their role bit)
+  __device__ __forceinline__ unsigned lshfl_xor(unsigned v, int m) const {
+    return __shfl_xor_sync(FULL, v, m * DUP);
+  }
+  __device__ __forceinline__ unsigned lshfl_idx(unsigned v, int src) const {
+    return __shfl_sync(FULL, v, src * DUP + (INTRA ? r : 0));
+  }
+  // value of logical lane (llane - d); lanes with llane < d get their own value
+  __device__ __forceinline__ unsigned lshfl_up(unsigned v, int d) const {
+    unsigned u = __shfl_up_sync(FULL, v, d * DUP);
+    return llane >= d ? u : v;
+  }
+  __device__ __forceinline__ unsigned long long lshfl_xor64(unsigned long long v, int m) const {
+    return __shfl_xor_sync(FULL, v, m * DUP);
+  }
+  // logical ballot: bit l set iff logical lane l (this replica) has p
+  __device__ __forceinline__ unsigned lballot(bool p) const {
+    unsigned b = __ballot_sync(FULL, p);
+    if constexpr (INTRA) {
+      b >>= r;
+      unsigned o = 0;
+#pragma unroll
+      for (int i = 0; i < 16; ++i) o |= ((b >> (2 * i)) & 1u) << i;
+      return o;
+    } else {
+      return b;
+    }
+  }
+
+  // ---- fault hooks (compiled out unless MODE == M_FAULT)
+  __device__ __forceinline__ unsigned fault(int site, long long elem, unsigned x) const {
+    if constexpr (FAULT) {
+      if (c.f.site == site && c.f.elem == elem && c.f.replica == r) x ^= 1u << c.f.bit;
+    }
+    return x;
+  }
+  __device__ __forceinline__ float faultf(int site, long long elem, float x) const {
+    if constexpr (FAULT) return __uint_as_float(fault(site, elem, __float_as_uint(x)));
+    return x;
+  }
+
+  // ---- error aggregation: one atomic per warp that saw mismatches
+  __device__ __forceinline__ void count_mismatch(bool mism) const {
+    unsigned m = __ballot_sync(FULL, mism);
+    if (m != 0u && lane == __ffs(m) - 1) atomicAdd(c.err, (unsigned long long)__popc(m));
+  }
+
+  // ---- the commit.  Warp-collective: every lane of the warp must
+  // call it at the same program point (uniform control flow around commits).
+  //   mask  bit k set = word k is stored (a store instruction's predicate)
+  //   idx   element index of word 0 in the destination (multiple of NW if NW>1)
+  //   v     the NW 32-bit value words
+  //   limit destination element count (bounds for address faults in V_NONE)
+  //   store functor store(idx, mask, v) performing the actual global store(s)
+  //   SID   store-site id (faults on STORE_* sites target SID 0)
+  //   LIVE  liveness-critical store (other CTAs spin on it): on a mismatch the
+  //         consumer still stores its own value (reading R-RMT5) and counts it.
+  template <int NW, int SID = 0, bool LIVE = false, class Store>
+  __device__ __forceinline__ void commit(unsigned mask, unsigned idx, unsigned (&v)[NW], unsigned limit,
+                                         Store&& store) {
+    static_assert(NW >= 1 && NW <= MAXW, "commit width");
+    if constexpr (FAULT) {
+      if (c.f.sid == SID && c.f.replica == r && c.f.elem >= (long long)idx &&
+          c.f.elem < (long long)idx + NW) {
+        if (c.f.site == SITE_STORE_VAL) {
+          int w = (int)(c.f.elem - (long long)idx);
+#pragma unroll
+          for (int k = 0; k < NW; ++k)
+            if (k == w) v[k] ^= 1u << c.f.bit;
+        } else if (c.f.site == SITE_STORE_ADDR) {
+          idx ^= (NW == 1 ? 1u : (unsigned)NW) << c.f.bit;  // bit of the (vector) index
+        }
+      }
+    }
+    if constexpr (V == V_NONE) {
+      if (mask != 0u) {
+        if constexpr (FAULT) {
+          if (idx + NW > limit) return;  // a faulted address outside the buffer: dropped
+        }
+        store(idx, mask, v);
+      }
+      return;
+    } else {
+      if constexpr (NOCOMM) {
+        // Ablation: both replicas computed; no exchange, no compare.
+        if (consumer) {
+          if (mask != 0u) store(idx, mask, v);
+        } else {
+#pragma unroll
+          for (int k = 0; k < NW; ++k) keep_alive(v[k]);
+        }
+        if constexpr (INTER) ++j;
+        return;
+      }
+      // Record key: address + predicate in one word.
+      unsigned key;
+      if constexpr (NW == 1) key = mask ? idx : 0xffffffffu;
+      else key = mask ? (((idx / NW) << NW) | mask) : 0u;
+      unsigned pk = 0, pv[NW];
+      bool have = true;  // consumer got the producer's record
+      if constexpr (V == V_INTRA_REG) {
+        pk = __shfl_xor_sync(FULL, key, 1);
+#pragma unroll
+        for (int k = 0; k < NW; ++k) pv[k] = __shfl_xor_sync(FULL, v[k], 1);
+      } else if constexpr (V == V_INTRA_SMEM) {
+        const int slot = lane >> 1;
+        if (!consumer) {
+          mbox[slot] = key;
+#pragma unroll
+          for (int k = 0; k < NW; ++k) mbox[(1 + k) * 16 + slot] = v[k];
+        }
+        __syncwarp();
+        if (consumer) {
+          pk = mbox[slot];
+#pragma unroll
+          for (int k = 0; k < NW; ++k) pv[k] = mbox[(1 + k) * 16 + slot];
+        }
+        __syncwarp();
+      } else {  // V_INTER: per-(region, warp) queue of S records
+        const unsigned slot = j % (unsigned)c.S;
+        const size_t fi = ((size_t)region * c.W + warp) * c.S + slot;
+        unsigned* fl = c.flags + fi;
+        unsigned* pl = c.payload + fi * (RING_WORDS * 32);
+        if (!consumer) {
+          if (j >= (unsigned)c.S) {  // first S slots of a fresh region are free
+            if (lane == 0) spin_until(fl, 0u, c);
+            __syncwarp();
+          }
+          pl[lane] = key;
+#pragma unroll
+          for (int k = 0; k < NW; ++k) pl[(1 + k) * 32 + lane] = v[k];
+          __syncwarp();
+          if (lane == 0) st_release(fl, 1u);  // cumulative over the warp's payload stores
+        } else {
+          bool ok = true;
+          if (lane == 0) ok = spin_until(fl, 1u, c);
+          ok = __shfl_sync(FULL, ok, 0);
+          pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
+#pragma unroll
+          for (int k = 0; k < NW; ++k) pv[k] = ld_relaxed(pl + (1 + k) * 32 + lane);
+          __syncwarp();
+          if (lane == 0 && ok) st_release(fl, 0u);  // free the buffer
+          have = ok;
+        }
+        ++j;
+      }
+      bool mism = false;
+      if (consumer) {
+        bool eq = have && (pk == key);
+#pragma unroll
+        for (int k = 0; k < NW; ++k) eq = eq && (!((mask >> k) & 1u) || pv[k] == v[k]);
+        if (eq) {
+          if (mask != 0u) store(idx, mask, v);
+        } else {
+          mism = true;
+          if constexpr (LIVE) {
+            if (mask != 0u && idx + NW <= limit) store(idx, mask, v);
+          }
+        }
+      }
+      count_mismatch(mism);
+    }
+  }
+};
+
+// ---------------------------------------------------------------- launch geometry
+template <int V>
+struct Geom {
+  static constexpr int DUP = (V == V_INTRA_SMEM || V == V_INTRA_REG) ? 2 : 1;
+  static __host__ __device__ unsigned grid(unsigned lblocks) { return V == V_INTER ? 2u * lblocks : lblocks; }
+  static __host__ __device__ unsigned block(unsigned lthreads) { return lthreads * DUP; }
+};
+
+// Per-warp-mailbox shared memory words a kernel must reserve.
+template <int V>
+__host__ __device__ constexpr int mbox_words(int phys_threads) {
+  return V == V_INTRA_SMEM ? MBOX_WORDS * (phys_threads / 32) : 1;
+}
+
+}  // namespace rmt

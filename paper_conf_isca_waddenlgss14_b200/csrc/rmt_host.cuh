@@ -1,0 +1,139 @@
+// rmt_host.cuh -- host-side plumbing shared by the per-kernel launchers:
+// launch descriptor, variant x mode dispatch, workspace layout, error detail.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/rmt.h"
+#include "rmt_device.cuh"
+
+namespace rmt {
+
+// Inter-group queue geometry.
+constexpr int INTER_R = 1024;  // regions (> resident pairs, so a region is rarely waited for)
+constexpr int INTER_S = 8;     // slots (records in flight) per (region, warp)
+constexpr size_t CTRL_BYTES = (size_t)(CTRL_TURN + INTER_R) * 4;
+
+struct Launch {
+  int kernel, variant, mode;
+  bool inflate;               // RMT_ABL_INFLATE: run V_NONE with the RMT variant's residency
+  const rmt_bufs_t* bufs;
+  int64_t n;
+  Ctx ctx;                    // err + fault + inter queue pointers
+  char* scratch;              // kernel-specific scratch (after the inter queue)
+  size_t scratch_bytes;
+  cudaStream_t stream;
+  int launches;               // kernels launched (for rmt_last_launch_count)
+};
+
+void set_error(const std::string& msg);
+int cuda_check(cudaError_t e, const char* what);
+
+// Bytes of the inter-group queue for CTAs of `warps` physical warps.
+inline size_t inter_bytes(int warps) {
+  size_t slots = (size_t)INTER_R * warps * INTER_S;
+  return CTRL_BYTES + slots * 4 + slots * RING_WORDS * 32 * 4;
+}
+inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+template <int V_, int M_>
+struct VM {
+  static constexpr int V = V_;
+  static constexpr int M = M_;
+};
+
+// Call f(VM<V, M>{}) for the runtime (variant, mode).  M_NOCOMM only exists for
+// the RMT variants; the none variant ignores it.
+template <class F>
+int dispatch(int v, int m, F&& f) {
+  switch (v) {
+    case V_NONE:
+      return m == M_FAULT ? f(VM<V_NONE, M_FAULT>{}) : f(VM<V_NONE, M_NORMAL>{});
+    case V_INTRA_SMEM:
+      return m == M_FAULT ? f(VM<V_INTRA_SMEM, M_FAULT>{})
+           : m == M_NOCOMM ? f(VM<V_INTRA_SMEM, M_NOCOMM>{})
+                           : f(VM<V_INTRA_SMEM, M_NORMAL>{});
+    case V_INTRA_REG:
+      return m == M_FAULT ? f(VM<V_INTRA_REG, M_FAULT>{})
+           : m == M_NOCOMM ? f(VM<V_INTRA_REG, M_NOCOMM>{})
+                           : f(VM<V_INTRA_REG, M_NORMAL>{});
+    case V_INTER:
+      return m == M_FAULT ? f(VM<V_INTER, M_FAULT>{})
+           : m == M_NOCOMM ? f(VM<V_INTER, M_NOCOMM>{})
+                           : f(VM<V_INTER, M_NORMAL>{});
+  }
+  return RMT_EINVAL;
+}
+
+// Checks shared by the per-kernel validators.
+inline bool buf_ok(const rmt_buf_t& b, int dtype, int64_t numel) {
+  return (b.ptr != nullptr || numel == 0) && b.dtype == dtype && b.numel == numel && ((uintptr_t)b.ptr % 16) == 0;
+}
+
+// ---- per-kernel entry points (one translation unit each)
+#define RMT_DECLARE_KERNEL(name)                                              \
+  int name##_validate(const rmt_bufs_t* b, int64_t n);                        \
+  size_t name##_scratch(int64_t n, const int64_t* dims);                      \
+  int name##_inter_warps(int64_t n, const int64_t* dims);                     \
+  int name##_run(Launch& L);
+
+RMT_DECLARE_KERNEL(blackscholes)
+RMT_DECLARE_KERNEL(binarysearch)
+RMT_DECLARE_KERNEL(fwt)
+RMT_DECLARE_KERNEL(prefixsum)
+RMT_DECLARE_KERNEL(reduction)
+RMT_DECLARE_KERNEL(transpose)
+RMT_DECLARE_KERNEL(sobel)
+RMT_DECLARE_KERNEL(floydwarshall)
+RMT_DECLARE_KERNEL(dct)
+RMT_DECLARE_KERNEL(matmul)
+
+}  // namespace rmt
+
+namespace rmt {
+
+// Smallest dynamic-smem padding that brings kernel `kn` (block bn, smem sn) to
+// at most `target` CTAs per SM.
+template <class K>
+size_t pad_for_occupancy(K kn, int bn, size_t sn, int target) {
+  int occ = 0;
+  for (size_t extra = 0; extra + sn <= 227 * 1024; extra += 1024) {
+    if (sn + extra > 48 * 1024)
+      cudaFuncSetAttribute(kn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sn + extra));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kn, bn, sn + extra);
+    if (occ <= target) return extra;
+  }
+  return 0;
+}
+
+// Standard launch of one RMT kernel instance: logical grid G of BL-thread
+// logical CTAs, `smem` dynamic shared bytes.  kr = the variant's kernel,
+// kn = the V_NONE kernel (used for the INFLATE ablation).
+template <int V, class Args>
+int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned G, int BL, size_t smem,
+               const Args& a, const char* what) {
+  if (G == 0) return RMT_OK;
+  Ctx c = L.ctx;
+  c.nblocks = (int)G;
+  if (L.inflate) {
+    // run the original kernel with the RMT version's per-SM footprint
+    // (inter: the footprint of two RMT groups).
+    int occ = 0;
+    if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kr, Geom<V>::block(BL), smem);
+    int target = V == V_INTER ? (occ / 2 > 1 ? occ / 2 : 1) : (occ > 1 ? occ : 1);
+    size_t pad = pad_for_occupancy(kn, BL, smem, target);
+    if (smem + pad > 48 * 1024)
+      cudaFuncSetAttribute(kn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem + pad));
+    kn<<<G, BL, smem + pad, L.stream>>>(a, c);
+  } else {
+    if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    kr<<<Geom<V>::grid(G), Geom<V>::block(BL), smem, L.stream>>>(a, c);
+  }
+  L.launches += 1;
+  return cuda_check(cudaGetLastError(), what);
+}
+
+}  // namespace rmt

@@ -1,0 +1,87 @@
+"""GPU parity (-m gpu): CUDA path vs oracle, RMT variants vs the unprotected
+kernel (bitwise), determinism, and single-bit fault detection, all through the
+C ABI (librmt.so)."""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_isca_waddenlgss14_b200 import rmt
+from cases import small_cases
+from helpers import VARIANTS, run
+
+pytestmark = pytest.mark.gpu
+
+CASES = small_cases()
+IDS = [f"{c.kernel}-{c.n}" for c in CASES]
+
+
+def _run_case(case, variant):
+    b = case.buffers()
+    err = run(case.kernel, variant, b, case.n, case.dims)
+    return err, case.outputs(b)
+
+
+@pytest.mark.parametrize("case", CASES, ids=IDS)
+def test_none_matches_oracle(case):
+    err, outs = _run_case(case, "none")
+    assert err == 0
+    case.check(outs)
+
+
+@pytest.mark.parametrize("variant", rmt.RMT_VARIANTS)
+@pytest.mark.parametrize("case", CASES, ids=IDS)
+def test_variant_bit_identical_to_none(case, variant):
+    _, ref = _run_case(case, "none")
+    for _ in range(2):  # determinism: two runs
+        err, outs = _run_case(case, variant)
+        assert err == 0, f"{variant}: {err} false alarms"
+        for a, b in zip(outs, ref):
+            assert np.array_equal(a, b), f"{variant} output differs from none"
+
+
+FAULT_CASES = [c for c in CASES if c.n >= 1000]
+
+
+@pytest.mark.parametrize("variant", rmt.RMT_VARIANTS)
+@pytest.mark.parametrize("replica", [0, 1])
+@pytest.mark.parametrize("case", FAULT_CASES, ids=[f"{c.kernel}-{c.n}" for c in FAULT_CASES])
+def test_store_value_fault_detected(case, replica, variant):
+    """A flipped store value in one replica: exactly one mismatching commit, the
+    faulted word is not committed (sentinel kept), everything else is clean."""
+    _, ref = _run_case(case, "none")
+    bi, ne = case.out_elems()
+    rng = np.random.default_rng(case.n + replica)
+    e = int(rng.integers(0, ne))
+    bit = int(rng.integers(0, 32))
+    rmt.inject_fault(replica, "store_val", bit, e)
+    try:
+        err, outs = _run_case(case, variant)
+    finally:
+        rmt.clear_faults()
+    assert err == 1
+    if case.kernel == "reduction":
+        return  # the uncommitted word is a per-CTA partial in the workspace
+    o = outs[0].reshape(-1)
+    r = ref[0].reshape(-1)
+    grp = case.commit_group(e)
+    assert np.all(o[grp] == 0xFFFFFFFF), "faulted commit must not be stored"
+    mask = np.ones(o.size, bool)
+    mask[grp] = False
+    assert np.array_equal(o[mask], r[mask])
+    for a, b in zip(outs[1:], ref[1:]):
+        assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("case", FAULT_CASES, ids=[f"{c.kernel}-{c.n}" for c in FAULT_CASES])
+def test_fault_is_live_in_none(case):
+    """Liveness control: the same flip in the unprotected kernel corrupts the output."""
+    _, ref = _run_case(case, "none")
+    bi, ne = case.out_elems()
+    e = ne // 2
+    rmt.inject_fault(0, "store_val", 5, e)
+    try:
+        err, outs = _run_case(case, "none")
+    finally:
+        rmt.clear_faults()
+    assert err == 0
+    assert any(not np.array_equal(a, b) for a, b in zip(outs, ref))
