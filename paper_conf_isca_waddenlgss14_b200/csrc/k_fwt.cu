@@ -1,0 +1,198 @@
+// k_fwt.cu -- FastWalshTransform ("FWT"; memory-bound, Intra
+// <=10% on HD 7790; an Inter outlier >7x).
+// y = H_N x, natural order, unnormalised (reading R-FWT1): log2 N radix-2
+// stages h = 1, 2, ..., N/2, butterfly (a, b) -> (a + b, a - b).
+//
+// B200 design: the stages are fused into passes over 4096-element tiles staged
+// in (duplicated, +LDS) shared memory.  Pass 1 runs stages 0..11 on contiguous
+// tiles; later passes run up to 7 stages on tiles of 2^b strided rows x 2^c
+// contiguous columns (c >= 5 -> 128-B coalesced rows).  Inside a pass, stages
+// run as register rounds of up to 4 stages (16 elements per thread).  The
+// butterfly DAG -- hence every fp32 rounding -- is fixed by the stage order
+// alone, so every variant and every fusion is bit-identical to the fp32-DAG
+// oracle (reading R-FWT2).  HBM traffic: 8 B/elem per pass.
+#include "rmt_host.cuh"
+
+namespace rmt {
+namespace {
+
+constexpr int BL = 256;
+constexpr int TB_MAX = 12;
+constexpr int TE_MAX = 1 << TB_MAX;
+constexpr int SM_WORDS = TE_MAX + TE_MAX / 32;  // pad32 swizzle: <=2-way conflicts for all rounds
+
+__device__ __forceinline__ int phys(int e) { return e + (e >> 5); }
+
+struct FwtArgs {
+  const float* src;
+  float* dst;
+  unsigned N;
+  int tb;  // tile bits (TE = 2^tb)
+  int s0;  // first stage (bit position in the global index)
+  int b;   // stages in this pass
+  int c;   // contiguous column bits in the tile (0 for pass 1)
+};
+
+__device__ __forceinline__ unsigned gindex(const FwtArgs& a, unsigned tile, unsigned e) {
+  if (a.s0 == 0) return (tile << a.tb) | e;
+  const unsigned col = e & ((1u << a.c) - 1u), st = e >> a.c;
+  const int midb = a.s0 - a.c;
+  const unsigned mid = tile & ((1u << midb) - 1u), hi = tile >> midb;
+  return (hi << (a.s0 + a.b)) | (st << a.s0) | (mid << a.c) | col;
+}
+
+// One register round: NB consecutive stages at tile-bit q on groups of 2^NB.
+template <int NB, class R>
+__device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int te, const FwtArgs& a, unsigned tileid,
+                                          int round_no) {
+  constexpr int G = 1 << NB;
+  const int groups = te >> NB;
+  for (int gi = rep.ltid; gi < groups; gi += BL) {
+    const int lowmask = (1 << q) - 1;
+    const int ebase = (gi & lowmask) | ((gi >> q) << (q + NB));
+    float v[G];
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      v[k] = rep.sm(tile, phys(ebase | (k << q)));
+      if constexpr (R::FAULT) {
+        if (a.s0 == 0 && round_no == 1)
+          v[k] = rep.faultf(SITE_SMEM, (long long)gindex(a, tileid, ebase | (k << q)), v[k]);
+      }
+    }
+#pragma unroll
+    for (int s = 0; s < NB; ++s) {
+      const int h = 1 << s;
+#pragma unroll
+      for (int k = 0; k < G; ++k) {
+        if (k & h) continue;
+        const float x0 = v[k], x1 = v[k + h];
+        v[k] = __fadd_rn(x0, x1);
+        v[k + h] = __fsub_rn(x0, x1);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      if constexpr (R::FAULT) {
+        if (a.s0 == 0 && round_no == 0)
+          v[k] = rep.faultf(SITE_COMPUTE, (long long)gindex(a, tileid, ebase | (k << q)), v[k]);
+      }
+      rep.sm(tile, phys(ebase | (k << q))) = v[k];
+    }
+  }
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c) {
+  constexpr int DUP = Geom<V>::DUP;
+  __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
+  __shared__ float tile[SM_WORDS * DUP];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const unsigned tileid = (unsigned)rep.lblock;
+  const int te = 1 << a.tb;
+  // load: 16-B vectors, contiguous in both the tile and global memory
+  for (int e0 = 4 * rep.ltid; e0 < te; e0 += 4 * BL) {
+    const unsigned g = gindex(a, tileid, (unsigned)e0);
+    float w[4];
+    if (te >= 4) {
+      float4 f = *reinterpret_cast<const float4*>(a.src + g);
+      w[0] = f.x; w[1] = f.y; w[2] = f.z; w[3] = f.w;
+    } else {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) w[k] = e0 + k < te ? a.src[g + k] : 0.0f;
+    }
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      if (e0 + k < te) {
+        float x = w[k];
+        if constexpr (M == M_FAULT) {
+          if (a.s0 == 0) x = rep.faultf(SITE_LOAD, (long long)g + k, x);
+        }
+        rep.sm(tile, phys(e0 + k)) = x;
+      }
+    }
+  }
+  __syncthreads();
+  // stages [s0, s0 + b) live at tile bits [c, c + b); rounds of <= 4 stages
+  int round_no = 0;
+  for (int q = a.c; q < a.c + a.b; q += 4, ++round_no) {
+    const int nb = min(4, a.c + a.b - q);
+    switch (nb) {
+      case 4: fwt_round<4>(rep, tile, q, te, a, tileid, round_no); break;
+      case 3: fwt_round<3>(rep, tile, q, te, a, tileid, round_no); break;
+      case 2: fwt_round<2>(rep, tile, q, te, a, tileid, round_no); break;
+      default: fwt_round<1>(rep, tile, q, te, a, tileid, round_no); break;
+    }
+    __syncthreads();
+  }
+  // store: one vector commit per 4 elements
+#pragma unroll 1
+  for (int it = 0; it < TE_MAX / (4 * BL); ++it) {
+    const int e0 = 4 * rep.ltid + it * 4 * BL;
+    unsigned w[4];
+    unsigned mask = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const bool in = e0 + k < te;
+      w[k] = in ? __float_as_uint(rep.sm(tile, phys(e0 + k))) : 0u;
+      mask |= (in ? 1u : 0u) << k;
+    }
+    const unsigned g = e0 < te ? gindex(a, tileid, (unsigned)e0) : 0u;
+    rep.template commit<4, 0>(mask, g, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
+      if (m == 0xFu)
+        *reinterpret_cast<float4*>(a.dst + idx) =
+            make_float4(__uint_as_float(x[0]), __uint_as_float(x[1]), __uint_as_float(x[2]), __uint_as_float(x[3]));
+      else
+        for (int k = 0; k < 4; ++k)
+          if ((m >> k) & 1u) a.dst[idx + k] = __uint_as_float(x[k]);
+    });
+  }
+  rep.finish();
+}
+
+int log2u(int64_t n) {
+  int m = 0;
+  while ((1LL << m) < n) ++m;
+  return m;
+}
+
+}  // namespace
+
+int fwt_validate(const rmt_bufs_t* b, int64_t n) {
+  if (b->nbuf < 2 || n < 1 || n > (1LL << 30) || (n & (n - 1)) || !buf_ok(b->buf[0], RMT_F32, n) ||
+      !buf_ok(b->buf[1], RMT_F32, n)) {
+    set_error("fwt: expected {x,y} F32[N], N a power of two in [1, 2^30]");
+    return RMT_EINVAL;
+  }
+  return RMT_OK;
+}
+size_t fwt_scratch(int64_t, const int64_t*) { return 0; }
+int fwt_inter_warps(int64_t, const int64_t*) { return BL / 32; }
+
+int fwt_run(Launch& L) {
+  const int m = log2u(L.n);
+  const int tb = m < TB_MAX ? m : TB_MAX;
+  const float* x = (const float*)L.bufs->buf[0].ptr;
+  float* y = (float*)L.bufs->buf[1].ptr;
+  return dispatch(L.variant, L.mode, [&](auto vm) {
+    constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+    const unsigned tiles = (unsigned)(L.n >> tb);
+    // STORE_* fault sites target the final pass (the stored y); LOAD/COMPUTE/SMEM
+    // sites target pass 1 (gated in the kernel by s0 == 0).
+    const int sid = L.ctx.f.sid;
+    L.ctx.f.sid = (tb < m) ? -1 : sid;
+    FwtArgs a{x, y, (unsigned)L.n, tb, 0, tb, 0};
+    int rc = launch_std<V>(L, fwt_kernel<V, M>, fwt_kernel<V_NONE, M_NORMAL>, tiles, BL, 0, a, "fwt/pass1");
+    for (int s = tb; s < m && rc == RMT_OK; ) {  // strided passes, in place on y
+      const int b = (m - s) < 7 ? (m - s) : 7;
+      L.ctx.f.sid = (s + b < m) ? -1 : sid;
+      FwtArgs p{y, y, (unsigned)L.n, TB_MAX, s, b, TB_MAX - b};
+      rc = launch_std<V>(L, fwt_kernel<V, M>, fwt_kernel<V_NONE, M_NORMAL>, tiles, BL, 0, p, "fwt/pass");
+      s += b;
+    }
+    L.ctx.f.sid = sid;
+    return rc;
+  });
+}
+
+}  // namespace rmt

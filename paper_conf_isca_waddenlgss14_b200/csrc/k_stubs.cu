@@ -10,10 +10,6 @@ namespace rmt {
     set_error(#name ": not implemented yet");                                            \
     return RMT_EUNSUPPORTED;                                                             \
   }
-RMT_STUB(binarysearch)
-RMT_STUB(fwt)
-RMT_STUB(prefixsum)
-RMT_STUB(sobel)
 RMT_STUB(floydwarshall)
 RMT_STUB(dct)
 RMT_STUB(matmul)

@@ -94,7 +94,9 @@ __device__ __forceinline__ void stcs4(void* p, uint4 v) { __stcs(reinterpret_cas
 
 // Spin until *p == want (acquire), with back-off and a watchdog that converts a
 // hang (a fault that desynchronised a pair) into err+1 and a sticky flag.
-__device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, const Ctx& c) {
+// Every thread that will touch the guarded data must do its own acquire: a lane
+// of a (possibly diverged) warp is not ordered after another lane's acquire.
+__device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, const Ctx& c, bool count = true) {
   if (ld_acquire(p) == want) return true;
   unsigned long long t0 = clock64();
   unsigned ns = 32;
@@ -103,8 +105,10 @@ __device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, con
     if (ld_acquire(p) == want) return true;
     if (ns < 512) ns <<= 1;
     if (clock64() - t0 > WATCHDOG_CYCLES) {
-      atomicAdd(c.err, 1ull);
-      atomicExch(c.ctrl + 2, 1u);
+      if (count) {
+        atomicAdd(c.err, 1ull);
+        atomicExch(c.ctrl + 2, 1u);
+      }
       return false;
     }
   }
@@ -325,27 +329,26 @@ struct Rep {
         unsigned* fl = c.flags + fi;
         unsigned* pl = c.payload + fi * (RING_WORDS * 32);
         if (!consumer) {
-          if (j >= (unsigned)c.S) {  // first S slots of a fresh region are free
-            if (lane == 0) spin_until(fl, 0u, c);
-            __syncwarp();
-          }
+          // wait for a free buffer; the first S slots of a fresh region are free
+          if (j >= (unsigned)c.S) spin_until(fl, 0u, c, lane == 0);
           pl[lane] = key;
 #pragma unroll
           for (int k = 0; k < NW; ++k) pl[(1 + k) * 32 + lane] = v[k];
+          // Every lane fences its own payload stores (a release by lane 0 alone
+          // does not order the other lanes' in-flight stores), then lane 0
+          // signals "ready" ("signals the work-item in the consumer").
+          __threadfence();
           __syncwarp();
-          if (lane == 0) st_release(fl, 1u);  // cumulative over the warp's payload stores
+          if (lane == 0) st_relaxed(fl, 1u);
         } else {
-          bool ok = true;
-          if (lane == 0) ok = spin_until(fl, 1u, c);
-          ok = __shfl_sync(FULL, ok, 0);
+          const bool ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
           pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
 #pragma unroll
           for (int k = 0; k < NW; ++k) pv[k] = ld_relaxed(pl + (1 + k) * 32 + lane);
-          __syncwarp();
-          if (lane == 0 && ok) st_release(fl, 0u);  // free the buffer
           have = ok;
+          // the buffer is freed only after every lane has consumed its words
+          // (below, after the compare's warp ballot)
         }
-        ++j;
       }
       bool mism = false;
       if (consumer) {
@@ -361,7 +364,16 @@ struct Rep {
           }
         }
       }
-      count_mismatch(mism);
+      // warp ballot over the compare results: completes every lane's loads
+      const unsigned mb = __ballot_sync(FULL, mism);
+      if (mb != 0u && lane == __ffs(mb) - 1) atomicAdd(c.err, (unsigned long long)__popc(mb));
+      if constexpr (INTER) {
+        if (consumer && lane == 0 && have) {
+          const size_t fi = ((size_t)region * c.W + warp) * c.S + (j % (unsigned)c.S);
+          st_release(c.flags + fi, 0u);  // free the buffer
+        }
+        ++j;
+      }
     }
   }
 };

@@ -1,0 +1,145 @@
+"""Benchmark workloads: BASELINE.json configs as named presets.
+
+A Job is one kernel at one size: host inputs (numpy, from the seeded
+generators in inputs.py), device buffers in schema order, and the kernel's
+algorithmic HBM bytes per launch (SURVEY 8(d) / DESIGN.md "Roofline").  No
+method arithmetic lives here.  Shards: rank r of G takes rows/elements
+[r*n, (r+1)*n) of the global index space (weak scaling: fixed per-GPU size).
+"""
+from __future__ import annotations
+
+import dataclasses
+
+import numpy as np
+import torch
+
+from . import inputs
+
+MiB = 1 << 20
+
+
+@dataclasses.dataclass
+class Job:
+    kernel: str
+    n: int
+    dims: tuple
+    host_in: list          # numpy arrays, schema order, None for outputs
+    out_shapes: list       # (index, nbytes) of output buffers
+    alg_bytes: int         # algorithmic HBM bytes per launch
+    unit: str              # what n counts
+    bound: str = "hbm"
+    note: str = ""
+    dev: list | None = None
+
+    def device_buffers(self):
+        """Allocate device buffers once (inputs copied, outputs zeroed)."""
+        if self.dev is None:
+            bufs = []
+            for i, h in enumerate(self.host_in):
+                if h is not None:
+                    bufs.append(_to_dev(h))
+                else:
+                    nbytes = dict(self.out_shapes)[i]
+                    bufs.append(torch.zeros(max(nbytes // 4, 4), dtype=torch.int32, device="cuda")[: nbytes // 4])
+            self.dev = bufs
+        return self.dev
+
+    def pinned_host(self):
+        """Pinned host buffers (inputs filled, outputs empty) for the end-to-end call."""
+        hb = []
+        for i, h in enumerate(self.host_in):
+            if h is not None:
+                t = torch.from_numpy(_as_signed(h).reshape(-1).copy()).pin_memory()
+            else:
+                t = torch.empty(dict(self.out_shapes)[i] // 4, dtype=torch.int32).pin_memory()
+            hb.append(t)
+        return hb
+
+
+def _as_signed(a: np.ndarray) -> np.ndarray:
+    m = {np.dtype(np.uint32): np.int32, np.dtype(np.uint16): np.int16, np.dtype(np.uint8): np.uint8,
+         np.dtype(np.uint64): np.int64}
+    a = np.ascontiguousarray(a)
+    return a.view(m.get(a.dtype, a.dtype))
+
+
+def _to_dev(a: np.ndarray) -> torch.Tensor:
+    a = _as_signed(a).reshape(-1)
+    if a.dtype == np.uint8:
+        a = a.view(np.int32)
+    return torch.from_numpy(a.copy()).cuda()
+
+
+# ---------------------------------------------------------------- per-kernel jobs
+
+def job_binarysearch(N, Q, seed=6, rank=0):
+    A, _ = inputs.binarysearch_inputs(seed, N, 1)
+    q = inputs.u32(seed, Q, rank * Q, stream=2)
+    return Job("binarysearch", Q, (N, Q), [A, q, None], [(2, 4 * Q)], alg_bytes=8 * Q, unit="queries",
+               bound="latency", note="8 B/query compulsory; probes are dependent random 32-B sectors")
+
+
+def job_fwt(N, seed=5, rank=0):
+    m = N.bit_length() - 1
+    passes = 1 + (max(0, m - 12) + 6) // 7
+    x = inputs.fwt_x(seed, N, rank * N)
+    return Job("fwt", N, (), [x, None], [(1, 4 * N)], alg_bytes=8 * N * passes, unit="elements",
+               note=f"{passes} passes x 8 B/elem")
+
+
+def job_prefixsum(n, seed=4, rank=0):
+    return Job("prefixsum", n, (), [inputs.prefixsum_x(seed, n, rank * n), None], [(1, 4 * n)],
+               alg_bytes=8 * n, unit="elements")
+
+
+def job_reduction(n, seed=2, rank=0):
+    return Job("reduction", n, (), [inputs.reduction_x(seed, n, rank * n), None], [(1, 8)],
+               alg_bytes=4 * n, unit="elements")
+
+
+def job_transpose(H, W, seed=3, rank=0):
+    A = inputs.transpose_a(seed, H, W, rank * H)
+    return Job("transpose", H * W, (H, W), [A.view(np.uint32), None], [(1, 4 * H * W)],
+               alg_bytes=8 * H * W, unit="elements")
+
+
+def job_sobel(H, W, seed=7, rank=0):
+    I = inputs.sobel_image(seed, H, W, rank * H).view(np.uint32).reshape(-1)
+    return Job("sobel", H * W, (H, W), [I, None], [(1, 4 * H * W)], alg_bytes=8 * H * W, unit="pixels")
+
+
+def job_blackscholes(n, seed=1, rank=0):
+    return Job("blackscholes", n, (), [inputs.blackscholes_r(seed, n, rank * n), None, None],
+               [(1, 4 * n), (2, 4 * n)], alg_bytes=12 * n, unit="options")
+
+
+# ---------------------------------------------------------------- BASELINE.json configs
+
+def config_jobs(name: str, rank: int = 0):
+    if name == "suite":      # configs[1]: the APP SDK-style suite, "paper's sizes"
+        return [job_binarysearch(1 << 26, 1 << 24, rank=rank), job_fwt(1 << 26, rank=rank),
+                job_prefixsum(1 << 26, rank=rank), job_reduction(1 << 26, rank=rank),
+                job_transpose(8192, 8192, rank=rank), job_sobel(8192, 8192, rank=rank)]
+    if name == "suite28":    # configs[2]: 2^28 elements
+        return [job_binarysearch(1 << 28, 1 << 26, rank=rank), job_fwt(1 << 28, rank=rank),
+                job_prefixsum(1 << 28, rank=rank), job_reduction(1 << 28, rank=rank),
+                job_transpose(16384, 16384, rank=rank), job_sobel(16384, 16384, rank=rank)]
+    if name == "bs16":       # configs[0]
+        return [job_blackscholes(1 << 16, rank=rank)]
+    if name == "bs30":       # configs[4] (BlackScholes part)
+        return [job_blackscholes(1 << 30, rank=rank)]
+    if name == "small":      # smoke-sized
+        return [job_binarysearch(1 << 16, 1 << 14, rank=rank), job_fwt(1 << 14, rank=rank),
+                job_prefixsum(1 << 16, rank=rank), job_reduction(1 << 16, rank=rank),
+                job_transpose(256, 256, rank=rank), job_sobel(256, 256, rank=rank)]
+    raise ValueError(f"unknown config {name}")
+
+
+CONFIG_TITLES = {
+    "suite": "APP SDK-style suite (BinarySearch N=2^26 Q=2^24, FWT 2^26, PrefixSum 2^26, Reduction 2^26, "
+             "Transpose 8192^2, Sobel 8192^2) x {none, intra_smem, intra_reg, inter_group}",
+    "suite28": "suite at 2^28 elements (BinarySearch N=2^28 Q=2^26, Transpose/Sobel 16384^2)",
+    "bs16": "BlackScholes 2^16 options",
+    "bs30": "BlackScholes 2^30 options",
+    "small": "suite at smoke sizes",
+}

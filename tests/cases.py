@@ -134,10 +134,139 @@ class Transpose(Case):
         return 1, self.n
 
 
+class PrefixSum(Case):
+    kernel = "prefixsum"
+
+    def __init__(self, n, seed=4, x=None):
+        self.n = n
+        self.x = inputs.prefixsum_x(seed, n) if x is None else x
+
+    @functools.cached_property
+    def x_d(self):
+        return dev(self.x if self.n else np.zeros(4, np.uint32))
+
+    def buffers(self):
+        return [self.x_d[: self.n], out_like(4 * max(self.n, 1))[: self.n]]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32)]
+
+    def check(self, outs, x=None):
+        x = self.x if x is None else x
+        assert np.array_equal(outs[0], oracle.prefixsum_u32(x))
+
+    def out_elems(self):
+        return 1, self.n
+
+
+class FWT(Case):
+    kernel = "fwt"
+
+    def __init__(self, n, seed=5, ternary=False):
+        self.n = n
+        self.multipass = n > 4096
+        self.x = inputs.fwt_ternary(seed, n) if ternary else inputs.fwt_x(seed, n)
+
+    @functools.cached_property
+    def x_d(self):
+        return dev(self.x)
+
+    def buffers(self):
+        return [self.x_d, out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32)]
+
+    def check(self, outs, x=None):
+        x = self.x if x is None else x
+        # R-FWT2: bit-exact vs the fp32 butterfly DAG in the normative stage order
+        assert np.array_equal(outs[0], oracle.fwt_f32dag(x).view(np.uint32))
+        # and within fp32 rounding of the fp64 definition (BJ 1e-5 relative, scaled by ||x||_1)
+        y64 = oracle.fwt_f64(x)
+        got = outs[0].view(np.float32).astype(np.float64)
+        assert np.max(np.abs(got - y64)) <= 1e-5 * max(1.0, float(np.sum(np.abs(x))) / np.sqrt(len(x)))
+
+    def out_elems(self):
+        return 1, self.n
+
+
+class BinarySearch(Case):
+    kernel = "binarysearch"
+
+    def __init__(self, N, Q, seed=6, odd=False):
+        self.N, self.Q = N, Q
+        self.n = Q
+        self.dims = (N, Q)
+        if odd:
+            self.A = (2 * np.arange(N, dtype=np.uint64) + 1).astype(np.uint32)
+            self.q = inputs.u32(seed, Q) % np.uint32(2 * N + 8)
+        else:
+            self.A, self.q = inputs.binarysearch_inputs(seed, max(N, 1), Q)
+            self.A = self.A[:N]
+
+    @functools.cached_property
+    def A_d(self):
+        return dev(self.A if self.N else np.zeros(4, np.uint32))[: self.N]
+
+    @functools.cached_property
+    def q_d(self):
+        return dev(self.q)
+
+    def buffers(self):
+        return [self.A_d, self.q_d, out_like(4 * self.Q)]
+
+    def outputs(self, b):
+        return [host(b[2], np.uint32)]
+
+    def check(self, outs, A=None, q=None):
+        A = self.A if A is None else A
+        q = self.q if q is None else q
+        assert np.array_equal(outs[0], oracle.binarysearch(A, q))
+
+    def out_elems(self):
+        return 2, self.Q
+
+
+class Sobel(Case):
+    kernel = "sobel"
+
+    def __init__(self, H, W, seed=7, noise=False):
+        self.H, self.W = H, W
+        self.n = H * W
+        self.dims = (H, W)
+        if noise:
+            self.I = (inputs.u32(seed, H * W * 4) & np.uint32(255)).astype(np.uint8).reshape(H, W, 4)
+        else:
+            self.I = inputs.sobel_image(seed, H, W)
+
+    @functools.cached_property
+    def I_d(self):
+        return dev(self.I.view(np.uint32).reshape(-1))
+
+    def buffers(self):
+        return [self.I_d, out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32)]
+
+    def check(self, outs, I=None):
+        I = self.I if I is None else I
+        ref = oracle.sobel(I).view(np.uint32).reshape(-1)
+        assert np.array_equal(outs[0], ref), f"{np.sum(outs[0] != ref)} pixels differ"
+
+    def out_elems(self):
+        return 1, self.n
+
+
 def small_cases():
     """Sizes the oracle finishes in seconds that still span several tiles and a ragged tail."""
     return [
         BlackScholes(1), BlackScholes(7), BlackScholes(1024 * 3 + 5), BlackScholes(1 << 16),
         Reduction(0), Reduction(3), Reduction(1000003), Reduction(1 << 22),
         Transpose(4, 4), Transpose(68, 132), Transpose(256, 512, index_coded=True), Transpose(1000, 764),
+        PrefixSum(1), PrefixSum(4095), PrefixSum(4096 * 37 + 11), PrefixSum(1 << 22),
+        FWT(1), FWT(2), FWT(64), FWT(4096), FWT(1 << 13), FWT(1 << 20), FWT(1 << 16, ternary=True),
+        BinarySearch(0, 16), BinarySearch(1, 7), BinarySearch(1000, 1003), BinarySearch(1 << 16, 50000, odd=True),
+        BinarySearch(1 << 22, 1 << 18),
+        Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
     ]

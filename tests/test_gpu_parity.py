@@ -64,7 +64,12 @@ def test_store_value_fault_detected(case, replica, variant):
     o = outs[0].reshape(-1)
     r = ref[0].reshape(-1)
     grp = case.commit_group(e)
-    assert np.all(o[grp] == 0xFFFFFFFF), "faulted commit must not be stored"
+    if getattr(case, "multipass", False):
+        # in-place multi-pass kernel: the suppressed final store leaves the
+        # previous pass's intermediate in place (not the committed result)
+        assert not np.array_equal(o[grp], r[grp]), "faulted commit must not be stored"
+    else:
+        assert np.all(o[grp] == 0xFFFFFFFF), "faulted commit must not be stored"
     mask = np.ones(o.size, bool)
     mask[grp] = False
     assert np.array_equal(o[mask], r[mask])
