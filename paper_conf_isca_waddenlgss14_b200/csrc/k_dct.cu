@@ -1,0 +1,145 @@
+// k_dct.cu -- DCT ("DCT"; high Intra overhead despite being
+// memory-bound; Inter ~2x and the only kernel hurt by doubling groups,
+// P:809).  Forward orthonormal 8x8 DCT-II per block (reading R-DCT1):
+//   Y = C X C^T,  C[u][x] = alpha(u) cos((2x+1) u pi / 16).
+//
+// Logical CTA = a strip of 8 image rows x 256 columns (32 blocks); logical
+// thread (block b, row r) does the row pass Z[r][.] = X[r][.] C^T (8 FMA-chains
+// of length 8), Z goes through (duplicated, +LDS) shared memory, then logical
+// thread (b, u) does the column pass Y[u][.] = C[u][.] Z and commits its output
+// row as two 16-B vector stores.  Fixed FMA order with explicit rounding, so
+// every variant is bit-identical.  The C table (fp64 -> fp32, computed here on
+// the host, independently of the oracle) travels in the kernel arguments.
+#include <math.h>
+
+#include "rmt_host.cuh"
+
+namespace rmt {
+namespace {
+
+constexpr int BL = 256;
+constexpr int BLOCKS = 32;       // 8x8 blocks per logical CTA
+constexpr int BSTRIDE = 68;      // words per block in smem (64 + 4: conflict-free column pass)
+constexpr int ZWORDS = BLOCKS * BSTRIDE;
+constexpr int PLANE = ZWORDS + 16;  // replica plane offset (16 banks apart)
+
+struct DctArgs {
+  const float* X;
+  float* Y;
+  unsigned H, W;
+  unsigned nbx;  // logical CTAs across a row strip
+  float C[8][8];
+};
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c) {
+  constexpr int DUP = Geom<V>::DUP;
+  __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
+  __shared__ __align__(16) float Zs[DUP == 2 ? PLANE + ZWORDS : ZWORDS];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
+  const int b = rep.ltid / 8, r = rep.ltid % 8;
+  const unsigned col0 = (bx * BLOCKS + b) * 8;
+  const bool active = col0 < a.W;
+  const unsigned row = by * 8 + r;
+  // row pass
+  float x[8];
+  if (active) {
+    const float4* src = reinterpret_cast<const float4*>(a.X + (size_t)row * a.W + col0);
+    float4 p = __ldcs(src), q = __ldcs(src + 1);
+    x[0] = p.x; x[1] = p.y; x[2] = p.z; x[3] = p.w; x[4] = q.x; x[5] = q.y; x[6] = q.z; x[7] = q.w;
+  } else {
+#pragma unroll
+    for (int y = 0; y < 8; ++y) x[y] = 0.0f;
+  }
+  if constexpr (M == M_FAULT) {
+#pragma unroll
+    for (int y = 0; y < 8; ++y) x[y] = rep.faultf(SITE_LOAD, (long long)row * a.W + col0 + y, x[y]);
+  }
+  float z[8];
+#pragma unroll
+  for (int v = 0; v < 8; ++v) {
+    float s = __fmul_rn(x[0], a.C[v][0]);
+#pragma unroll
+    for (int y = 1; y < 8; ++y) s = __fmaf_rn(x[y], a.C[v][y], s);
+    if constexpr (M == M_FAULT) s = rep.faultf(SITE_COMPUTE, (long long)row * a.W + col0 + v, s);
+    z[v] = s;
+  }
+  float* zrow = &rep.template smp<PLANE>(Zs, b * BSTRIDE + r * 8);
+  reinterpret_cast<float4*>(zrow)[0] = make_float4(z[0], z[1], z[2], z[3]);
+  reinterpret_cast<float4*>(zrow)[1] = make_float4(z[4], z[5], z[6], z[7]);
+  __syncthreads();
+  // column pass: thread (b, u) produces output row u of block b
+  const int u = r;
+  float y[8];
+#pragma unroll
+  for (int v = 0; v < 8; ++v) y[v] = 0.0f;
+  const float* zb = &rep.template smp<PLANE>(Zs, b * BSTRIDE);
+#pragma unroll
+  for (int xr = 0; xr < 8; ++xr) {
+    float4 p = reinterpret_cast<const float4*>(zb + xr * 8)[0];
+    float4 q = reinterpret_cast<const float4*>(zb + xr * 8)[1];
+    float zz[8] = {p.x, p.y, p.z, p.w, q.x, q.y, q.z, q.w};
+    if constexpr (M == M_FAULT) {
+#pragma unroll
+      for (int v = 0; v < 8; ++v)
+        zz[v] = rep.faultf(SITE_SMEM, (long long)(by * 8 + xr) * a.W + col0 + v, zz[v]);
+    }
+    const float cu = a.C[u][xr];
+#pragma unroll
+    for (int v = 0; v < 8; ++v) y[v] = xr == 0 ? __fmul_rn(cu, zz[v]) : __fmaf_rn(cu, zz[v], y[v]);
+  }
+  const unsigned orow = by * 8 + u;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    unsigned w[4] = {__float_as_uint(y[4 * h]), __float_as_uint(y[4 * h + 1]), __float_as_uint(y[4 * h + 2]),
+                     __float_as_uint(y[4 * h + 3])};
+    const unsigned idx = orow * a.W + col0 + 4 * h;
+    rep.template commit<4, 0>(active ? 0xFu : 0u, active ? idx : 0u, w, a.H * a.W,
+                              [&](unsigned i, unsigned m, const unsigned* v) {
+                                if (m == 0xFu)
+                                  __stcs(reinterpret_cast<float4*>(a.Y + i),
+                                         make_float4(__uint_as_float(v[0]), __uint_as_float(v[1]),
+                                                     __uint_as_float(v[2]), __uint_as_float(v[3])));
+                                else
+                                  for (int k = 0; k < 4; ++k)
+                                    if ((m >> k) & 1u) a.Y[i + k] = __uint_as_float(v[k]);
+                              });
+  }
+  rep.finish();
+}
+
+}  // namespace
+
+int dct_validate(const rmt_bufs_t* b, int64_t n) {
+  int64_t H = b->dims[0], W = b->dims[1];
+  if (b->nbuf < 2 || H < 0 || W < 0 || n != H * W || H % 8 || W % 8 || n >= (1LL << 30) ||
+      !buf_ok(b->buf[0], RMT_F32, n) || !buf_ok(b->buf[1], RMT_F32, n)) {
+    set_error("dct: expected {X,Y} F32[H*W], dims {H,W}, H%8 = W%8 = 0");
+    return RMT_EINVAL;
+  }
+  return RMT_OK;
+}
+size_t dct_scratch(int64_t, const int64_t*) { return 0; }
+int dct_inter_warps(int64_t, const int64_t*) { return BL / 32; }
+
+int dct_run(Launch& L) {
+  const unsigned H = (unsigned)L.bufs->dims[0], W = (unsigned)L.bufs->dims[1];
+  const unsigned nbx = (W / 8 + BLOCKS - 1) / BLOCKS, nby = H / 8;
+  DctArgs a;
+  a.X = (const float*)L.bufs->buf[0].ptr;
+  a.Y = (float*)L.bufs->buf[1].ptr;
+  a.H = H;
+  a.W = W;
+  a.nbx = nbx;
+  for (int u = 0; u < 8; ++u)  // C[u][x] = alpha(u) cos((2x+1) u pi / 16), in fp64 then rounded
+    for (int x = 0; x < 8; ++x)
+      a.C[u][x] = (float)((u == 0 ? sqrt(0.125) : 0.5) * cos((2.0 * x + 1.0) * u * 3.14159265358979323846 / 16.0));
+  return dispatch(L.variant, L.mode, [&](auto vm) {
+    constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+    return launch_std<V>(L, dct_kernel<V, M>, dct_kernel<V_NONE, M_NORMAL>, nbx * nby, BL, 0, a, "dct");
+  });
+}
+
+}  // namespace rmt

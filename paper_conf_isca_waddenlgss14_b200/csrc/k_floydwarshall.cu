@@ -1,0 +1,127 @@
+// k_floydwarshall.cu -- FloydWarshall ("FW"; memory-bound with
+// minimal Intra overhead at large sizes; Inter ~2x; FAST
+// slower).  All-pairs shortest paths, canonical k order (readings
+// R-FW1..4): for k: if D[i][k] + D[k][j] < D[i][j]: D[i][j] = that, P[i][j] = k.
+//
+// One launch per k (naive schedule, the faithful primary: row k and column k
+// do not change during step k, so the in-place update is race-free and P is
+// unique).  Logical thread = 4 consecutive j of one row i: 16-B loads of
+// D[i][j..], D[k][j..], one broadcast D[i][k]; the stores are CONDITIONAL (only
+// improving relaxations write) and are committed with a per-word
+// predicate mask: (mask, address, D words) and (mask, address, P words).
+// D (n^2 u32 = 64 MiB at n = 4096) stays L2-resident across passes.
+#include "rmt_host.cuh"
+
+namespace rmt {
+namespace {
+
+constexpr int BL = 256;
+
+struct FwArgs {
+  unsigned* D;
+  unsigned* P;
+  unsigned n;
+  unsigned k;
+};
+
+__device__ __forceinline__ void store4(unsigned* base, unsigned idx, unsigned m, const unsigned* v) {
+  if (m == 0xFu) *reinterpret_cast<uint4*>(base + idx) = make_uint4(v[0], v[1], v[2], v[3]);
+  else
+    for (int q = 0; q < 4; ++q)
+      if ((m >> q) & 1u) base[idx + q] = v[q];
+}
+
+// P[i][j] = i for all (i, j) (reading R-FW2).
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_init_kernel(FwArgs a, Ctx c) {
+  __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const unsigned e0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * 4;
+  const unsigned nn = a.n * a.n;
+  unsigned w[4];
+  unsigned i = e0 / a.n;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) w[q] = i;
+  rep.template commit<4, 2>(e0 < nn ? 0xFu : 0u, e0 < nn ? e0 : 0u, w, nn,
+                            [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
+  rep.finish();
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ctx c) {
+  __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const unsigned e0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * 4;
+  const unsigned nn = a.n * a.n;
+  const bool active = e0 < nn;
+  const unsigned i = active ? e0 / a.n : 0u, j = active ? e0 - i * a.n : 0u;
+  unsigned dik = 0;
+  uint4 dkj = make_uint4(0, 0, 0, 0), dij = make_uint4(0, 0, 0, 0);
+  if (active) {
+    dik = a.D[(size_t)i * a.n + a.k];
+    dkj = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
+    dij = *reinterpret_cast<const uint4*>(a.D + e0);
+  }
+  unsigned kj[4] = {dkj.x, dkj.y, dkj.z, dkj.w};
+  unsigned ij[4] = {dij.x, dij.y, dij.z, dij.w};
+  if constexpr (M == M_FAULT) {
+    dik = rep.fault(SITE_LOAD, (long long)i * a.n + a.k, dik);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) ij[q] = rep.fault(SITE_LOAD, (long long)e0 + q, ij[q]);
+  }
+  unsigned nd[4], np[4], mask = 0;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    unsigned cand = dik + kj[q];
+    if constexpr (M == M_FAULT) cand = rep.fault(SITE_COMPUTE, (long long)e0 + q, cand);
+    const bool better = active && cand < ij[q];
+    mask |= (better ? 1u : 0u) << q;
+    nd[q] = cand;
+    np[q] = a.k;
+  }
+  rep.template commit<4, 0>(mask, e0, nd, nn, [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); });
+  rep.template commit<4, 1>(mask, e0, np, nn, [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
+  rep.finish();
+}
+
+}  // namespace
+
+int floydwarshall_validate(const rmt_bufs_t* b, int64_t n) {
+  if (b->nbuf < 2 || n < 0 || n % 4 || n * n >= (1LL << 30) || !buf_ok(b->buf[0], RMT_U32, n * n) ||
+      !buf_ok(b->buf[1], RMT_U32, n * n)) {
+    set_error("floydwarshall: expected {D (in/out), P} U32[n*n], n%4 = 0, n*n < 2^30");
+    return RMT_EINVAL;
+  }
+  return RMT_OK;
+}
+size_t floydwarshall_scratch(int64_t, const int64_t*) { return 0; }
+int floydwarshall_inter_warps(int64_t, const int64_t*) { return BL / 32; }
+
+int floydwarshall_run(Launch& L) {
+  const unsigned n = (unsigned)L.n;
+  if (n == 0) return RMT_OK;
+  const unsigned nn = n * n;
+  const unsigned G = (nn / 4 + BL - 1) / BL;
+  FwArgs a{(unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, n, 0};
+  // Fault element = k0 * n^2 + e: the pass k0 and the element e.
+  const FaultDesc f = L.ctx.f;
+  const unsigned k0 = (unsigned)(f.elem / nn);
+  return dispatch(L.variant, L.mode, [&](auto vm) {
+    constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+    L.ctx.f.site = -1;  // the init pass carries no fault
+    int rc = launch_std<V>(L, fw_init_kernel<V, M>, fw_init_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "fw/init");
+    for (unsigned k = 0; k < n && rc == RMT_OK; ++k) {
+      a.k = k;
+      L.ctx.f = f;
+      if (k == k0) L.ctx.f.elem = f.elem - (long long)k0 * nn;
+      else L.ctx.f.site = -1;
+      rc = launch_std<V>(L, fw_pass_kernel<V, M>, fw_pass_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "fw/pass");
+    }
+    L.ctx.f = f;
+    return rc;
+  });
+}
+
+}  // namespace rmt

@@ -10,7 +10,5 @@ namespace rmt {
     set_error(#name ": not implemented yet");                                            \
     return RMT_EUNSUPPORTED;                                                             \
   }
-RMT_STUB(floydwarshall)
-RMT_STUB(dct)
 RMT_STUB(matmul)
 }  // namespace rmt

@@ -205,6 +205,15 @@ struct Rep {
     else return base[i];
   }
 
+  // ---- duplicated shared memory in planes: replica r owns base[PLANE*r + i].
+  // PLANE is chosen per kernel so the two replicas of a pair land in disjoint
+  // banks for that kernel's access patterns (interleaving conflicts otherwise).
+  template <int PLANE, class T>
+  __device__ __forceinline__ T& smp(T* base, int i) const {
+    if constexpr (INTRA) return base[PLANE * r + i];
+    else return base[i];
+  }
+
   // ---- logical-warp shuffles (replica-private: lanes keep their role bit)
   __device__ __forceinline__ unsigned lshfl_xor(unsigned v, int m) const {
     return __shfl_xor_sync(FULL, v, m * DUP);

@@ -38,6 +38,16 @@ class Case:
         """(buffer index, element count) of the first output buffer (STORE_* fault site)."""
         raise NotImplementedError
 
+    def fault_target(self, rng):
+        """(elem for rmt_inject_fault, word index in the first output buffer)."""
+        b, ne = self.out_elems()
+        e = int(rng.integers(0, ne))
+        return e, e
+
+    def fault_propagates(self):
+        """True if a suppressed store feeds later computation (multi-pass, in place)."""
+        return False
+
     def commit_group(self, e):
         """Word indices of the first output buffer stored by the same commit as
         word e (one commit per store instruction; vector stores are 4 words)."""
@@ -258,6 +268,92 @@ class Sobel(Case):
         return 1, self.n
 
 
+class DCT(Case):
+    kernel = "dct"
+
+    def __init__(self, H, W, seed=9):
+        self.H, self.W = H, W
+        self.n = H * W
+        self.dims = (H, W)
+        self.X = inputs.dct_x(seed, H, W)
+
+    @functools.cached_property
+    def X_d(self):
+        return dev(self.X)
+
+    def buffers(self):
+        return [self.X_d, out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32)]
+
+    def check(self, outs, X=None):
+        X = self.X if X is None else X
+        H, W = X.shape
+        got = outs[0].view(np.float32).reshape(H, W).astype(np.float64)
+        ref = oracle.dct8x8(X)
+        bound = oracle.dct8x8_absbound(X)
+        # reading R-DCT3: componentwise condition-scaled 1e-5, and per-block normwise 1e-5
+        assert np.all(np.abs(got - ref) <= 1e-5 * bound + 1e-30)
+        d = (got - ref).reshape(H // 8, 8, W // 8, 8)
+        x = X.astype(np.float64).reshape(H // 8, 8, W // 8, 8)
+        num = np.sqrt((d ** 2).sum(axis=(1, 3)))
+        den = np.sqrt((x ** 2).sum(axis=(1, 3)))
+        assert np.all(num <= 1e-5 * np.maximum(den, 1e-30))
+
+    def out_elems(self):
+        return 1, self.n
+
+
+class FloydWarshall(Case):
+    kernel = "floydwarshall"
+
+    def __init__(self, n, seed=8):
+        self.n = n
+        self.Wm = inputs.floydwarshall_w(seed, n)
+
+    @functools.cached_property
+    def W_d(self):
+        return dev(self.Wm)
+
+    def buffers(self):
+        return [self.W_d.clone(), out_like(4 * self.n * self.n)]
+
+    def outputs(self, b):
+        return [host(b[0], np.uint32).reshape(self.n, self.n), host(b[1], np.uint32).reshape(self.n, self.n)]
+
+    def check(self, outs, Wm=None):
+        Wm = self.Wm if Wm is None else Wm
+        D, P = oracle.floydwarshall(Wm)
+        assert np.array_equal(outs[0], D)
+        assert np.array_equal(outs[1], P)
+
+    def out_elems(self):
+        return 0, self.n * self.n
+
+    def fault_target(self, rng):
+        # an element whose LAST improving relaxation happens at pass k0: suppressing
+        # that store leaves a visibly different final D[e]
+        n = self.n
+        D = self.Wm.astype(np.int64)
+        last = np.full((n, n), -1)
+        for k in range(n):
+            cand = D[:, k:k + 1] + D[k:k + 1, :]
+            better = cand < D
+            last[better] = k
+            D = np.where(better, cand, D)
+        idx = np.flatnonzero(last.reshape(-1) > 0)
+        e = int(idx[rng.integers(0, idx.size)])
+        k0 = int(last.reshape(-1)[e])
+        return k0 * n * n + e, e
+
+    def fault_propagates(self):
+        return True
+
+    def commit_group(self, e):
+        return np.array([e])  # masked vector commit: only improving words are stored
+
+
 def small_cases():
     """Sizes the oracle finishes in seconds that still span several tiles and a ragged tail."""
     return [
@@ -269,4 +365,6 @@ def small_cases():
         BinarySearch(0, 16), BinarySearch(1, 7), BinarySearch(1000, 1003), BinarySearch(1 << 16, 50000, odd=True),
         BinarySearch(1 << 22, 1 << 18),
         Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
+        DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8),
+        FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
     ]
