@@ -10,5 +10,4 @@ namespace rmt {
     set_error(#name ": not implemented yet");                                            \
     return RMT_EUNSUPPORTED;                                                             \
   }
-RMT_STUB(matmul)
 }  // namespace rmt

@@ -354,6 +354,52 @@ class FloydWarshall(Case):
         return np.array([e])  # masked vector commit: only improving words are stored
 
 
+class MatMul(Case):
+    kernel = "matmul"
+
+    def __init__(self, M, N, K, seed=10, integer=False):
+        self.M, self.N, self.K = M, N, K
+        self.n = M * N
+        self.dims = (M, N, K)
+        self.integer = integer
+        if integer:
+            self.A = inputs.matmul_bf16_int(seed, M, K, stream=20)
+            self.Bt = inputs.matmul_bf16_int(seed, N, K, stream=21)
+        else:
+            self.A = inputs.matmul_bf16_normal(seed, M, K, stream=22)
+            self.Bt = inputs.matmul_bf16_normal(seed, N, K, stream=24)
+
+    @functools.cached_property
+    def A_d(self):
+        return dev(self.A)
+
+    @functools.cached_property
+    def B_d(self):
+        return dev(self.Bt)
+
+    def buffers(self):
+        return [self.A_d, self.B_d, out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[2], np.uint32).reshape(self.M, self.N)]
+
+    def check(self, outs):
+        got = outs[0].view(np.float32).astype(np.float64)
+        ref = oracle.matmul_bf16(self.A, self.Bt)
+        if self.integer:
+            # exactness pin: |partial sums| <= 16 K < 2^24 -> exact in fp32 regardless of order
+            assert np.array_equal(got, ref)
+            return
+        # reading R-MM2: normwise 1e-5, plus the loose elementwise catch-all K 2^-23 (|A||B|)
+        assert np.linalg.norm(got - ref) <= 1e-5 * np.linalg.norm(ref)
+        Af = np.abs(inputs.bf16_bits_to_f32(self.A).astype(np.float64))
+        Bf = np.abs(inputs.bf16_bits_to_f32(self.Bt).astype(np.float64))
+        assert np.all(np.abs(got - ref) <= self.K * 2.0 ** -23 * (Af @ Bf.T) + 1e-30)
+
+    def out_elems(self):
+        return 2, self.n
+
+
 def small_cases():
     """Sizes the oracle finishes in seconds that still span several tiles and a ragged tail."""
     return [
@@ -367,4 +413,5 @@ def small_cases():
         Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
         DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8),
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
+        MatMul(128, 128, 64), MatMul(256, 384, 192, integer=True), MatMul(512, 256, 1024),
     ]
