@@ -136,10 +136,14 @@ def matmul_bf16_normal(seed: int, rows: int, cols: int, stream: int, row_offset:
     """bf16 N(0,1) (Box-Muller on two counter streams), returned as uint16 bits."""
     n = rows * cols
     off = row_offset * cols
-    u1 = (u64(seed, n, off, stream=stream) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
-    u2 = (u64(seed, n, off, stream=stream + 1) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
-    g = np.sqrt(-2.0 * np.log1p(-u1)) * np.cos(2.0 * np.pi * u2)
-    return f32_to_bf16_bits(g.astype(np.float32)).reshape(rows, cols)
+    out = np.empty(n, np.uint16)
+    for s in range(0, n, _CHUNK):
+        e = min(n, s + _CHUNK)
+        u1 = (u64(seed, e - s, off + s, stream=stream) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+        u2 = (u64(seed, e - s, off + s, stream=stream + 1) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+        g = np.sqrt(-2.0 * np.log1p(-u1)) * np.cos(2.0 * np.pi * u2)
+        out[s:e] = f32_to_bf16_bits(g.astype(np.float32))
+    return out.reshape(rows, cols)
 
 
 def matmul_bf16_int(seed: int, rows: int, cols: int, stream: int, lo: int = -4, hi: int = 4,

@@ -113,6 +113,25 @@ def job_blackscholes(n, seed=1, rank=0):
                [(1, 4 * n), (2, 4 * n)], alg_bytes=12 * n, unit="options")
 
 
+def job_matmul(M, N, K, seed=10, rank=0):
+    A = inputs.matmul_bf16_normal(seed, M, K, stream=22, row_offset=rank * M)
+    Bt = inputs.matmul_bf16_normal(seed, N, K, stream=24)
+    return Job("matmul", M * N, (M, N, K), [A, Bt, None], [(2, 4 * M * N)],
+               alg_bytes=2 * (M * K + N * K) + 4 * M * N, unit="C elements", bound="tensor",
+               note=f"{2 * M * N * K:.3e} flop")
+
+
+def job_dct(H, W, seed=9, rank=0):
+    return Job("dct", H * W, (H, W), [inputs.dct_x(seed, H, W, rank * H), None], [(1, 4 * H * W)],
+               alg_bytes=8 * H * W, unit="elements")
+
+
+def job_floydwarshall(n, seed=8):
+    return Job("floydwarshall", n, (), [inputs.floydwarshall_w(seed, n), None], [(1, 4 * n * n)],
+               alg_bytes=(n + 1) * 4 * n * n, unit="nodes", bound="l2",
+               note="per pass: 4 B/elem read of D (L2-resident) + conditional writes; n passes + init")
+
+
 # ---------------------------------------------------------------- BASELINE.json configs
 
 def config_jobs(name: str, rank: int = 0):
@@ -128,6 +147,12 @@ def config_jobs(name: str, rank: int = 0):
         return [job_blackscholes(1 << 16, rank=rank)]
     if name == "bs30":       # configs[4] (BlackScholes part)
         return [job_blackscholes(1 << 30, rank=rank)]
+    if name == "mm16k":      # configs[4] (MatrixMultiplication part)
+        return [job_matmul(16384, 16384, 16384, rank=rank)]
+    if name == "mm8k":
+        return [job_matmul(8192, 8192, 8192, rank=rank)]
+    if name == "fwdct":      # configs[3]
+        return [job_floydwarshall(4096), job_dct(8192, 8192, rank=rank)]
     if name == "small":      # smoke-sized
         return [job_binarysearch(1 << 16, 1 << 14, rank=rank), job_fwt(1 << 14, rank=rank),
                 job_prefixsum(1 << 16, rank=rank), job_reduction(1 << 16, rank=rank),
@@ -142,4 +167,7 @@ CONFIG_TITLES = {
     "bs16": "BlackScholes 2^16 options",
     "bs30": "BlackScholes 2^30 options",
     "small": "suite at smoke sizes",
+    "mm16k": "MatrixMultiplication 16384^3 bf16 -> fp32 (tcgen05)",
+    "mm8k": "MatrixMultiplication 8192^3 bf16 -> fp32 (tcgen05)",
+    "fwdct": "FloydWarshall 4096 nodes + DCT 8192^2",
 }
