@@ -20,6 +20,7 @@ constexpr int BL = 256;
 constexpr int TB_MAX = 12;
 constexpr int TE_MAX = 1 << TB_MAX;
 constexpr int SM_WORDS = TE_MAX + TE_MAX / 32;  // pad32 swizzle: <=2-way conflicts for all rounds
+constexpr int PLANE = SM_WORDS + 16;            // intra replica plane: 16 banks apart (fewest conflicts over all rounds)
 
 __device__ __forceinline__ int phys(int e) { return e + (e >> 5); }
 
@@ -53,7 +54,7 @@ __device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int 
     float v[G];
 #pragma unroll
     for (int k = 0; k < G; ++k) {
-      v[k] = rep.sm(tile, phys(ebase | (k << q)));
+      v[k] = rep.template smp<PLANE>(tile, phys(ebase | (k << q)));
       if constexpr (R::FAULT) {
         if (a.s0 == 0 && round_no == 1)
           v[k] = rep.faultf(SITE_SMEM, (long long)gindex(a, tileid, ebase | (k << q)), v[k]);
@@ -76,16 +77,67 @@ __device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int 
         if (a.s0 == 0 && round_no == 0)
           v[k] = rep.faultf(SITE_COMPUTE, (long long)gindex(a, tileid, ebase | (k << q)), v[k]);
       }
-      rep.sm(tile, phys(ebase | (k << q))) = v[k];
+      rep.template smp<PLANE>(tile, phys(ebase | (k << q))) = v[k];
     }
   }
 }
 
-template <int V, int M>
+// Compile-time round (full 4096-element tile): with Q known, phys(ebase | k<<Q)
+// = phys(ebase) + C(k) with a constant C(k) (ebase has zeros in bits Q..Q+NB),
+// so every element costs one LDS and one STS with an immediate offset.
+template <int NB, int Q>
+__device__ __forceinline__ constexpr int coff(int k) {
+  return (k << Q) + ((Q >= 5) ? (k << (Q - 5)) : ((k << Q) >> 5));
+}
+template <int NB, int Q, class R>
+__device__ __forceinline__ void fwt_round_ct(const R& rep, float* tile, const FwtArgs& a, unsigned tileid,
+                                             int round_no) {
+  constexpr int G = 1 << NB;
+  constexpr int GPT = (TE_MAX >> NB) / BL;  // groups per thread
+#pragma unroll
+  for (int w = 0; w < GPT; ++w) {
+    const int gi = rep.ltid + BL * w;
+    const int ebase = (gi & ((1 << Q) - 1)) | ((gi >> Q) << (Q + NB));
+    float* pb = &rep.template smp<PLANE>(tile, phys(ebase));
+    float v[G];
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      v[k] = pb[coff<NB, Q>(k)];
+      if constexpr (R::FAULT) {
+        if (a.s0 == 0 && round_no == 1)
+          v[k] = rep.faultf(SITE_SMEM, (long long)gindex(a, tileid, ebase | (k << Q)), v[k]);
+      }
+    }
+#pragma unroll
+    for (int s = 0; s < NB; ++s) {
+      const int h = 1 << s;
+#pragma unroll
+      for (int k = 0; k < G; ++k) {
+        if (k & h) continue;
+        const float x0 = v[k], x1 = v[k + h];
+        v[k] = __fadd_rn(x0, x1);
+        v[k + h] = __fsub_rn(x0, x1);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < G; ++k) {
+      if constexpr (R::FAULT) {
+        if (a.s0 == 0 && round_no == 0)
+          v[k] = rep.faultf(SITE_COMPUTE, (long long)gindex(a, tileid, ebase | (k << Q)), v[k]);
+      }
+      pb[coff<NB, Q>(k)] = v[k];
+    }
+  }
+}
+
+// KIND 0: generic (any tile size / stage range, runtime rounds)
+// KIND 1: pass 1 on full 4096-element tiles (stages 0..11: rounds at q = 0, 4, 8)
+// KIND 2: strided pass with b = 7, c = 5 (rounds at q = 5 (4 stages), q = 9 (3 stages))
+template <int V, int M, int KIND>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ float tile[SM_WORDS * DUP];
+  __shared__ float tile[DUP == 2 ? PLANE + SM_WORDS : SM_WORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned tileid = (unsigned)rep.lblock;
@@ -108,22 +160,36 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
         if constexpr (M == M_FAULT) {
           if (a.s0 == 0) x = rep.faultf(SITE_LOAD, (long long)g + k, x);
         }
-        rep.sm(tile, phys(e0 + k)) = x;
+        rep.template smp<PLANE>(tile, phys(e0 + k)) = x;
       }
     }
   }
   __syncthreads();
   // stages [s0, s0 + b) live at tile bits [c, c + b); rounds of <= 4 stages
-  int round_no = 0;
-  for (int q = a.c; q < a.c + a.b; q += 4, ++round_no) {
-    const int nb = min(4, a.c + a.b - q);
-    switch (nb) {
-      case 4: fwt_round<4>(rep, tile, q, te, a, tileid, round_no); break;
-      case 3: fwt_round<3>(rep, tile, q, te, a, tileid, round_no); break;
-      case 2: fwt_round<2>(rep, tile, q, te, a, tileid, round_no); break;
-      default: fwt_round<1>(rep, tile, q, te, a, tileid, round_no); break;
-    }
+  if constexpr (KIND == 1) {
+    fwt_round_ct<4, 0>(rep, tile, a, tileid, 0);
     __syncthreads();
+    fwt_round_ct<4, 4>(rep, tile, a, tileid, 1);
+    __syncthreads();
+    fwt_round_ct<4, 8>(rep, tile, a, tileid, 2);
+    __syncthreads();
+  } else if constexpr (KIND == 2) {
+    fwt_round_ct<4, 5>(rep, tile, a, tileid, 0);
+    __syncthreads();
+    fwt_round_ct<3, 9>(rep, tile, a, tileid, 1);
+    __syncthreads();
+  } else {
+    int round_no = 0;
+    for (int q = a.c; q < a.c + a.b; q += 4, ++round_no) {
+      const int nb = min(4, a.c + a.b - q);
+      switch (nb) {
+        case 4: fwt_round<4>(rep, tile, q, te, a, tileid, round_no); break;
+        case 3: fwt_round<3>(rep, tile, q, te, a, tileid, round_no); break;
+        case 2: fwt_round<2>(rep, tile, q, te, a, tileid, round_no); break;
+        default: fwt_round<1>(rep, tile, q, te, a, tileid, round_no); break;
+      }
+      __syncthreads();
+    }
   }
   // store: one vector commit per 4 elements
 #pragma unroll 1
@@ -134,7 +200,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
       const bool in = e0 + k < te;
-      w[k] = in ? __float_as_uint(rep.sm(tile, phys(e0 + k))) : 0u;
+      w[k] = in ? __float_as_uint(rep.template smp<PLANE>(tile, phys(e0 + k))) : 0u;
       mask |= (in ? 1u : 0u) << k;
     }
     const unsigned g = e0 < te ? gindex(a, tileid, (unsigned)e0) : 0u;
@@ -182,12 +248,15 @@ int fwt_run(Launch& L) {
     const int sid = L.ctx.f.sid;
     L.ctx.f.sid = (tb < m) ? -1 : sid;
     FwtArgs a{x, y, (unsigned)L.n, tb, 0, tb, 0};
-    int rc = launch_std<V>(L, fwt_kernel<V, M>, fwt_kernel<V_NONE, M_NORMAL>, tiles, BL, 0, a, "fwt/pass1");
+    int rc = tb == TB_MAX
+                 ? launch_std<V>(L, fwt_kernel<V, M, 1>, fwt_kernel<V_NONE, M_NORMAL, 1>, tiles, BL, 0, a, "fwt/pass1")
+                 : launch_std<V>(L, fwt_kernel<V, M, 0>, fwt_kernel<V_NONE, M_NORMAL, 0>, tiles, BL, 0, a, "fwt/pass1");
     for (int s = tb; s < m && rc == RMT_OK; ) {  // strided passes, in place on y
       const int b = (m - s) < 7 ? (m - s) : 7;
       L.ctx.f.sid = (s + b < m) ? -1 : sid;
       FwtArgs p{y, y, (unsigned)L.n, TB_MAX, s, b, TB_MAX - b};
-      rc = launch_std<V>(L, fwt_kernel<V, M>, fwt_kernel<V_NONE, M_NORMAL>, tiles, BL, 0, p, "fwt/pass");
+      rc = b == 7 ? launch_std<V>(L, fwt_kernel<V, M, 2>, fwt_kernel<V_NONE, M_NORMAL, 2>, tiles, BL, 0, p, "fwt/pass")
+                  : launch_std<V>(L, fwt_kernel<V, M, 0>, fwt_kernel<V_NONE, M_NORMAL, 0>, tiles, BL, 0, p, "fwt/pass");
       s += b;
     }
     L.ctx.f.sid = sid;

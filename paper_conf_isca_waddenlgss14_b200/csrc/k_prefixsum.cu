@@ -1,14 +1,19 @@
 // k_prefixsum.cu -- PrefixSum ("PS"; Intra comm >1/2 of the
 // overhead; FAST helps).  Inclusive scan of u32 mod 2^32
-// (readings R-PS1, R-PS2), single pass with decoupled look-back: 8 B/elem.
+// (readings R-PS1, R-PS2).
 //
-// Tile = 256 logical threads x 16 items.  Tile ids are taken in start order
-// (none/intra: a tile counter; inter: the RMT pair id, itself start-ordered,
-// P:679), so look-back never waits on an unstarted tile.  Integer addition is
-// associative, so every variant -- and every look-back timing -- produces the
-// identical result (determinism rule: look-back only on integers).
-// Tile status words are liveness-critical stores (other CTAs spin on them):
-// they are committed with LIVE=true (reading R-RMT5).
+// B200 design: reduce-then-scan over NCH = 1184 contiguous chunks (a multiple
+// of 4096-element tiles each).  A single-pass decoupled look-back was measured
+// (globaltimer trace of every tile) to serialise behind straggler tiles: one
+// slow tile's aggregate stalls every later tile's look-back while the waiting
+// CTAs hold all SM slots, so HBM idles.  Here no CTA waits on another:
+//   pass 1: each logical CTA sums its chunk and commits ONE partial (u32);
+//   pass 2: each logical CTA sums the partials of the chunks before it (its
+//           carry-in; <= 1183 L2-resident words), then scans its chunk tile by
+//           tile with a running carry and commits y.  Pass 2 visits chunks in
+//           the REVERSE order of pass 1, so the chunks pass 1 read last are
+//           still L2-resident.
+// Integer addition is associative: every variant produces the identical result.
 #include "rmt_host.cuh"
 
 namespace rmt {
@@ -16,136 +21,166 @@ namespace {
 
 constexpr int BL = 256;
 constexpr int ITEMS = 16;
-constexpr unsigned TILE = BL * ITEMS;
-constexpr unsigned long long FLAG_AGG = 1ull << 32, FLAG_INC = 2ull << 32;
+constexpr unsigned TILE = BL * ITEMS;   // 4096 elements
+constexpr unsigned NCH = 148u * 8u;     // chunks (logical CTAs per pass)
 
 struct PsArgs {
   const unsigned* x;
   unsigned* y;
-  unsigned long long* status;  // [ntiles]: (flag << 32) | value
-  unsigned* tile_counter;
+  unsigned* partial;   // [NCH]
   unsigned n;
+  unsigned chunk;      // elements per chunk (multiple of TILE)
+  unsigned nch;        // chunks actually used
 };
 
+// u32 sum over the logical CTA (logical warps + duplicated smem)
 template <int V, int M>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_kernel(PsArgs a, Ctx c) {
+__device__ __forceinline__ unsigned block_sum_u32(const Rep<V, M>& rep, unsigned s, unsigned* sw) {
+  constexpr int LW = Rep<V, M>::LW;
+  constexpr int NLW = BL / LW;
+#pragma unroll
+  for (int m = LW / 2; m >= 1; m >>= 1) s += rep.lshfl_xor(s, m);
+  if (rep.llane == 0) rep.sm(sw, rep.ltid / LW) = s;
+  __syncthreads();
+  unsigned t = rep.llane < NLW ? rep.sm(sw, rep.llane) : 0u;
+#pragma unroll
+  for (int m = LW / 2; m >= 1; m >>= 1) t += rep.lshfl_xor(t, m);
+  __syncthreads();
+  return t;
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_reduce_kernel(PsArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
-  constexpr int LW = 32 / DUP;
-  constexpr int NLW = BL / LW;  // logical warps per CTA
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned s_wtot[NLW * DUP];
-  __shared__ unsigned s_bcast[2 * DUP];
-  __shared__ unsigned s_tile;
+  __shared__ unsigned sw[(BL / (32 / DUP)) * DUP];
   Rep<V, M> rep(c);
   rep.init(mb);
-  unsigned tile;
-  if constexpr (V == V_INTER) {
-    tile = (unsigned)rep.lblock;
-  } else {
-    if (threadIdx.x == 0) s_tile = atomicAdd(a.tile_counter, 1u);
-    __syncthreads();
-    tile = s_tile;
-  }
-  const unsigned base = tile * TILE + (unsigned)rep.ltid * ITEMS;
-  unsigned v[ITEMS];
-  if (base + ITEMS <= a.n) {
+  const unsigned ch = (unsigned)rep.lblock;
+  const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
+  unsigned s = 0;
+  // 16-B coalesced loads, 4 in flight per thread (chunk starts are 16-B aligned)
+  for (unsigned e = lo + 4 * rep.ltid; e < hi; e += 4 * BL * 4) {
+    uint4 v[4];
 #pragma unroll
-    for (int q = 0; q < ITEMS / 4; ++q) {
-      uint4 w = __ldg(reinterpret_cast<const uint4*>(a.x + base) + q);
-      v[4 * q] = w.x; v[4 * q + 1] = w.y; v[4 * q + 2] = w.z; v[4 * q + 3] = w.w;
+    for (int u = 0; u < 4; ++u) {
+      const unsigned f = e + u * 4 * BL;
+      if (f + 4 <= hi) {
+        v[u] = __ldg(reinterpret_cast<const uint4*>(a.x + f));
+      } else {  // ragged tail of the array
+        v[u].x = f < hi ? a.x[f] : 0u;
+        v[u].y = f + 1 < hi ? a.x[f + 1] : 0u;
+        v[u].z = f + 2 < hi ? a.x[f + 2] : 0u;
+        v[u].w = 0u;
+      }
     }
-  } else {
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) v[i] = base + i < a.n ? a.x[base + i] : 0u;
+    for (int u = 0; u < 4; ++u) {
+      if constexpr (M == M_FAULT) {
+        const unsigned f = e + u * 4 * BL;
+        v[u].x = rep.fault(SITE_LOAD, (long long)f, v[u].x);
+        v[u].y = rep.fault(SITE_LOAD, (long long)f + 1, v[u].y);
+        v[u].z = rep.fault(SITE_LOAD, (long long)f + 2, v[u].z);
+        v[u].w = rep.fault(SITE_LOAD, (long long)f + 3, v[u].w);
+      }
+      s += v[u].x + v[u].y + v[u].z + v[u].w;
+    }
   }
-  if constexpr (M == M_FAULT) {
-#pragma unroll
-    for (int i = 0; i < ITEMS; ++i) v[i] = rep.fault(SITE_LOAD, (long long)base + i, v[i]);
+  s = rep.fault(SITE_COMPUTE, (long long)ch * BL + rep.ltid, s);
+  const unsigned t = block_sum_u32(rep, s, sw);
+  if (rep.warp == 0) {  // one store per CTA leaves the SoR ("ghost" warps)
+    unsigned w[1] = {t};
+    rep.template commit<1, 2>(rep.llane == 0 ? 1u : 0u, ch, w, a.nch,
+                              [&](unsigned i, unsigned, const unsigned* x) { a.partial[i] = x[0]; });
   }
-  // thread-local inclusive scan
-#pragma unroll
-  for (int i = 1; i < ITEMS; ++i) v[i] += v[i - 1];
-  unsigned tsum = rep.fault(SITE_COMPUTE, (long long)tile * BL + rep.ltid, v[ITEMS - 1]);
-  // logical-warp inclusive scan of thread totals
-  unsigned ws = tsum;
-#pragma unroll
-  for (int d = 1; d < LW; d <<= 1) {
-    unsigned u = rep.lshfl_up(ws, d);
-    if (rep.llane >= d) ws += u;
-  }
+  rep.finish();
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ctx c) {
+  constexpr int DUP = Geom<V>::DUP;
+  constexpr int LW = 32 / DUP;
+  constexpr int NLW = BL / LW;
+  __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
+  __shared__ unsigned sw[NLW * DUP];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const unsigned ch = a.nch - 1u - (unsigned)rep.lblock;  // reverse order: L2-hot chunks first
+  // carry-in: sum of the partials of all earlier chunks (L2-resident)
+  unsigned cs = 0;
+  for (unsigned i = rep.ltid; i < ch; i += BL) cs += __ldcg(a.partial + i);
+  unsigned carry = block_sum_u32(rep, cs, sw);
+  const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
   const int lw = rep.ltid / LW;
-  if (rep.llane == LW - 1) rep.sm(s_wtot, lw) = ws;
-  __syncthreads();
-  // warp 0: scan warp totals, then look-back
-  if (rep.warp == 0) {
-    unsigned t = rep.llane < NLW ? rep.sm(s_wtot, rep.llane) : 0u;
-    if constexpr (M == M_FAULT) t = rep.fault(SITE_SMEM, (long long)tile * BL + rep.llane * LW, t);
-    unsigned inc = t;
+  // register double buffer: the next tile's loads are in flight while this
+  // tile is scanned and stored
+  auto load_tile = [&](unsigned t0, unsigned (&v)[ITEMS]) {
+    const unsigned base = t0 + (unsigned)rep.ltid * ITEMS;
+    if (base + ITEMS <= hi) {
+#pragma unroll
+      for (int q = 0; q < ITEMS / 4; ++q) {
+        uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.x + base) + q);
+        v[4 * q] = w.x; v[4 * q + 1] = w.y; v[4 * q + 2] = w.z; v[4 * q + 3] = w.w;
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) v[i] = base + i < hi ? a.x[base + i] : 0u;
+    }
+  };
+  unsigned nxt[ITEMS];
+  if (lo < hi) load_tile(lo, nxt);
+#pragma unroll 1
+  for (unsigned t0 = lo; t0 < hi; t0 += TILE) {  // uniform trip count per CTA
+    const unsigned base = t0 + (unsigned)rep.ltid * ITEMS;
+    unsigned v[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) v[i] = nxt[i];
+    if (t0 + TILE < hi) load_tile(t0 + TILE, nxt);
+    if constexpr (M == M_FAULT) {
+#pragma unroll
+      for (int i = 0; i < ITEMS; ++i) v[i] = rep.fault(SITE_LOAD, (long long)base + i, v[i]);
+    }
+#pragma unroll
+    for (int i = 1; i < ITEMS; ++i) v[i] += v[i - 1];  // thread-local inclusive scan
+    const unsigned tsum = v[ITEMS - 1];
+    unsigned ws = tsum;  // logical-warp inclusive scan of thread totals
 #pragma unroll
     for (int d = 1; d < LW; d <<= 1) {
-      unsigned u = rep.lshfl_up(inc, d);
-      if (rep.llane >= d) inc += u;
+      const unsigned u = rep.lshfl_up(ws, d);
+      if (rep.llane >= d) ws += u;
     }
-    const unsigned agg = rep.lshfl_idx(inc, NLW - 1);
-    if (rep.llane < NLW) rep.sm(s_wtot, rep.llane) = inc - t;  // exclusive per logical warp
-    auto publish = [&](unsigned long long st, bool live_word) {
-      unsigned w2[2] = {(unsigned)st, (unsigned)(st >> 32)};
-      unsigned mask = (rep.llane == 0 && live_word) ? 3u : 0u;
-      rep.template commit<2, 2, true>(mask, 2u * tile, w2, 2u * (unsigned)((a.n + TILE - 1) / TILE),
-                                      [&](unsigned idx, unsigned m, const unsigned* w) {
-                                        if (m == 3u)
-                                          st_relaxed64(a.status + idx / 2,
-                                                       (unsigned long long)w[0] | ((unsigned long long)w[1] << 32));
-                                      });
-    };
-    unsigned excl = 0;
-    if (tile == 0) {
-      publish(FLAG_INC | agg, true);
-    } else {
-      publish(FLAG_AGG | agg, true);
-      // decoupled look-back over a window of LW predecessors
-      int p = (int)tile - 1;
-      while (true) {
-        const int idx = p - rep.llane;
-        unsigned long long st;
-        while (true) {  // warp-uniform spin until the whole window is valid
-          st = idx >= 0 ? ld_relaxed64(a.status + idx) : FLAG_INC;
-          // Intra: the pair shares one status load (replicated input, load path
-          // outside the SoR) so both replicas take identical control flow.
-          if constexpr (Rep<V, M>::INTRA) st = __shfl_sync(FULL, st, rep.lane & ~1);
-          if (__ballot_sync(FULL, (st >> 32) == 0ull) == 0u) break;
-        }
-        const unsigned incmask = rep.lballot((st >> 32) == 2ull);
-        const int stop = incmask ? __ffs(incmask) - 1 : LW - 1;  // closest inclusive predecessor
-        unsigned contrib = rep.llane <= stop ? (unsigned)st : 0u;
+    if (rep.llane == LW - 1) rep.sm(sw, lw) = ws;
+    __syncthreads();
+    unsigned wt = rep.llane < NLW ? rep.sm(sw, rep.llane) : 0u;  // every warp scans the warp totals
+    if constexpr (M == M_FAULT) wt = rep.fault(SITE_SMEM, (long long)ch * BL + rep.llane * LW, wt);
+    unsigned winc = wt;
 #pragma unroll
-        for (int m = LW / 2; m >= 1; m >>= 1) contrib += rep.lshfl_xor(contrib, m);
-        excl += contrib;
-        if (incmask) break;
-        p -= LW;
+    for (int d = 1; d < NLW; d <<= 1) {
+      const unsigned u = rep.lshfl_up(winc, d);
+      if (rep.llane >= d) winc += u;
+    }
+    const unsigned wexcl = rep.lshfl_idx(winc - wt, lw);
+    const unsigned total = rep.lshfl_idx(winc, NLW - 1);
+    __syncthreads();  // sw is reused by the next tile
+    const unsigned prefix = carry + wexcl + (ws - tsum);
+#pragma unroll
+    for (int q = 0; q < ITEMS / 4; ++q) {
+      const unsigned e0 = base + 4 * q;
+      unsigned w[4];
+      unsigned mask = 0;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        w[k] = prefix + v[4 * q + k];
+        mask |= (e0 + k < hi ? 1u : 0u) << k;
       }
-      publish(FLAG_INC | (excl + agg), true);
+      rep.template commit<4, 0>(mask, mask ? e0 : 0u, w, a.n, [&](unsigned idx, unsigned m, const unsigned* x) {
+        if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.y + idx), make_uint4(x[0], x[1], x[2], x[3]));
+        else
+          for (int k = 0; k < 4; ++k)
+            if ((m >> k) & 1u) a.y[idx + k] = x[k];
+      });
     }
-    if (rep.llane == 0) rep.sm(s_bcast, 0) = excl;
-  }
-  __syncthreads();
-  const unsigned prefix = rep.sm(s_bcast, 0) + rep.sm(s_wtot, lw) + (ws - tsum);
-#pragma unroll
-  for (int q = 0; q < ITEMS / 4; ++q) {
-    const unsigned e0 = base + 4 * q;
-    unsigned w[4];
-    unsigned mask = 0;
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      w[k] = prefix + v[4 * q + k];
-      mask |= (e0 + k < a.n ? 1u : 0u) << k;
-    }
-    rep.template commit<4, 0>(mask, e0, w, a.n, [&](unsigned idx, unsigned m, const unsigned* x) {
-      if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.y + idx), make_uint4(x[0], x[1], x[2], x[3]));
-      else
-        for (int k = 0; k < 4; ++k)
-          if ((m >> k) & 1u) a.y[idx + k] = x[k];
-    });
+    carry += total;
   }
   rep.finish();
 }
@@ -159,23 +194,23 @@ int prefixsum_validate(const rmt_bufs_t* b, int64_t n) {
   }
   return RMT_OK;
 }
-size_t prefixsum_scratch(int64_t n, const int64_t*) {
-  size_t tiles = (size_t)((n + TILE - 1) / TILE);
-  return 256 + tiles * 8;
-}
+size_t prefixsum_scratch(int64_t, const int64_t*) { return NCH * 4; }
 int prefixsum_inter_warps(int64_t, const int64_t*) { return BL / 32; }
 
 int prefixsum_run(Launch& L) {
-  unsigned n = (unsigned)L.n;
-  unsigned G = (n + TILE - 1) / TILE;
-  if (G == 0) return RMT_OK;
-  int rc = cuda_check(cudaMemsetAsync(L.scratch, 0, L.scratch_bytes, L.stream), "prefixsum: reset status");
-  if (rc) return rc;
-  PsArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr,
-           (unsigned long long*)(L.scratch + 256), (unsigned*)L.scratch, n};
+  const unsigned n = (unsigned)L.n;
+  if (n == 0) return RMT_OK;
+  const unsigned tiles = (n + TILE - 1) / TILE;
+  const unsigned tiles_per_chunk = (tiles + NCH - 1) / NCH;
+  const unsigned chunk = tiles_per_chunk * TILE;
+  const unsigned nch = (n + chunk - 1) / chunk;
+  PsArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, (unsigned*)L.scratch, n, chunk, nch};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
-    return launch_std<V>(L, ps_kernel<V, M>, ps_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "prefixsum");
+    int rc = launch_std<V>(L, ps_reduce_kernel<V, M>, ps_reduce_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a,
+                           "prefixsum/reduce");
+    if (rc) return rc;
+    return launch_std<V>(L, ps_scan_kernel<V, M>, ps_scan_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a, "prefixsum/scan");
   });
 }
 

@@ -1,66 +1,82 @@
 // k_transpose.cu -- MatrixTranspose (BASELINE.json configs[1]; not one of the
 // paper's 16 kernels).  B[j][i] = A[i][j], 32-bit words.
-// 64x64 tile staged in (duplicated, +LDS P:197) shared memory; 16-B coalesced
-// loads and stores; one vector commit per 4 output words.
+//
+// A logical CTA moves a 32-row x 128-column strip of A as four 32x32 tiles
+// through (duplicated, +LDS P:197) shared memory: 16-B coalesced loads of A
+// rows, scalar smem stores into a 33-word-pitch tile, scalar smem loads down
+// tile columns, 16-B coalesced stores of B rows -- one vector commit per 4
+// output words.  Bank mapping (per warp): load phase r + 4l' + k, store phase
+// 4l'' + k + c, both 32 distinct banks; for the intra variants the replica
+// planes are 2 words apart mod 4, so the two replicas of every pair also land
+// in disjoint banks (conflict-free in every variant).
 #include "rmt_host.cuh"
 
 namespace rmt {
 namespace {
 
 constexpr int BL = 256;
-constexpr int TILE = 64;
-constexpr int PITCH = TILE + 1;
+constexpr int TS = 32;          // tile side
+constexpr int NT = 4;           // tiles per logical CTA (along A's columns)
+constexpr int PITCH = TS + 1;
+constexpr int TWORDS = TS * PITCH;
+constexpr int SWORDS = NT * TWORDS;
+constexpr int PLANE = SWORDS + 2;  // replica plane offset: == 2 (mod 4)
 
 struct TrArgs {
   const unsigned* A;
   unsigned* B;
   unsigned H, W;     // A is H x W
-  unsigned ntx;      // tiles along W
+  unsigned nsx;      // strips along W
 };
 
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) tr_kernel(TrArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned tile[TILE * PITCH * DUP];
+  __shared__ unsigned tile[DUP == 2 ? PLANE + SWORDS : SWORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned ty = (unsigned)rep.lblock / a.ntx, tx = (unsigned)rep.lblock % a.ntx;
-  const unsigned c4 = (rep.ltid % 16) * 4;
-  const unsigned r0 = rep.ltid / 16;
-  // load A tile: rows ty*64 + r, cols tx*64 + c4..c4+3
+  const unsigned ty = (unsigned)rep.lblock / a.nsx, sx = (unsigned)rep.lblock % a.nsx;
+  const unsigned r = rep.ltid / 8, l4 = (rep.ltid % 8) * 4;
+  // load phase: A row ty*32 + r, columns sx*128 + 32t + l4 .. +3
+  uint4 v[NT];
+  const unsigned gi = ty * TS + r;
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    unsigned r = r0 + 16 * q;
-    unsigned gi = ty * TILE + r, gj = tx * TILE + c4;
-    uint4 v = make_uint4(0, 0, 0, 0);
-    if (gi < a.H && gj < a.W) v = __ldcs(reinterpret_cast<const uint4*>(a.A + (size_t)gi * a.W + gj));
-    unsigned w[4] = {v.x, v.y, v.z, v.w};
+  for (int t = 0; t < NT; ++t) {
+    const unsigned gj = sx * (NT * TS) + t * TS + l4;
+    v[t] = (gi < a.H && gj < a.W) ? __ldcs(reinterpret_cast<const uint4*>(a.A + (size_t)gi * a.W + gj))
+                                  : make_uint4(0, 0, 0, 0);
+  }
+#pragma unroll
+  for (int t = 0; t < NT; ++t) {
+    unsigned w[4] = {v[t].x, v[t].y, v[t].z, v[t].w};
+    const unsigned gj = sx * (NT * TS) + t * TS + l4;
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
       if constexpr (M == M_FAULT) w[k] = rep.fault(SITE_LOAD, (long long)gi * a.W + gj + k, w[k]);
-      rep.sm(tile, r * PITCH + c4 + k) = w[k];
+      rep.template smp<PLANE>(tile, t * TWORDS + r * PITCH + l4 + k) = w[k];
     }
   }
   __syncthreads();
-  // store B tile: B row = tx*64 + r (a column of A), cols ty*64 + c4..c4+3
+  // store phase: B row sx*128 + 32t + c (= a column of A), columns ty*32 + l4 .. +3
+  const unsigned cc = rep.ltid / 8;
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    unsigned r = r0 + 16 * q;
-    unsigned bi = tx * TILE + r, bj = ty * TILE + c4;
-    unsigned v[4];
+  for (int t = 0; t < NT; ++t) {
+    const unsigned bi = sx * (NT * TS) + t * TS + cc, bj = ty * TS + l4;
+    unsigned w[4];
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      v[k] = rep.sm(tile, (c4 + k) * PITCH + r);
-      if constexpr (M == M_FAULT) v[k] = rep.fault(SITE_SMEM, (long long)bi * a.H + bj + k, v[k]);
+      w[k] = rep.template smp<PLANE>(tile, t * TWORDS + (l4 + k) * PITCH + cc);
+      if constexpr (M == M_FAULT) w[k] = rep.fault(SITE_SMEM, (long long)bi * a.H + bj + k, w[k]);
     }
-    unsigned mask = (bi < a.W && bj < a.H) ? 0xFu : 0u;
-    rep.template commit<4, 0>(mask, bi * a.H + bj, v, a.H * a.W, [&](unsigned idx, unsigned m, const unsigned* w) {
-      if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.B + idx), make_uint4(w[0], w[1], w[2], w[3]));
-      else
-        for (int k = 0; k < 4; ++k)
-          if ((m >> k) & 1u) a.B[idx + k] = w[k];
-    });
+    const unsigned mask = (bi < a.W && bj < a.H) ? 0xFu : 0u;
+    rep.template commit<4, 0>(mask, mask ? bi * a.H + bj : 0u, w, a.H * a.W,
+                              [&](unsigned idx, unsigned m, const unsigned* x) {
+                                if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.B + idx), make_uint4(x[0], x[1], x[2], x[3]));
+                                else
+                                  for (int k = 0; k < 4; ++k)
+                                    if ((m >> k) & 1u) a.B[idx + k] = x[k];
+                              });
   }
   rep.finish();
 }
@@ -82,11 +98,11 @@ int transpose_inter_warps(int64_t, const int64_t*) { return BL / 32; }
 
 int transpose_run(Launch& L) {
   unsigned H = (unsigned)L.bufs->dims[0], W = (unsigned)L.bufs->dims[1];
-  unsigned ntx = (W + TILE - 1) / TILE, nty = (H + TILE - 1) / TILE;
-  TrArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, H, W, ntx};
+  unsigned nsx = (W + NT * TS - 1) / (NT * TS), nty = (H + TS - 1) / TS;
+  TrArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, H, W, nsx};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
-    return launch_std<V>(L, tr_kernel<V, M>, tr_kernel<V_NONE, M_NORMAL>, ntx * nty, BL, 0, a, "transpose");
+    return launch_std<V>(L, tr_kernel<V, M>, tr_kernel<V_NONE, M_NORMAL>, nsx * nty, BL, 0, a, "transpose");
   });
 }
 
