@@ -33,17 +33,53 @@ __device__ __forceinline__ float sqrt_approx(float x) {
   return r;
 }
 
-// One channel: biased 16-bit lanes gxb, gyb (value + 1024) -> output byte in the
-// low 8 bits of the returned word.
-__device__ __forceinline__ unsigned sobel_mag(unsigned gxb, unsigned gyb) {
-  const int gx = (int)gxb - 1024, gy = (int)gyb - 1024;
-  // s = gx^2 + gy^2 < 2^21; float(s) exactly via the 2^23 magic
-  const unsigned sm = (unsigned)(gx * gx) + (unsigned)(gy * gy) + 0x4B000000u;
-  const float f = __fmaf_rn(__uint_as_float(sm), 0.25f, 0.125f - 2097152.0f);  // s/4 + 1/8, exact
-  float r = fminf(sqrt_approx(f), 255.25f);
-  r = __fadd_rn(r, -0.5f);
-  r = __fadd_rn(r, 12582912.0f);  // round-to-nearest of r - 1/2 = floor(r)
-  return __float_as_uint(r) & 0xFFu;
+// Packed fp32x2 helpers (Blackwell FADD2/FFMA2/FMUL2).
+typedef unsigned long long f2_t;
+__device__ __forceinline__ f2_t f2(unsigned lo, unsigned hi) {
+  f2_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "r"(lo), "r"(hi));
+  return r;
+}
+__device__ __forceinline__ void f2_split(f2_t v, unsigned& lo, unsigned& hi) {
+  asm("mov.b64 {%0, %1}, %2;" : "=r"(lo), "=r"(hi) : "l"(v));
+}
+__device__ __forceinline__ f2_t add2(f2_t a, f2_t b) {
+  f2_t r;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+__device__ __forceinline__ f2_t mul2(f2_t a, f2_t b) {
+  f2_t r;
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+  return r;
+}
+__device__ __forceinline__ f2_t fma2(f2_t a, f2_t b, f2_t c) {
+  f2_t r;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+  return r;
+}
+
+// Two channels at once: gw, yw hold two biased 16-bit lanes (value + 1024) of
+// Gx and Gy.  Returns two words whose low byte is the output of the low / high
+// lane channel.  s = Gx^2 + Gy^2 < 2^21 is exact in fp32; out = min(255,
+// floor(sqrt_approx(s/4 + 1/8))) (exact: see the header).  The 16-bit lanes
+// become floats through the 2^23 magic (PRMT + FADD2), no conversion pipe.
+__device__ __forceinline__ void sobel_mag2(unsigned gw, unsigned yw, unsigned& out_lo, unsigned& out_hi) {
+  const unsigned MAG = 0x4B000000u;
+  const f2_t gx = add2(f2(__byte_perm(gw, MAG, 0x7610), __byte_perm(gw, MAG, 0x7632)),
+                       f2(__float_as_uint(-8389632.0f), __float_as_uint(-8389632.0f)));  // -(2^23 + 1024)
+  const f2_t gy = add2(f2(__byte_perm(yw, MAG, 0x7610), __byte_perm(yw, MAG, 0x7632)),
+                       f2(__float_as_uint(-8389632.0f), __float_as_uint(-8389632.0f)));
+  const f2_t ss = fma2(gx, gx, mul2(gy, gy));
+  const f2_t f = fma2(ss, f2(__float_as_uint(0.25f), __float_as_uint(0.25f)),
+                      f2(__float_as_uint(0.125f), __float_as_uint(0.125f)));  // s/4 + 1/8, exact
+  unsigned f0, f1;
+  f2_split(f, f0, f1);
+  const float r0 = fminf(sqrt_approx(__uint_as_float(f0)), 255.25f);
+  const float r1 = fminf(sqrt_approx(__uint_as_float(f1)), 255.25f);
+  f2_t r = add2(f2(__float_as_uint(r0), __float_as_uint(r1)), f2(__float_as_uint(-0.5f), __float_as_uint(-0.5f)));
+  r = add2(r, f2(__float_as_uint(12582912.0f), __float_as_uint(12582912.0f)));  // RN(r - 1/2) = floor(r)
+  f2_split(r, out_lo, out_hi);
 }
 
 struct Row {
@@ -71,8 +107,8 @@ __device__ __forceinline__ void load_row(const Rep<V, M>& rep, const SobArgs& a,
   }
 #pragma unroll
   for (int k = 0; k < 6; ++k) {
-    R.lo[k] = p[k] & 0x00FF00FFu;
-    R.hi[k] = (p[k] >> 8) & 0x00FF00FFu;
+    R.lo[k] = __byte_perm(p[k], 0u, 0x4240);  // channels 0, 2 -> 16-bit lanes
+    R.hi[k] = __byte_perm(p[k], 0u, 0x4341);  // channels 1, 3
   }
 }
 
@@ -85,19 +121,18 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) sobel_kernel(SobArgs a, Ctx
   const unsigned x0 = (bx * BL + (unsigned)rep.ltid) * 4;
   const bool active = x0 < a.W;
   const int y0 = (int)(by * RY);
-  Row top, mid, bot;
-  load_row(rep, a, y0 - 1, x0, active, top);
-  load_row(rep, a, y0, x0, active, mid);
-#pragma unroll 1
-  for (int y = y0; y < y0 + RY; ++y) {
-    load_row(rep, a, y + 1, x0, active, bot);
+  unsigned xin = 0;  // interior columns among this thread's 4 pixels (loop-invariant)
+#pragma unroll
+  for (int p = 0; p < 4; ++p) xin |= ((x0 + p >= 1 && x0 + p < a.W - 1) ? 1u : 0u) << p;
+  // one output row from the window (t = y-1, m = y, b = y+1)
+  auto row_out = [&](int y, const Row& t, const Row& m, const Row& b) {
     unsigned vs_lo[6], vs_hi[6], vd_lo[6], vd_hi[6];
 #pragma unroll
     for (int k = 0; k < 6; ++k) {
-      vs_lo[k] = top.lo[k] + 2u * mid.lo[k] + bot.lo[k];   // <= 1020 per lane
-      vs_hi[k] = top.hi[k] + 2u * mid.hi[k] + bot.hi[k];
-      vd_lo[k] = top.lo[k] + 0x01000100u - bot.lo[k];      // 256 + (top - bot)
-      vd_hi[k] = top.hi[k] + 0x01000100u - bot.hi[k];
+      vs_lo[k] = t.lo[k] + 2u * m.lo[k] + b.lo[k];   // <= 1020 per lane
+      vs_hi[k] = t.hi[k] + 2u * m.hi[k] + b.hi[k];
+      vd_lo[k] = t.lo[k] + 0x01000100u - b.lo[k];    // 256 + (top - bot)
+      vd_hi[k] = t.hi[k] + 0x01000100u - b.hi[k];
     }
     const bool yin = y >= 1 && y < (int)a.H - 1;
     unsigned out[4];
@@ -106,27 +141,33 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) sobel_kernel(SobArgs a, Ctx
       const int w = p + 1;
       // biased by 1024 per 16-bit lane
       unsigned gx_lo = vd_lo[w - 1] + 2u * vd_lo[w] + vd_lo[w + 1];
-      unsigned gx_hi = vd_hi[w - 1] + 2u * vd_hi[w] + vd_hi[w + 1];
+      const unsigned gx_hi = vd_hi[w - 1] + 2u * vd_hi[w] + vd_hi[w + 1];
       const unsigned gy_lo = vs_lo[w - 1] + 0x04000400u - vs_lo[w + 1];
       const unsigned gy_hi = vs_hi[w - 1] + 0x04000400u - vs_hi[w + 1];
       if constexpr (M == M_FAULT) gx_lo = rep.fault(SITE_COMPUTE, (long long)y * a.W + x0 + p, gx_lo);
-      const unsigned o0 = sobel_mag(gx_lo & 0xFFFFu, gy_lo & 0xFFFFu);
-      const unsigned o2 = sobel_mag(gx_lo >> 16, gy_lo >> 16);
-      const unsigned o1 = sobel_mag(gx_hi & 0xFFFFu, gy_hi & 0xFFFFu);
-      const unsigned o3 = sobel_mag(gx_hi >> 16, gy_hi >> 16);
-      const unsigned x = x0 + p;
-      const bool in = yin && x >= 1 && x < a.W - 1;
-      out[p] = in ? (o0 | (o1 << 8) | (o2 << 16) | (o3 << 24)) : 0u;
+      unsigned m0, m2, m1, m3;
+      sobel_mag2(gx_lo, gy_lo, m0, m2);  // channels 0, 2
+      sobel_mag2(gx_hi, gy_hi, m1, m3);  // channels 1, 3
+      const unsigned px = __byte_perm(__byte_perm(m0, m1, 0x0040), __byte_perm(m2, m3, 0x0040), 0x5410);
+      out[p] = (yin && ((xin >> p) & 1u)) ? px : 0u;
     }
     const unsigned mask = (active && y < (int)a.H) ? 0xFu : 0u;
     rep.template commit<4, 0>(mask, (unsigned)y * a.W + x0, out, a.H * a.W,
-                              [&](unsigned idx, unsigned m, const unsigned* w) {
-                                if (m == 0xFu)
+                              [&](unsigned idx, unsigned mm, const unsigned* w) {
+                                if (mm == 0xFu)
                                   __stcs(reinterpret_cast<uint4*>(a.O + idx), make_uint4(w[0], w[1], w[2], w[3]));
                                 else
                                   for (int k = 0; k < 4; ++k)
-                                    if ((m >> k) & 1u) a.O[idx + k] = w[k];
+                                    if ((mm >> k) & 1u) a.O[idx + k] = w[k];
                               });
+  };
+  Row top, mid, bot;
+  load_row(rep, a, y0 - 1, x0, active, top);
+  load_row(rep, a, y0, x0, active, mid);
+#pragma unroll 1
+  for (int y = y0; y < y0 + RY; ++y) {
+    load_row(rep, a, y + 1, x0, active, bot);
+    row_out(y, top, mid, bot);
     top = mid;
     mid = bot;
   }
