@@ -119,37 +119,28 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_kernel(BsArgs a, Ctx c
   // Groups of 4 logical lanes descend together: for each of the group's 16
   // queries the 4 members load one 16-B quarter of the same 64-B block, so a
   // warp-wide load touches one cache line per query (1 L1 wavefront instead
-  // of 4).  Every lane tracks the block index J[i][s] of all 16 queries.
+  // of 4).  Each lane tracks the block base of its OWN 4 queries and fetches the
+  // other members' bases by shuffle.
   const int gm = rep.llane & 3;
   const int g0 = rep.llane & ~3;
-  unsigned K[4][VEC], J[4][VEC];
+  unsigned K[4][VEC];
 #pragma unroll
   for (int i = 0; i < 4; ++i)
 #pragma unroll
-    for (int s = 0; s < VEC; ++s) {
-      K[i][s] = rep.lshfl_idx(key[s], g0 + i);
-      J[i][s] = a.N ? 1u : 0u;  // "block 0" of the top level
-    }
-  for (int lv = a.L.T; lv >= 0; --lv) {
-    const unsigned* P = lv ? a.lev + a.L.off[lv] : a.A;
-    const unsigned lim = lv ? a.L.padded[lv] : a.N;
-    if constexpr (M == M_FAULT) {
-      if (lv == a.L.T - 1) {  // control-flow fault: this lane's copy of a block index
+    for (int s = 0; s < VEC; ++s) K[i][s] = rep.lshfl_idx(key[s], g0 + i);
+  unsigned jj[VEC];
 #pragma unroll
-        for (int s = 0; s < VEC; ++s) {
-          const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, J[gm][s]);
-          J[gm][s] = f > a.L.n[lv + 1] ? a.L.n[lv + 1] : f;
-        }
-      }
-    }
-    // b = max(J,1) - 1: when J = 0 (key <= every entry) block 0 counts 0, so J stays 0.
-    const bool tail = (lv == 0);  // only the caller's A is unpadded
+  for (int s = 0; s < VEC; ++s) jj[s] = a.N ? 1u : 0u;  // "block 0" of the top level
+  // one level: J <- 16 (max(J,1) - 1) + #{block < key}.  When J = 0 (key <= every
+  // entry) block 0 counts 0, so J stays 0 with no special case.
+  auto level = [&](const unsigned* P, unsigned lim, bool tail) {
 #pragma unroll
     for (int s = 0; s < VEC; ++s) {
+      const unsigned mybase = (max(jj[s], 1u) - 1u) * FAN;
       unsigned packed = 0;
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
-        const unsigned base = (max(J[i][s], 1u) - 1u) * FAN + 4u * gm;
+        const unsigned base = rep.lshfl_idx(mybase, g0 + i) + 4u * gm;
         uint4 w;
         if (!tail || base + 4u <= lim) {
           w = __ldg(reinterpret_cast<const uint4*>(P + base));
@@ -160,17 +151,36 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_kernel(BsArgs a, Ctx c
           w.w = base + 3 < lim ? __ldg(P + base + 3) : 0xFFFFFFFFu;
         }
         const unsigned k = K[i][s];
-        packed += ((w.x < k) + (w.y < k) + (w.z < k) + (w.w < k)) << (8 * i);
+        const unsigned bits = (w.x < k ? 1u : 0u) | (w.y < k ? 2u : 0u) | (w.z < k ? 4u : 0u) | (w.w < k ? 8u : 0u);
+        packed += (unsigned)__popc(bits) << (8 * i);
       }
       packed += rep.lshfl_xor(packed, 1);  // sum the 4 quarters (bytes <= 16: no carries)
       packed += rep.lshfl_xor(packed, 2);
+      jj[s] = mybase + ((packed >> (8 * gm)) & 0xFFu);
+    }
+  };
+  for (int lv = a.L.T; lv >= 1; --lv) {  // padded sample levels: no bounds checks
+    if constexpr (M == M_FAULT) {
+      if (lv == a.L.T - 1) {  // control-flow fault: a flipped block index, kept in range
 #pragma unroll
-      for (int i = 0; i < 4; ++i) J[i][s] = (max(J[i][s], 1u) - 1u) * FAN + ((packed >> (8 * i)) & 0xFFu);
+        for (int s = 0; s < VEC; ++s) {
+          const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, jj[s]);
+          jj[s] = f > a.L.n[lv + 1] ? a.L.n[lv + 1] : f;
+        }
+      }
+    }
+    level(a.lev + a.L.off[lv], a.L.padded[lv], false);
+  }
+  if constexpr (M == M_FAULT) {
+    if (a.L.T == 1) {
+#pragma unroll
+      for (int s = 0; s < VEC; ++s) {
+        const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, jj[s]);
+        jj[s] = f > a.L.n[1] ? a.L.n[1] : f;
+      }
     }
   }
-  unsigned jj[VEC];
-#pragma unroll
-  for (int s = 0; s < VEC; ++s) jj[s] = J[gm][s];
+  level(a.A, a.N, true);  // the caller's A
   rep.template commit<VEC, 0>(mask, j0, jj, a.Q, [&](unsigned i, unsigned m, const unsigned* w) {
     if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.idx + i), make_uint4(w[0], w[1], w[2], w[3]));
     else
