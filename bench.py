@@ -44,6 +44,8 @@ def parse():
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--variants", default=",".join(VARIANTS))
+    p.add_argument("--dist-backend", default="nccl",
+                   help="nccl (one GPU per rank); gloo only to exercise the multi-rank path on one GPU")
     return p.parse_args()
 
 
@@ -207,23 +209,47 @@ def main():
 
     from paper_conf_isca_waddenlgss14_b200 import rmt
 
-    torch.cuda.set_device(local_rank)
+    dev_index = local_rank % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(dev_index)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev_index))
+        else:
+            dist.init_process_group(args.dist_backend)
     variants = [v for v in args.variants.split(",") if v]
     jobs = workloads.config_jobs(args.config, rank)
     stream = torch.cuda.current_stream()
     err = torch.zeros(1, dtype=torch.int64, device="cuda")
     ws = {}
+    ws_red = {}
     for j in jobs:
         j.device_buffers()
         for v in variants:
             ws[(j.kernel, v)] = rmt.make_workspace(j.kernel, v, j.n, j.dims)
+            if j.kernel == "prefixsum":
+                ws_red[v] = rmt.make_workspace("reduction", v, j.n)
     torch.cuda.synchronize()
 
     launches = [(j, v) for j in jobs for v in variants]
     ev = {(j.kernel, v): [] for j, v in launches}
     counts = {"gpu_launches": 0}
+
+    from paper_conf_isca_waddenlgss14_b200 import parallel
+    s_tmp = torch.zeros(2, dtype=torch.int32, device="cuda")
+
+    def one(j, v):
+        """One launch of job j under variant v; for N > 1 the kernels that need a
+        cross-shard exchange do it here."""
+        if world > 1 and j.kernel == "prefixsum":
+            # local total (Reduction kernel) -> all-gather -> carry-in -> scan
+            parallel.global_prefixsum(j.dev[0], j.dev[1], s_tmp, err, rmt, variant=v,
+                                      ws_red=ws_red[v], ws_ps=ws[(j.kernel, v)])
+            return 2
+        nk = rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=ws[(j.kernel, v)],
+                        stream=stream.cuda_stream)
+        if world > 1 and j.kernel == "reduction":
+            parallel.allreduce_sum_(j.dev[1].view(torch.int64))
+        return nk
 
     def step(timed):
         for j, v in launches:
@@ -231,15 +257,13 @@ def main():
                 a = torch.cuda.Event(enable_timing=True)
                 b = torch.cuda.Event(enable_timing=True)
                 a.record(stream)
-            nk = rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=ws[(j.kernel, v)],
-                            stream=stream.cuda_stream)
+            nk = one(j, v)
             if timed:
                 b.record(stream)
                 ev[(j.kernel, v)].append((a, b))
                 counts["gpu_launches"] += nk
         if world > 1:
-            # the only data-path collectives: error counters and the Reduction result
-            dist.all_reduce(err)
+            parallel.allreduce_sum_(err)  # error counters of every rank
 
     for _ in range(args.warmup):
         step(False)
@@ -250,7 +274,7 @@ def main():
     torch.cuda.synchronize()
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local_rank) as clk:
+    with ClockSampler(dev_index) as clk:
         t0.record(stream)
         for _ in range(args.steps):
             step(True)

@@ -89,7 +89,8 @@ typedef struct {
  *   BLACKSCHOLES  buf {r:F32[n], call:F32[n], put:F32[n]}           n = options
  *   BINARYSEARCH  buf {A:U32[N] sorted, q:U32[Q], idx:U32[Q]}       n = Q, dims {N, Q}
  *   FWT           buf {x:F32[N], y:F32[N]}                          n = N = 2^m
- *   PREFIXSUM     buf {x:U32[n], y:U32[n]}  inclusive, mod 2^32     n
+ *   PREFIXSUM     buf {x:U32[n], y:U32[n]}  inclusive, mod 2^32     n, dims {carry_in} (u32 added
+ *                 to every y: the exclusive prefix of earlier shards in a multi-GPU scan; 0 = none)
  *   REDUCTION     buf {x:U32[n], s:U64[1]}                          n
  *   TRANSPOSE     buf {A:U32|F32[H*W], B:same[W*H]}                 n = H*W, dims {H, W}, H%4 = W%4 = 0
  *   SOBEL         buf {I:U8X4[H*W], O:U8X4[H*W]}                    n = H*W, dims {H, W}, W%4 = 0

@@ -31,6 +31,7 @@ struct PsArgs {
   unsigned n;
   unsigned chunk;      // elements per chunk (multiple of TILE)
   unsigned nch;        // chunks actually used
+  unsigned carry_in;   // added to every output (multi-GPU shard offset)
 };
 
 // u32 sum over the logical CTA (logical warps + duplicated smem)
@@ -109,7 +110,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ct
   // carry-in: sum of the partials of all earlier chunks (L2-resident)
   unsigned cs = 0;
   for (unsigned i = rep.ltid; i < ch; i += BL) cs += __ldcg(a.partial + i);
-  unsigned carry = block_sum_u32(rep, cs, sw);
+  unsigned carry = a.carry_in + block_sum_u32(rep, cs, sw);
   const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
   const int lw = rep.ltid / LW;
   // register double buffer: the next tile's loads are in flight while this
@@ -204,7 +205,8 @@ int prefixsum_run(Launch& L) {
   const unsigned tiles_per_chunk = (tiles + NCH - 1) / NCH;
   const unsigned chunk = tiles_per_chunk * TILE;
   const unsigned nch = (n + chunk - 1) / chunk;
-  PsArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, (unsigned*)L.scratch, n, chunk, nch};
+  PsArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, (unsigned*)L.scratch, n, chunk, nch,
+           (unsigned)(L.bufs->dims[0] & 0xFFFFFFFFu)};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     int rc = launch_std<V>(L, ps_reduce_kernel<V, M>, ps_reduce_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a,

@@ -92,3 +92,18 @@ def test_fault_is_live_in_none(case):
         rmt.clear_faults()
     assert err == 0
     assert any(not np.array_equal(a, b) for a, b in zip(outs, ref))
+
+
+@pytest.mark.parametrize("variant", ["none"] + list(rmt.RMT_VARIANTS))
+def test_prefixsum_carry_in(variant):
+    """The multi-GPU shard offset (dims[0] = carry-in) is added to every output."""
+    import oracle
+    from cases import PrefixSum
+    c = PrefixSum(4096 * 5 + 7)
+    carry = 0xFFFFFF00
+    b = c.buffers()
+    err = run("prefixsum", variant, b, c.n, dims=(carry,))
+    assert err == 0
+    y = c.outputs(b)[0].astype(np.uint64)
+    ref = (oracle.prefixsum_u32(c.x).astype(np.uint64) + carry) % 2**32
+    assert np.array_equal(y, ref)
