@@ -93,7 +93,8 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
 }
 
 template <int V, int M>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_kernel(BsArgs a, Ctx c) {
+// Intra variants: 512-thread CTAs would hold 72 registers (1 CTA/SM); cap at 40.
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 3 : 4) bins_kernel(BsArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
