@@ -44,6 +44,8 @@ def parse():
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--variants", default=",".join(VARIANTS))
+    p.add_argument("--ablations", action="store_true",
+                   help="also time the INFLATE and NOCOMM ablations per kernel x RMT variant (cost attribution)")
     p.add_argument("--dist-backend", default="nccl",
                    help="nccl (one GPU per rank); gloo only to exercise the multi-rank path on one GPU")
     return p.parse_args()
@@ -361,6 +363,40 @@ def main():
                "h2d_bytes_per_step": h2d // args.e2e_steps, "d2h_bytes_per_step": d2h // args.e2e_steps,
                "ms_per_step": round(ems / args.e2e_steps, 3)}
 
+    # Cost attribution "as the paper does": t(none) ->
+    # inflate (none with the RMT variant's per-SM residency: redundant scheduling)
+    # -> nocomm (both replicas, no exchange: redundant compute) -> full (+ comm).
+    attribution = None
+    if args.ablations:
+        attribution = {}
+        for j in jobs:
+            d = {}
+            for v in [x for x in variants if x != "none"]:
+                row = {}
+                for mode in ("inflate", "nocomm", "full"):
+                    rmt.set_ablation(mode)
+                    ts = []
+                    for r in range(4):
+                        a = torch.cuda.Event(enable_timing=True)
+                        b = torch.cuda.Event(enable_timing=True)
+                        a.record(stream)
+                        rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=ws[(j.kernel, v)],
+                                   stream=stream.cuda_stream)
+                        b.record(stream)
+                        torch.cuda.synchronize()
+                        if r:
+                            ts.append(a.elapsed_time(b))
+                    row[mode] = statistics.median(ts)
+                rmt.set_ablation("full")
+                base = per[(j.kernel, "none")]
+                row = {k: round(x, 4) for k, x in row.items()}
+                row["scheduling"] = round(row["inflate"] / base - 1, 3)
+                row["redundant_compute"] = round((row["nocomm"] - row["inflate"]) / base, 3)
+                row["communication"] = round((row["full"] - row["nocomm"]) / base, 3)
+                d[v] = row
+            attribution[j.kernel] = d
+        err.zero_()
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rate, secs, cores, desc = oracle_sample_rate(jobs)
@@ -380,6 +416,7 @@ def main():
                                "gbs": kernels[best_none.kernel]["none"]["gbs"],
                                "frac": kernels[best_none.kernel]["none"]["frac"]} if best_none else None),
             "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "attribution": attribution,
             "gpu_launches": counts["gpu_launches"], "err_count": errs,
             "clocks": clk.summary(),
         }

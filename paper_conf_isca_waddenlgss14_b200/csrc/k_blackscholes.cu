@@ -23,42 +23,46 @@ struct BsArgs {
 
 // A&S 26.2.17: tail = phi(|x|) k (a1 + k(a2 + k(a3 + k(a4 + k a5)))),
 // k = 1/(1 + 0.2316419|x|);  N(x) = 1 - tail (x >= 0), tail (x < 0).
+// phi(x) = exp(-x^2/2 - ln sqrt(2 pi)).
 __device__ __forceinline__ void cnd_pair(float x, float& nx, float& nmx) {
-  float ax = fabsf(x);
-  float k = __frcp_rn(__fadd_rn(1.0f, __fmul_rn(0.2316419f, ax)));
+  const float ax = fabsf(x);
+  const float k = __fdividef(1.0f, __fmaf_rn(0.2316419f, ax, 1.0f));  // one MUFU.RCP
   float poly = __fmaf_rn(k, 1.330274429f, -1.821255978f);
   poly = __fmaf_rn(k, poly, 1.781477937f);
   poly = __fmaf_rn(k, poly, -0.356563782f);
   poly = __fmaf_rn(k, poly, 0.319381530f);
-  poly = __fmul_rn(k, poly);
-  float phi = __fmul_rn(0.398942280401432678f, __expf(__fmul_rn(-0.5f, __fmul_rn(ax, ax))));
-  float tail = __fmul_rn(phi, poly);
-  float body = __fsub_rn(1.0f, tail);
+  const float phi = __expf(__fmaf_rn(__fmul_rn(-0.5f, ax), ax, -0.918938533204672742f));
+  const float tail = __fmul_rn(__fmul_rn(phi, k), poly);
+  const float body = __fsub_rn(1.0f, tail);
   nx = x >= 0.0f ? body : tail;
   nmx = x >= 0.0f ? tail : body;
 }
 
+// Explicit fp32 operations only (fixed rounding in every variant).  The
+// transcendentals are single-MUFU approximate intrinsics (rsqrt, rcp, lg2, ex2:
+// ~2 ulp each, far inside the 1e-4 tolerance, and deterministic): 9 MUFU and
+// ~35 FMA-pipe operations per option, balanced against 12 B of HBM traffic.
 template <int V, int M>
 __device__ __forceinline__ void bs_option(const Rep<V, M>& rep, float r, long long elem, float& call, float& put) {
   // R-BS1: S = K = 10r + 100(1-r), T = r + 10(1-r), R = .01r + .05(1-r), sigma = .01r + .1(1-r)
-  float omr = __fsub_rn(1.0f, r);
-  float S = __fadd_rn(__fmul_rn(10.0f, r), __fmul_rn(100.0f, omr));
-  float K = __fadd_rn(__fmul_rn(10.0f, r), __fmul_rn(100.0f, omr));
-  float T = __fadd_rn(r, __fmul_rn(10.0f, omr));
-  float R = __fadd_rn(__fmul_rn(0.01f, r), __fmul_rn(0.05f, omr));
-  float sig = __fadd_rn(__fmul_rn(0.01f, r), __fmul_rn(0.10f, omr));
-  float sT = __fmul_rn(sig, __fsqrt_rn(T));
+  const float S = __fmaf_rn(-90.0f, r, 100.0f);
+  const float K = __fmaf_rn(-90.0f, r, 100.0f);
+  const float T = __fmaf_rn(-9.0f, r, 10.0f);
+  const float R = __fmaf_rn(-0.04f, r, 0.05f);
+  const float sig = __fmaf_rn(-0.09f, r, 0.10f);
+  const float rsT = rsqrtf(T);
+  const float sT = __fmul_rn(__fmul_rn(sig, T), rsT);  // sigma sqrt(T)
   // d1 = (ln(S/K) + (R + sigma^2/2) T) / (sigma sqrt T), d2 = d1 - sigma sqrt T
-  float drift = __fmul_rn(__fadd_rn(R, __fmul_rn(0.5f, __fmul_rn(sig, sig))), T);
-  float d1 = __fdiv_rn(__fadd_rn(__logf(__fdiv_rn(S, K)), drift), sT);
+  const float drift = __fmul_rn(__fmaf_rn(__fmul_rn(0.5f, sig), sig, R), T);
+  float d1 = __fmul_rn(__fadd_rn(__logf(__fdividef(S, K)), drift), __fdividef(rsT, sig));
   d1 = rep.faultf(SITE_COMPUTE, elem, d1);
-  float d2 = __fsub_rn(d1, sT);
-  float disc = __fmul_rn(K, __expf(-__fmul_rn(R, T)));
+  const float d2 = __fsub_rn(d1, sT);
+  const float disc = __fmul_rn(K, __expf(__fmul_rn(-R, T)));
   float n1, nm1, n2, nm2;
   cnd_pair(d1, n1, nm1);
   cnd_pair(d2, n2, nm2);
-  call = __fsub_rn(__fmul_rn(S, n1), __fmul_rn(disc, n2));
-  put = __fsub_rn(__fmul_rn(disc, nm2), __fmul_rn(S, nm1));
+  call = __fmaf_rn(S, n1, -__fmul_rn(disc, n2));
+  put = __fmaf_rn(disc, nm2, -__fmul_rn(S, nm1));
 }
 
 template <int V, int M>
@@ -110,9 +114,9 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bs_kernel(BsArgs a, Ctx c) 
 }  // namespace
 
 int blackscholes_validate(const rmt_bufs_t* b, int64_t n) {
-  if (b->nbuf < 3 || n < 0 || n >= (1LL << 30) || !buf_ok(b->buf[0], RMT_F32, n) ||
+  if (b->nbuf < 3 || n < 0 || n > (1LL << 30) || !buf_ok(b->buf[0], RMT_F32, n) ||
       !buf_ok(b->buf[1], RMT_F32, n) || !buf_ok(b->buf[2], RMT_F32, n)) {
-    set_error("blackscholes: expected {r,call,put} F32[n], n < 2^30, 16-B aligned");
+    set_error("blackscholes: expected {r,call,put} F32[n], n <= 2^30, 16-B aligned");
     return RMT_EINVAL;
   }
   return RMT_OK;

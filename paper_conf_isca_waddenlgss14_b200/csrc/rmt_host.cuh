@@ -98,14 +98,21 @@ namespace rmt {
 // at most `target` CTAs per SM.
 template <class K>
 size_t pad_for_occupancy(K kn, int bn, size_t sn, int target) {
-  int occ = 0;
-  for (size_t extra = 0; extra + sn <= 227 * 1024; extra += 1024) {
-    if (sn + extra > 48 * 1024)
-      cudaFuncSetAttribute(kn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sn + extra));
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kn, bn, sn + extra);
-    if (occ <= target) return extra;
+  cudaFuncAttributes fa;
+  if (cudaFuncGetAttributes(&fa, kn) != cudaSuccess) return 0;
+  const size_t cap = 227 * 1024 - fa.sharedSizeBytes;  // static + dynamic <= 227 KiB per CTA
+  size_t best = 0;
+  for (size_t extra = 0; sn + extra <= cap; extra += 1024) {
+    if (sn + extra > 48 * 1024 &&
+        cudaFuncSetAttribute(kn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(sn + extra)) != cudaSuccess)
+      break;
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kn, bn, sn + extra) != cudaSuccess || occ < 1) break;
+    best = extra;
+    if (occ <= target) break;
   }
-  return 0;
+  cudaGetLastError();  // clear any error from probing
+  return best;
 }
 
 // Standard launch of one RMT kernel instance: logical grid G of BL-thread
