@@ -10,6 +10,9 @@
 // improving relaxations write) and are committed with a per-word
 // predicate mask: (mask, address, D words) and (mask, address, P words).
 // D (n^2 u32 = 64 MiB at n = 4096) stays L2-resident across passes.
+#include <map>
+#include <tuple>
+
 #include "rmt_host.cuh"
 
 namespace rmt {
@@ -99,9 +102,11 @@ int floydwarshall_validate(const rmt_bufs_t* b, int64_t n) {
 size_t floydwarshall_scratch(int64_t, const int64_t*) { return 0; }
 int floydwarshall_inter_warps(int64_t, const int64_t*) { return BL / 32; }
 
-int floydwarshall_run(Launch& L) {
+namespace {
+
+// The n + 1 launches of one FloydWarshall call, issued on L.stream.
+int fw_issue(Launch& L) {
   const unsigned n = (unsigned)L.n;
-  if (n == 0) return RMT_OK;
   const unsigned nn = n * n;
   const unsigned G = (nn / 4 + BL - 1) / BL;
   FwArgs a{(unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, n, 0};
@@ -122,6 +127,55 @@ int floydwarshall_run(Launch& L) {
     L.ctx.f = f;
     return rc;
   });
+}
+
+// Host launch overhead (~n launches per call) would starve the GPU: the pass
+// sequence is captured once into a CUDA graph (keyed by every launch parameter)
+// and replayed on the caller's stream.  Inside a caller's capture the launches
+// are simply recorded into the caller's graph.
+typedef std::tuple<int, int, int, void*, void*, unsigned, void*, void*, void*, void*, int, int, int, int, long long>
+    FwKey;
+std::map<FwKey, cudaGraphExec_t> g_fw_graphs;
+cudaStream_t g_fw_capture_stream = nullptr;
+
+}  // namespace
+
+int floydwarshall_run(Launch& L) {
+  const unsigned n = (unsigned)L.n;
+  if (n == 0) return RMT_OK;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(L.stream, &cs) != cudaSuccess) {
+    cudaGetLastError();
+    cs = cudaStreamCaptureStatusNone;
+  }
+  if (cs != cudaStreamCaptureStatusNone || n < 64) return fw_issue(L);
+  const FaultDesc& f = L.ctx.f;
+  FwKey key{L.variant, L.mode, (int)L.inflate, L.bufs->buf[0].ptr, L.bufs->buf[1].ptr, n, (void*)L.ctx.err,
+            (void*)L.ctx.ctrl, (void*)L.ctx.flags, (void*)L.ctx.payload, f.replica, f.site, f.bit, f.sid, f.elem};
+  auto it = g_fw_graphs.find(key);
+  if (it == g_fw_graphs.end()) {
+    int rc;
+    if (!g_fw_capture_stream &&
+        (rc = cuda_check(cudaStreamCreateWithFlags(&g_fw_capture_stream, cudaStreamNonBlocking), "fw: stream")))
+      return rc;
+    Launch C = L;
+    C.stream = g_fw_capture_stream;
+    C.launches = 0;
+    if ((rc = cuda_check(cudaStreamBeginCapture(C.stream, cudaStreamCaptureModeThreadLocal), "fw: begin capture")))
+      return rc;
+    rc = fw_issue(C);
+    cudaGraph_t g = nullptr;
+    cudaError_t ec = cudaStreamEndCapture(C.stream, &g);
+    if (rc) return rc;
+    if ((rc = cuda_check(ec, "fw: end capture"))) return rc;
+    cudaGraphExec_t ge = nullptr;
+    rc = cuda_check(cudaGraphInstantiate(&ge, g, 0), "fw: instantiate");
+    cudaGraphDestroy(g);
+    if (rc) return rc;
+    it = g_fw_graphs.emplace(key, ge).first;
+  }
+  L.launches += (int)n + 1;
+  return cuda_check(cudaGraphLaunch(it->second, L.stream), "fw: graph launch");
 }
 
 }  // namespace rmt
