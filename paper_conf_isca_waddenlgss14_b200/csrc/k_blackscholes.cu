@@ -106,7 +106,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bs_kernel(BsArgs a, Ctx c) 
       }
     };
   };
-  rep.template commit<VEC, 0>(mask, i0, cv, a.n, store_to(a.call));
+  rep.template commit<VEC, 0>(mask, i0, cv, a.n, store_to(a.call), /*defer=*/true);
   rep.template commit<VEC, 1>(mask, i0, pv, a.n, store_to(a.put));
   rep.finish();
 }

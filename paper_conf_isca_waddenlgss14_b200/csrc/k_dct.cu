@@ -105,7 +105,8 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c
                                 else
                                   for (int k = 0; k < 4; ++k)
                                     if ((m >> k) & 1u) a.Y[i + k] = __uint_as_float(v[k]);
-                              });
+                              },
+                              /*defer=*/h == 0);
   }
   rep.finish();
 }

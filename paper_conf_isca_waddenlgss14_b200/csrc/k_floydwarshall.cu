@@ -51,41 +51,51 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_init_kernel(FwArgs a, Ct
   rep.finish();
 }
 
+// One pass k.  Each logical thread handles VPT 16-B vectors strided by the CTA
+// width (coalesced); fat CTAs amortise the per-CTA RMT handshakes (inter-group
+// ticket / turn / queue latency) over 8192 elements.
+constexpr int VPT = 8;
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned e0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * 4;
   const unsigned nn = a.n * a.n;
-  const bool active = e0 < nn;
-  const unsigned i = active ? e0 / a.n : 0u, j = active ? e0 - i * a.n : 0u;
-  unsigned dik = 0;
-  uint4 dkj = make_uint4(0, 0, 0, 0), dij = make_uint4(0, 0, 0, 0);
-  if (active) {
-    dik = a.D[(size_t)i * a.n + a.k];
-    dkj = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
-    dij = *reinterpret_cast<const uint4*>(a.D + e0);
-  }
-  unsigned kj[4] = {dkj.x, dkj.y, dkj.z, dkj.w};
-  unsigned ij[4] = {dij.x, dij.y, dij.z, dij.w};
-  if constexpr (M == M_FAULT) {
-    dik = rep.fault(SITE_LOAD, (long long)i * a.n + a.k, dik);
+#pragma unroll 1
+  for (int it = 0; it < VPT; ++it) {
+    const unsigned e0 = ((unsigned)rep.lblock * (BL * VPT) + (unsigned)it * BL + (unsigned)rep.ltid) * 4;
+    const bool active = e0 < nn;
+    const unsigned i = active ? e0 / a.n : 0u, j = active ? e0 - i * a.n : 0u;
+    unsigned dik = 0;
+    uint4 dkj = make_uint4(0, 0, 0, 0), dij = make_uint4(0, 0, 0, 0);
+    if (active) {
+      dik = a.D[(size_t)i * a.n + a.k];
+      dkj = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
+      dij = *reinterpret_cast<const uint4*>(a.D + e0);
+    }
+    unsigned kj[4] = {dkj.x, dkj.y, dkj.z, dkj.w};
+    unsigned ij[4] = {dij.x, dij.y, dij.z, dij.w};
+    if constexpr (M == M_FAULT) {
+      dik = rep.fault(SITE_LOAD, (long long)i * a.n + a.k, dik);
 #pragma unroll
-    for (int q = 0; q < 4; ++q) ij[q] = rep.fault(SITE_LOAD, (long long)e0 + q, ij[q]);
-  }
-  unsigned nd[4], np[4], mask = 0;
+      for (int q = 0; q < 4; ++q) ij[q] = rep.fault(SITE_LOAD, (long long)e0 + q, ij[q]);
+    }
+    unsigned nd[4], np[4], mask = 0;
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    unsigned cand = dik + kj[q];
-    if constexpr (M == M_FAULT) cand = rep.fault(SITE_COMPUTE, (long long)e0 + q, cand);
-    const bool better = active && cand < ij[q];
-    mask |= (better ? 1u : 0u) << q;
-    nd[q] = cand;
-    np[q] = a.k;
+    for (int q = 0; q < 4; ++q) {
+      unsigned cand = dik + kj[q];
+      if constexpr (M == M_FAULT) cand = rep.fault(SITE_COMPUTE, (long long)e0 + q, cand);
+      const bool better = active && cand < ij[q];
+      mask |= (better ? 1u : 0u) << q;
+      nd[q] = cand;
+      np[q] = a.k;
+    }
+    rep.template commit<4, 0>(mask, active ? e0 : 0u, nd, nn,
+                              [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); },
+                              /*defer=*/true);
+    rep.template commit<4, 1>(mask, active ? e0 : 0u, np, nn,
+                              [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
   }
-  rep.template commit<4, 0>(mask, e0, nd, nn, [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); });
-  rep.template commit<4, 1>(mask, e0, np, nn, [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
   rep.finish();
 }
 
@@ -108,7 +118,8 @@ namespace {
 int fw_issue(Launch& L) {
   const unsigned n = (unsigned)L.n;
   const unsigned nn = n * n;
-  const unsigned G = (nn / 4 + BL - 1) / BL;
+  const unsigned G = (nn / 4 + BL - 1) / BL;                // init: one vector per thread
+  const unsigned Gp = (nn / 4 + BL * VPT - 1) / (BL * VPT);  // passes: VPT vectors per thread
   FwArgs a{(unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, n, 0};
   // Fault element = k0 * n^2 + e: the pass k0 and the element e.
   const FaultDesc f = L.ctx.f;
@@ -122,7 +133,7 @@ int fw_issue(Launch& L) {
       L.ctx.f = f;
       if (k == k0) L.ctx.f.elem = f.elem - (long long)k0 * nn;
       else L.ctx.f.site = -1;
-      rc = launch_std<V>(L, fw_pass_kernel<V, M>, fw_pass_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "fw/pass");
+      rc = launch_std<V>(L, fw_pass_kernel<V, M>, fw_pass_kernel<V_NONE, M_NORMAL>, Gp, BL, 0, a, "fw/pass");
     }
     L.ctx.f = f;
     return rc;

@@ -211,7 +211,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
       else
         for (int k = 0; k < 4; ++k)
           if ((m >> k) & 1u) a.dst[idx + k] = __uint_as_float(x[k]);
-    });
+    }, /*defer=*/it < TE_MAX / (4 * BL) - 1);
   }
   rep.finish();
 }

@@ -226,7 +226,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 1) mm_kernel(const __grid_c
         else
           for (int k = 0; k < 4; ++k)
             if ((m >> k) & 1u) a.C[e + k] = __uint_as_float(x[k]);
-      });
+      }, /*defer=*/(i & 3) != 3);
     }
   }
   tc_fence_before();

@@ -179,7 +179,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ct
         else
           for (int k = 0; k < 4; ++k)
             if ((m >> k) & 1u) a.y[idx + k] = x[k];
-      });
+      }, /*defer=*/q < ITEMS / 4 - 1);
     }
     carry += total;
   }

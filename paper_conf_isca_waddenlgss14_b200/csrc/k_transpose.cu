@@ -76,7 +76,8 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) tr_kernel(TrArgs a, Ctx c) 
                                 else
                                   for (int k = 0; k < 4; ++k)
                                     if ((m >> k) & 1u) a.B[idx + k] = x[k];
-                              });
+                              },
+                              /*defer=*/t < NT - 1);
   }
   rep.finish();
 }

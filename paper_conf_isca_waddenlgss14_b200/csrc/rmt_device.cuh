@@ -131,10 +131,11 @@ struct Rep {
   int lblock;     // logical CTA id
   int lane, warp, llane;
   unsigned j;     // records this warp has committed (inter)
+  unsigned pend;  // inter: records not yet published (producer) / freed (consumer)
   unsigned region, epoch;
   unsigned* mbox;  // intra_smem: this warp's mailbox
 
-  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), region(0), epoch(0), mbox(nullptr) {}
+  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), pend(0), region(0), epoch(0), mbox(nullptr) {}
 
   // Must be called by every thread of the CTA, first thing (may __syncthreads).
   // mbox_smem: MBOX_WORDS * (blockDim/32) words of shared memory (intra_smem only).
@@ -176,9 +177,34 @@ struct Rep {
   }
 
   // Must be called by every thread of the CTA, last thing.
+  // ---- inter queue: publish / free the pending records of this warp.
+  // Producer: one fence by every lane covers all pending payloads, then lane l
+  // sets the flag of pending record l.  Consumer: lane l frees pending slot l
+  // with one release store (the ballot after every compare already consumed the
+  // loaded words).  Called at every non-deferred commit and before finish().
+  __device__ __forceinline__ size_t slot_index(unsigned rec) const {
+    return ((size_t)region * c.W + warp) * c.S + (rec % (unsigned)c.S);
+  }
+  __device__ __forceinline__ void flush() {
+    if constexpr (INTER && !NOCOMM) {
+      if (pend == 0u) return;
+      const unsigned first = j - pend;
+      if (!consumer) {
+        asm volatile("fence.sc.gpu;" ::: "memory");
+        __syncwarp();
+        if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), 1u);
+      } else {
+        __syncwarp();
+        if ((unsigned)lane < pend) st_release(c.flags + slot_index(first + lane), 0u);
+      }
+      pend = 0u;
+    }
+  }
+
   __device__ __forceinline__ void finish() {
     if constexpr (INTER) {
       __shared__ unsigned s_last;
+      flush();
       __syncthreads();
       if (threadIdx.x == 0) {
         if (consumer && !NOCOMM) st_release(c.ctrl + CTRL_TURN + region, epoch + 1);
@@ -271,9 +297,14 @@ struct Rep {
   //   SID   store-site id (faults on STORE_* sites target SID 0)
   //   LIVE  liveness-critical store (other CTAs spin on it): on a mismatch the
   //         consumer still stores its own value (reading R-RMT5) and counts it.
+  //   defer (warp-uniform; inter only): do not publish/free yet.  A deferred
+  //         commit MUST be followed by a non-deferred commit (or finish())
+  //         before any CTA-wide barrier, and a run of deferred commits plus its
+  //         closing commit must not exceed INTER_S records (deadlock freedom,
+  //         DESIGN.md "Inter-Group queue").
   template <int NW, int SID = 0, bool LIVE = false, class Store>
   __device__ __forceinline__ void commit(unsigned mask, unsigned idx, unsigned (&v)[NW], unsigned limit,
-                                         Store&& store) {
+                                         Store&& store, bool defer = false) {
     static_assert(NW >= 1 && NW <= MAXW, "commit width");
     if constexpr (FAULT) {
       if (c.f.sid == SID && c.f.replica == r && c.f.elem >= (long long)idx &&
@@ -308,6 +339,7 @@ struct Rep {
         if constexpr (INTER) ++j;
         return;
       }
+      (void)defer;
       // Record key: address + predicate in one word.
       unsigned key;
       if constexpr (NW == 1) key = mask ? idx : 0xffffffffu;
@@ -333,22 +365,23 @@ struct Rep {
         }
         __syncwarp();
       } else {  // V_INTER: per-(region, warp) queue of S records
-        const unsigned slot = j % (unsigned)c.S;
-        const size_t fi = ((size_t)region * c.W + warp) * c.S + slot;
+        const size_t fi = slot_index(j);
         unsigned* fl = c.flags + fi;
         unsigned* pl = c.payload + fi * (RING_WORDS * 32);
         if (!consumer) {
-          // wait for a free buffer; the first S slots of a fresh region are free
-          if (j >= (unsigned)c.S) spin_until(fl, 0u, c, lane == 0);
+          // wait for a free buffer; the first S slots of a fresh region are
+          // free.  Publish our own pending records first, or our consumer could be
+          // waiting for them while we wait for it.
+          if (j >= (unsigned)c.S) {
+            flush();
+            spin_until(fl, 0u, c, lane == 0);
+          }
           pl[lane] = key;
 #pragma unroll
           for (int k = 0; k < NW; ++k) pl[(1 + k) * 32 + lane] = v[k];
-          // Every lane fences its own payload stores (a release by lane 0 alone
-          // does not order the other lanes' in-flight stores), then lane 0
-          // signals "ready" ("signals the work-item in the consumer").
-          __threadfence();
-          __syncwarp();
-          if (lane == 0) st_relaxed(fl, 1u);
+          // The "ready" signal ("signals the work-item in the consumer") is
+          // published by flush(): every lane fences its own payload stores (a
+          // release by one lane does not order the other lanes' in-flight stores).
         } else {
           const bool ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
           pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
@@ -377,11 +410,9 @@ struct Rep {
       const unsigned mb = __ballot_sync(FULL, mism);
       if (mb != 0u && lane == __ffs(mb) - 1) atomicAdd(c.err, (unsigned long long)__popc(mb));
       if constexpr (INTER) {
-        if (consumer && lane == 0 && have) {
-          const size_t fi = ((size_t)region * c.W + warp) * c.S + (j % (unsigned)c.S);
-          st_release(c.flags + fi, 0u);  // free the buffer
-        }
         ++j;
+        ++pend;
+        if (!defer) flush();  // publish (producer) / free the buffers (consumer)
       }
     }
   }
