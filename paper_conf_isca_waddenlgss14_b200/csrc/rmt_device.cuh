@@ -306,6 +306,7 @@ struct Rep {
   __device__ __forceinline__ void commit(unsigned mask, unsigned idx, unsigned (&v)[NW], unsigned limit,
                                          Store&& store, bool defer = false) {
     static_assert(NW >= 1 && NW <= MAXW, "commit width");
+    bool addr_faulted = false;
     if constexpr (FAULT) {
       if (c.f.sid == SID && c.f.replica == r && c.f.elem >= (long long)idx &&
           c.f.elem < (long long)idx + NW) {
@@ -316,13 +317,15 @@ struct Rep {
             if (k == w) v[k] ^= 1u << c.f.bit;
         } else if (c.f.site == SITE_STORE_ADDR) {
           idx ^= (NW == 1 ? 1u : (unsigned)NW) << c.f.bit;  // bit of the (vector) index
+          addr_faulted = true;
         }
       }
     }
     if constexpr (V == V_NONE) {
       if (mask != 0u) {
         if constexpr (FAULT) {
-          if (idx + NW > limit) return;  // a faulted address outside the buffer: dropped
+          // a faulted address whose stored words fall outside the buffer: dropped
+          if (addr_faulted && idx + (31u - (unsigned)__clz(mask)) >= limit) return;
         }
         store(idx, mask, v);
       }
@@ -401,8 +404,8 @@ struct Rep {
           if (mask != 0u) store(idx, mask, v);
         } else {
           mism = true;
-          if constexpr (LIVE) {
-            if (mask != 0u && idx + NW <= limit) store(idx, mask, v);
+          if constexpr (LIVE) {  // highest stored word must be inside the buffer
+            if (mask != 0u && idx + (31u - (unsigned)__clz(mask)) < limit) store(idx, mask, v);
           }
         }
       }

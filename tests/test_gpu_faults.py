@@ -1,0 +1,93 @@
+"""Fault-injection campaign (-m gpu): single-bit flips at every instrumented
+site of every kernel, in either replica, under every RMT variant.
+
+For each (kernel, site, element, bit) the same flip is first injected into the
+unprotected kernel: the fault is *live* iff it changes the output (faults
+masked by the computation are not silent data corruption).  Every live fault
+inside the sphere of replication must then be detected (err >= 1) by every RMT
+variant, in either replica; STORE_* flips corrupt exactly one commit, so they
+must give err == 1 exactly.  Sites outside the SoR by design are not expected
+to be caught.
+"""
+import numpy as np
+import pytest
+
+from paper_conf_isca_waddenlgss14_b200 import rmt
+from cases import (DCT, FWT, BinarySearch, BlackScholes, FloydWarshall, MatMul, PrefixSum, Reduction, Sobel,
+                   Transpose)
+from helpers import run
+
+pytestmark = pytest.mark.gpu
+
+# kernel case, sites with their element-index space (callable(case) -> upper bound)
+CAMPAIGN = [
+    (lambda: BlackScholes(5000), {"load": lambda c: c.n, "compute": lambda c: c.n, "store_val": lambda c: c.n,
+                                  "store_addr": lambda c: c.n}),
+    (lambda: BinarySearch(1 << 16, 4000), {"load": lambda c: c.Q, "compute": lambda c: c.Q,
+                                           "store_val": lambda c: c.Q, "store_addr": lambda c: c.Q}),
+    (lambda: FWT(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n, "smem": lambda c: c.n,
+                            "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
+    (lambda: PrefixSum(4096 * 9 + 5), {"load": lambda c: c.n, "compute": lambda c: 256 * 10,
+                                       "smem": lambda c: 256 * 10, "store_val": lambda c: c.n,
+                                       "store_addr": lambda c: c.n}),
+    (lambda: Reduction(300007), {"load": lambda c: c.n, "compute": lambda c: 1184 * 256,
+                                 "smem": lambda c: 1184 * 8, "store_val": lambda c: 1, "store_addr": lambda c: 1}),
+    (lambda: Transpose(96, 160), {"load": lambda c: c.n, "smem": lambda c: c.n, "store_val": lambda c: c.n,
+                                  "store_addr": lambda c: c.n}),
+    (lambda: Sobel(40, 132), {"load": lambda c: c.n, "compute": lambda c: c.n, "store_val": lambda c: c.n,
+                              "store_addr": lambda c: c.n}),
+    (lambda: DCT(32, 264), {"load": lambda c: c.n, "compute": lambda c: c.n, "smem": lambda c: c.n,
+                            "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
+    (lambda: FloydWarshall(48), {"load": lambda c: c.n ** 3, "compute": lambda c: c.n ** 3,
+                                 "store_val": lambda c: c.n ** 3, "store_addr": lambda c: c.n ** 3}),
+    (lambda: MatMul(256, 128, 128), {"compute": lambda c: c.n, "store_val": lambda c: c.n,
+                                     "store_addr": lambda c: c.n}),
+]
+SAMPLES = 6
+
+
+def _outputs(case, variant):
+    b = case.buffers()
+    err = run(case.kernel, variant, b, case.n, case.dims)
+    return err, case.outputs(b)
+
+
+def _with_fault(case, variant, replica, site, bit, elem):
+    rmt.inject_fault(replica, site, bit, elem)
+    try:
+        return _outputs(case, variant)
+    finally:
+        rmt.clear_faults()
+
+
+@pytest.mark.parametrize("idx", range(len(CAMPAIGN)), ids=[f().kernel for f, _ in CAMPAIGN])
+def test_fault_campaign(idx):
+    make, sites = CAMPAIGN[idx]
+    case = make()
+    _, ref = _outputs(case, "none")
+    rng = np.random.default_rng(1000 + idx)
+    report = {}
+    for site, bound in sites.items():
+        live = detected = 0
+        for _ in range(SAMPLES * (40 if case.kernel == "floydwarshall" else 4)):
+            if live >= SAMPLES:
+                break
+            elem = int(rng.integers(0, bound(case)))
+            bit = int(rng.integers(0, 32))
+            if site == "store_addr":
+                bit = int(rng.integers(0, 6))  # keep the flipped address inside small buffers
+            _, o0 = _with_fault(case, "none", 0, site, bit, elem)
+            if all(np.array_equal(a, b) for a, b in zip(o0, ref)):
+                continue  # masked by the computation: not an SDC, nothing to detect
+            live += 1
+            for variant in rmt.RMT_VARIANTS:
+                for replica in (0, 1):
+                    err, _ = _with_fault(case, variant, replica, site, bit, elem)
+                    assert err >= 1, (f"{case.kernel}: live {site} fault (elem {elem}, bit {bit}) in replica "
+                                      f"{replica} NOT detected by {variant}")
+                    if site.startswith("store") and case.kernel not in ("floydwarshall",):
+                        assert err == 1, f"{case.kernel}/{variant}: {site} flip must corrupt exactly one commit"
+                    detected += 1
+        report[site] = (live, detected)
+        assert live > 0, f"{case.kernel}/{site}: no live fault found (vacuous)"
+    print(case.kernel, report)
