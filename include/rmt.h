@@ -97,7 +97,7 @@ typedef struct {
  *   FLOYDWARSHALL buf {D:U32[n*n] in/out, P:U32[n*n] out}           n = nodes, n%4 = 0
  *   DCT           buf {X:F32[H*W], Y:F32[H*W]}                      n = H*W, dims {H, W}, H%8 = W%8 = 0
  *   MATMUL        buf {A:BF16[M*K], Bt:BF16[N*K], C:F32[M*N]}       n = M*N, dims {M, N, K}
- *                 C = A * Bt^T (both operands K-major); M%128 = N%128 = 0, K%64 = 0
+ *                 C = A * Bt^T (both operands K-major); M%128 = N%256 = 0, K%64 = 0
  * Vector-committed buffers must have < 2^30 elements.
  */
 typedef struct {

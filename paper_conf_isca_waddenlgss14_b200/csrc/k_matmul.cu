@@ -3,13 +3,13 @@
 // ~2x for compute-bound kernels).  C = A * Bt^T, bf16 operands (K-major
 // both), fp32 accumulation and result (reading R-MM1).
 //
-// B200 design (tcgen05 + TMEM + TMA): one 128x128 output tile per logical CTA,
+// B200 design (tcgen05 + TMEM + TMA): one 128x256 output tile per logical CTA,
 // K in blocks of 64 (128-B rows, SWIZZLE_128B).  Thread 0 streams A/B tiles
 // into a ring of smem stages with TMA (cp.async.bulk.tensor, mbarrier
-// complete_tx); thread 32 issues tcgen05.mma (M=128, N=128, K=16) into a TMEM
+// complete_tx); thread 32 issues tcgen05.mma (M=128, N=256, K=16) into a TMEM
 // accumulator and frees each stage with tcgen05.commit.  Both replicas run on
 // the tensor pipe (BASELINE.json): the intra variants issue every MMA twice, into
-// two TMEM accumulators (acc0 cols [0,128), acc1 cols [128,256)); INTRA_SMEM
+// two TMEM accumulators (acc0 cols [0,256), acc1 cols [256,512)); INTRA_SMEM
 // also keeps a private copy of every operand tile per replica (+LDS),
 // INTRA_REG shares one operand copy (the load path is outside the SoR).
 // Inter-group: two CTAs per tile, each with its own accumulator.
@@ -26,10 +26,10 @@
 namespace rmt {
 namespace {
 
-constexpr int BM = 128, BN = 128, BK = 64, UK = 16;
+constexpr int BM = 128, BN = 256, BK = 64, UK = 16;
 constexpr int BL = 128;                      // logical threads per CTA (4 warps)
-constexpr int TILE_BYTES = BM * BK * 2;      // 16 KiB per operand tile
-constexpr int NSTAGE = 3;
+constexpr int TILE_A = BM * BK * 2;          // 16 KiB A tile per stage
+constexpr int TILE_B = BN * BK * 2;          // 32 KiB B tile per stage
 constexpr int SPITCH = 68;                   // staging row pitch (floats): conflict-free
 constexpr int SPLANE = BM * SPITCH + 16;     // replica plane offset (16 banks apart)
 constexpr int ECHUNK = 64;                   // epilogue columns per chunk
@@ -38,14 +38,16 @@ template <int V>
 struct MmCfg {
   static constexpr int COPIES = (V == V_INTRA_SMEM) ? 2 : 1;       // operand copies in smem
   static constexpr int ACCS = (V == V_INTRA_SMEM || V == V_INTRA_REG) ? 2 : 1;
-  static constexpr int STAGE_BYTES = 2 * TILE_BYTES * COPIES;
+  static constexpr int COPY_BYTES = TILE_A + TILE_B;
+  static constexpr int STAGE_BYTES = COPY_BYTES * COPIES;
+  static constexpr int NSTAGE = COPIES == 2 ? 2 : 4;               // 192 KiB of operand ring
   static constexpr int SMEM = NSTAGE * STAGE_BYTES + 1024;
-  static constexpr int TMEM_COLS = 128 * ACCS;
+  static constexpr int TMEM_COLS = BN * ACCS;                     // 256 or 512 columns
 };
 
 struct MmArgs {
   CUtensorMap tmA;  // A: M x K bf16, box 64 x 128
-  CUtensorMap tmB;  // Bt: N x K bf16, box 64 x 128
+  CUtensorMap tmB;  // Bt: N x K bf16, box 64 x 256
   float* C;
   unsigned M, N, K;
   unsigned ntn;     // tiles along N
@@ -118,6 +120,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 1) mm_kernel(const __grid_c
   using Cfg = MmCfg<V>;
   extern __shared__ __align__(1024) unsigned char dsm[];
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  constexpr int NSTAGE = Cfg::NSTAGE;
   __shared__ __align__(8) unsigned long long bar_full[NSTAGE], bar_empty[NSTAGE], bar_done;
   __shared__ uint32_t s_tmem;
   unsigned char* smem = (unsigned char*)(((uintptr_t)dsm + 1023) & ~(uintptr_t)1023);
@@ -157,8 +160,8 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 1) mm_kernel(const __grid_c
       const uint32_t st = smem_u32(smem + s * Cfg::STAGE_BYTES);
 #pragma unroll
       for (int cp = 0; cp < Cfg::COPIES; ++cp) {  // INTRA_SMEM: one private copy per replica
-        tma_load_2d(st + cp * 2 * TILE_BYTES, &a.tmA, (int)(kb * BK), (int)(tm * BM), fb);
-        tma_load_2d(st + cp * 2 * TILE_BYTES + TILE_BYTES, &a.tmB, (int)(kb * BK), (int)(tn * BN), fb);
+        tma_load_2d(st + cp * Cfg::COPY_BYTES, &a.tmA, (int)(kb * BK), (int)(tm * BM), fb);
+        tma_load_2d(st + cp * Cfg::COPY_BYTES + TILE_A, &a.tmB, (int)(kb * BK), (int)(tn * BN), fb);
       }
     }
   } else if (threadIdx.x == 32) {
@@ -173,8 +176,8 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 1) mm_kernel(const __grid_c
         const uint32_t acc = (kb | (unsigned)k) != 0u;
 #pragma unroll
         for (int rr = 0; rr < Cfg::ACCS; ++rr) {  // replica rr: its own accumulator (and operand copy)
-          const uint32_t base = st + (Cfg::COPIES == 2 ? rr : 0) * 2 * TILE_BYTES + k * UK * 2;
-          tc_mma(tmem + rr * 128, sdesc(base), sdesc(base + TILE_BYTES), IDESC, acc);
+          const uint32_t base = st + (Cfg::COPIES == 2 ? rr : 0) * Cfg::COPY_BYTES + k * UK * 2;
+          tc_mma(tmem + rr * BN, sdesc(base), sdesc(base + TILE_A), IDESC, acc);
         }
       }
       tc_commit(smem_u32(&bar_empty[s]));  // frees the stage when these MMAs complete
@@ -196,7 +199,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 1) mm_kernel(const __grid_c
 #pragma unroll
     for (int cc = 0; cc < ECHUNK / 16; ++cc) {
       uint32_t v[16];
-      tc_ld16(tmem + ((uint32_t)(32 * q) << 16) + rrep * 128 + ch * ECHUNK + cc * 16, v);
+      tc_ld16(tmem + ((uint32_t)(32 * q) << 16) + rrep * BN + ch * ECHUNK + cc * 16, v);
       if constexpr (M == M_FAULT) {
 #pragma unroll
         for (int t = 0; t < 16; ++t) {
@@ -255,7 +258,7 @@ EncodeTiledFn get_encode() {
   return fn;
 }
 
-int make_tmap(CUtensorMap* tm, const void* base, unsigned rows, unsigned K) {
+int make_tmap(CUtensorMap* tm, const void* base, unsigned rows, unsigned K, unsigned box_rows) {
   EncodeTiledFn enc = get_encode();
   if (!enc) {
     set_error("matmul: cuTensorMapEncodeTiled unavailable");
@@ -263,7 +266,7 @@ int make_tmap(CUtensorMap* tm, const void* base, unsigned rows, unsigned K) {
   }
   cuuint64_t dims[2] = {K, rows};
   cuuint64_t strides[1] = {(cuuint64_t)K * 2};
-  cuuint32_t box[2] = {BK, 128};
+  cuuint32_t box[2] = {BK, box_rows};
   cuuint32_t es[2] = {1, 1};
   CUresult r = enc(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -279,10 +282,10 @@ int make_tmap(CUtensorMap* tm, const void* base, unsigned rows, unsigned K) {
 
 int matmul_validate(const rmt_bufs_t* b, int64_t n) {
   int64_t M = b->dims[0], N = b->dims[1], K = b->dims[2];
-  if (b->nbuf < 3 || M <= 0 || N <= 0 || K <= 0 || M % 128 || N % 128 || K % 64 || n != M * N ||
+  if (b->nbuf < 3 || M <= 0 || N <= 0 || K <= 0 || M % BM || N % BN || K % BK || n != M * N ||
       M * N >= (1LL << 30) || K >= (1LL << 24) || !buf_ok(b->buf[0], RMT_BF16, M * K) ||
       !buf_ok(b->buf[1], RMT_BF16, N * K) || !buf_ok(b->buf[2], RMT_F32, M * N)) {
-    set_error("matmul: expected {A:BF16[M*K], Bt:BF16[N*K], C:F32[M*N]}, dims {M,N,K}, M%128 = N%128 = 0, K%64 = 0");
+    set_error("matmul: expected {A:BF16[M*K], Bt:BF16[N*K], C:F32[M*N]}, dims {M,N,K}, M%128 = N%256 = 0, K%64 = 0");
     return RMT_EINVAL;
   }
   return RMT_OK;
@@ -294,9 +297,9 @@ int matmul_run(Launch& L) {
   const unsigned M = (unsigned)L.bufs->dims[0], N = (unsigned)L.bufs->dims[1], K = (unsigned)L.bufs->dims[2];
   MmArgs a;
   memset(&a, 0, sizeof(a));
-  int rc = make_tmap(&a.tmA, L.bufs->buf[0].ptr, M, K);
+  int rc = make_tmap(&a.tmA, L.bufs->buf[0].ptr, M, K, BM);
   if (rc) return rc;
-  rc = make_tmap(&a.tmB, L.bufs->buf[1].ptr, N, K);
+  rc = make_tmap(&a.tmB, L.bufs->buf[1].ptr, N, K, BN);
   if (rc) return rc;
   a.C = (float*)L.bufs->buf[2].ptr;
   a.M = M;

@@ -413,5 +413,5 @@ def small_cases():
         Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
         DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8),
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
-        MatMul(128, 128, 64), MatMul(256, 384, 192, integer=True), MatMul(512, 256, 1024),
+        MatMul(128, 256, 64), MatMul(256, 512, 192, integer=True), MatMul(384, 256, 1024),
     ]

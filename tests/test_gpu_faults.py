@@ -40,7 +40,7 @@ CAMPAIGN = [
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
     (lambda: FloydWarshall(48), {"load": lambda c: c.n ** 3, "compute": lambda c: c.n ** 3,
                                  "store_val": lambda c: c.n ** 3, "store_addr": lambda c: c.n ** 3}),
-    (lambda: MatMul(256, 128, 128), {"compute": lambda c: c.n, "store_val": lambda c: c.n,
+    (lambda: MatMul(256, 256, 128), {"compute": lambda c: c.n, "store_val": lambda c: c.n,
                                      "store_addr": lambda c: c.n}),
 ]
 SAMPLES = 6
