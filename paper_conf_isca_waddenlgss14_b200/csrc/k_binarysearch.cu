@@ -83,7 +83,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
   for (int q = 0; q < 4; ++q) {
     const unsigned j = j0 + q;
     const unsigned long long src = (unsigned long long)j * stride;
-    w[q] = (active && j < a.L.n[k]) ? __ldg(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[16^k j]
+    w[q] = (active && j < a.L.n[k]) ? __ldcs(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[16^k j] (A: evict-first)
   }
   rep.template commit<4, 1>(active ? 0xFu : 0u, active ? a.L.off[k] + j0 : 0u, w, 0xFFFFFFF0u,
                             [&](unsigned i, unsigned m, const unsigned* x) {
@@ -143,13 +143,15 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 3 : 4) 
       for (int i = 0; i < 4; ++i) {
         const unsigned base = rep.lshfl_idx(mybase, g0 + i) + 4u * gm;
         uint4 w;
-        if (!tail || base + 4u <= lim) {
+        if (!tail) {  // sample levels: keep them L2-resident (default policy)
           w = __ldg(reinterpret_cast<const uint4*>(P + base));
+        } else if (base + 4u <= lim) {  // the caller's A: random 64-B blocks, evict-first
+          w = __ldcs(reinterpret_cast<const uint4*>(P + base));
         } else {  // tail of the caller's A: element-wise, never past lim
-          w.x = base + 0 < lim ? __ldg(P + base + 0) : 0xFFFFFFFFu;
-          w.y = base + 1 < lim ? __ldg(P + base + 1) : 0xFFFFFFFFu;
-          w.z = base + 2 < lim ? __ldg(P + base + 2) : 0xFFFFFFFFu;
-          w.w = base + 3 < lim ? __ldg(P + base + 3) : 0xFFFFFFFFu;
+          w.x = base + 0 < lim ? __ldcs(P + base + 0) : 0xFFFFFFFFu;
+          w.y = base + 1 < lim ? __ldcs(P + base + 1) : 0xFFFFFFFFu;
+          w.z = base + 2 < lim ? __ldcs(P + base + 2) : 0xFFFFFFFFu;
+          w.w = base + 3 < lim ? __ldcs(P + base + 3) : 0xFFFFFFFFu;
         }
         const unsigned k = K[i][s];
         const unsigned bits = (w.x < k ? 1u : 0u) | (w.y < k ? 2u : 0u) | (w.z < k ? 4u : 0u) | (w.w < k ? 8u : 0u);

@@ -54,7 +54,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_init_kernel(FwArgs a, Ct
 // One pass k.  Each logical thread handles VPT 16-B vectors strided by the CTA
 // width (coalesced); fat CTAs amortise the per-CTA RMT handshakes (inter-group
 // ticket / turn / queue latency) over 8192 elements.
-constexpr int VPT = 8;
+constexpr int VPT = 1;
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
