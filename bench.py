@@ -4,7 +4,7 @@
 
 One step = one pass of the whole hot path over one batch of synthetic input:
 every kernel of the config launched once under each variant
-(none, intra_smem, intra_reg, inter_group) through the C ABI (librmt.so).
+(none, intra_smem, intra_reg, inter_group, inter_cluster) through the C ABI (librmt.so).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config suite] [--impl rmt|reference]
 
@@ -31,7 +31,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "RMT slowdown vs unprotected kernel per variant; baseline HBM GB/s vs peak"
-VARIANTS = ("none", "intra_smem", "intra_reg", "inter_group")
+VARIANTS = ("none", "intra_smem", "intra_reg", "inter_group", "inter_cluster")
 
 
 def parse():

@@ -36,6 +36,12 @@
  *                   through a bounded global-memory queue with release/acquire
  *                   flags ("two-tiered locking system"; L2-coherent
  *                   reads); the consumer compares and stores.
+ *   RMT_INTER_CLUSTER Inter-Group RMT, Blackwell-native:
+ *                   the pair is a 2-CTA thread-block cluster (hardware
+ *                   co-scheduling replaces the ticket); the producer CTA writes
+ *                   its store records into the consumer CTA's shared memory
+ *                   through distributed shared memory (DSMEM) with cluster-scope
+ *                   release/acquire flags, instead of an L2/HBM queue.
  *
  * Thread-safety: launches on different streams must use different workspaces.
  * The fault-injection and ablation state is process-global (test/bench use).
@@ -54,7 +60,8 @@ typedef enum {
     RMT_NONE = 0,
     RMT_INTRA_SMEM = 1,
     RMT_INTRA_REG = 2,
-    RMT_INTER_GROUP = 3
+    RMT_INTER_GROUP = 3,
+    RMT_INTER_CLUSTER = 4
 } rmt_variant_t;
 
 /* The AMD APP SDK-style kernels the paper evaluates (Fig. 2 axis

@@ -33,7 +33,7 @@
 
 namespace rmt {
 
-constexpr int V_NONE = 0, V_INTRA_SMEM = 1, V_INTRA_REG = 2, V_INTER = 3;
+constexpr int V_NONE = 0, V_INTRA_SMEM = 1, V_INTRA_REG = 2, V_INTER = 3, V_CLUSTER = 4;
 constexpr int M_NORMAL = 0, M_FAULT = 1, M_NOCOMM = 2;
 constexpr int SITE_LOAD = 0, SITE_COMPUTE = 1, SITE_SMEM = 2, SITE_STORE_VAL = 3, SITE_STORE_ADDR = 4;
 constexpr int MAXW = 4;               // max value words per commit
@@ -42,6 +42,8 @@ constexpr int MBOX_WORDS = RING_WORDS * 16;  // intra_smem mailbox words per war
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int CTRL_TURN = 64;         // ctrl[64 ..) = per-region turn counters
 constexpr unsigned long long WATCHDOG_CYCLES = 1ull << 32;  // ~2 s at 2 GHz
+constexpr int CL_S = 4;     // inter_cluster: mailbox slots per warp (in the consumer CTA's smem)
+constexpr int CL_MAXW = 8;  // inter_cluster: max warps per CTA
 
 struct FaultDesc {
   int replica, site, bit, sid;
@@ -92,6 +94,45 @@ __device__ __forceinline__ void stg4(void* p, uint4 v) { *reinterpret_cast<uint4
 __device__ __forceinline__ uint4 ldcs4(const void* p) { return __ldcs(reinterpret_cast<const uint4*>(p)); }
 __device__ __forceinline__ void stcs4(void* p, uint4 v) { __stcs(reinterpret_cast<uint4*>(p), v); }
 
+// ---- thread-block-cluster / distributed shared memory (inter_cluster)
+__device__ __forceinline__ unsigned cluster_ctarank() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ unsigned cluster_id_x() {
+  unsigned r;
+  asm volatile("mov.u32 %0, %%clusterid.x;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ unsigned mapa_rank(unsigned saddr, unsigned rank) {
+  unsigned r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void st_cl(unsigned addr, unsigned v) {
+  asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_cl(unsigned addr) {
+  unsigned v;
+  asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned ld_acquire_cl(unsigned addr) {
+  unsigned v;
+  asm volatile("ld.acquire.cluster.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_cl(unsigned addr, unsigned v) {
+  asm volatile("st.release.cluster.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_cl(unsigned addr, unsigned v) {
+  asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 // Spin until *p == want (acquire), with back-off and a watchdog that converts a
 // hang (a fault that desynchronised a pair) into err+1 and a sticky flag.
 // Every thread that will touch the guarded data must do its own acquire: a lane
@@ -114,11 +155,26 @@ __device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, con
   }
 }
 
+// Cluster-scope spin on a shared::cluster address (local or a peer CTA's).
+__device__ __forceinline__ bool spin_cl(unsigned addr, unsigned want, const Ctx& c, bool count) {
+  if (ld_acquire_cl(addr) == want) return true;
+  unsigned long long t0 = clock64();
+  while (true) {
+    __nanosleep(20);
+    if (ld_acquire_cl(addr) == want) return true;
+    if (clock64() - t0 > WATCHDOG_CYCLES) {
+      if (count) atomicAdd(c.err, 1ull);
+      return false;
+    }
+  }
+}
+
 // ---------------------------------------------------------------- replica state
 template <int V, int MODE>
 struct Rep {
   static constexpr bool INTRA = (V == V_INTRA_SMEM || V == V_INTRA_REG);
   static constexpr bool INTER = (V == V_INTER);
+  static constexpr bool CLUSTER = (V == V_CLUSTER);
   static constexpr int DUP = INTRA ? 2 : 1;  // physical threads per logical thread
   static constexpr int LW = 32 / DUP;        // logical warp width
   static constexpr bool FAULT = (MODE == M_FAULT);
@@ -134,8 +190,9 @@ struct Rep {
   unsigned pend;  // inter: records not yet published (producer) / freed (consumer)
   unsigned region, epoch;
   unsigned* mbox;  // intra_smem: this warp's mailbox
+  unsigned cl_pay, cl_full;  // inter_cluster: this warp's mailbox / flags in the consumer CTA (shared::cluster)
 
-  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), pend(0), region(0), epoch(0), mbox(nullptr) {}
+  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), pend(0), region(0), epoch(0), mbox(nullptr), cl_pay(0), cl_full(0) {}
 
   // Must be called by every thread of the CTA, first thing (may __syncthreads).
   // mbox_smem: MBOX_WORDS * (blockDim/32) words of shared memory (intra_smem only).
@@ -167,6 +224,27 @@ struct Rep {
         if (threadIdx.x == 0 && epoch != 0) spin_until(c.ctrl + CTRL_TURN + region, epoch, c);
         __syncthreads();
       }
+    } else if constexpr (CLUSTER) {
+      // The pair is a 2-CTA thread-block cluster: hardware co-schedules both
+      // CTAs, so no ticket or turn is needed (the B200 form of P:679's
+      // "co-scheduling" remark); rank 0 = producer, rank 1 = consumer.  Records go
+      // into a mailbox in the CONSUMER's shared memory through distributed
+      // shared memory (DSMEM), not through L2.
+      __shared__ __align__(16) unsigned cl_payload[CL_MAXW * CL_S * RING_WORDS * 32];
+      __shared__ unsigned cl_flags[CL_MAXW * CL_S];
+      r = (int)cluster_ctarank();
+      consumer = (r == 1);
+      lblock = (int)cluster_id_x();
+      ltid = threadIdx.x;
+      llane = lane;
+      if constexpr (!NOCOMM) {
+        for (int i = threadIdx.x; i < CL_MAXW * CL_S; i += blockDim.x) cl_flags[i] = 0u;
+        unsigned pb = (unsigned)__cvta_generic_to_shared(cl_payload) + (unsigned)(warp * CL_S * RING_WORDS * 32) * 4u;
+        unsigned fb = (unsigned)__cvta_generic_to_shared(cl_flags) + (unsigned)(warp * CL_S) * 4u;
+        cl_pay = consumer ? pb : mapa_rank(pb, 1u);
+        cl_full = consumer ? fb : mapa_rank(fb, 1u);
+        cluster_sync_all();  // both mailboxes initialised before any record
+      }
     } else {
       r = 0;
       consumer = true;
@@ -186,6 +264,19 @@ struct Rep {
     return ((size_t)region * c.W + warp) * c.S + (rec % (unsigned)c.S);
   }
   __device__ __forceinline__ void flush() {
+    if constexpr (CLUSTER && !NOCOMM) {
+      if (pend == 0u) return;
+      const unsigned first = j - pend;
+      if (!consumer) {
+        asm volatile("fence.acq_rel.cluster;" ::: "memory");
+        __syncwarp();
+        if ((unsigned)lane < pend) st_relaxed_cl(cl_full + ((first + lane) % CL_S) * 4u, 1u);
+      } else {
+        __syncwarp();
+        if ((unsigned)lane < pend) st_release_cl(cl_full + ((first + lane) % CL_S) * 4u, 0u);
+      }
+      pend = 0u;
+    }
     if constexpr (INTER && !NOCOMM) {
       if (pend == 0u) return;
       const unsigned first = j - pend;
@@ -202,6 +293,10 @@ struct Rep {
   }
 
   __device__ __forceinline__ void finish() {
+    if constexpr (CLUSTER && !NOCOMM) {
+      flush();
+      cluster_sync_all();  // no DSMEM access of either CTA is in flight when they exit
+    }
     if constexpr (INTER) {
       __shared__ unsigned s_last;
       flush();
@@ -339,7 +434,7 @@ struct Rep {
 #pragma unroll
           for (int k = 0; k < NW; ++k) keep_alive(v[k]);
         }
-        if constexpr (INTER) ++j;
+        if constexpr (INTER || CLUSTER) ++j;
         return;
       }
       (void)defer;
@@ -367,6 +462,24 @@ struct Rep {
           for (int k = 0; k < NW; ++k) pv[k] = mbox[(1 + k) * 16 + slot];
         }
         __syncwarp();
+      } else if constexpr (V == V_CLUSTER) {  // DSMEM mailbox in the consumer CTA
+        const unsigned slot = j % CL_S;
+        const unsigned pa = cl_pay + (slot * RING_WORDS * 32 + lane) * 4u;
+        const unsigned fa = cl_full + slot * 4u;
+        if (!consumer) {
+          if (j >= (unsigned)CL_S) {  // publish ours first, then wait for a free slot
+            flush();
+            spin_cl(fa, 0u, c, lane == 0);
+          }
+          st_cl(pa, key);
+#pragma unroll
+          for (int k = 0; k < NW; ++k) st_cl(pa + (1 + k) * 32 * 4, v[k]);
+        } else {
+          have = spin_cl(fa, 1u, c, lane == 0);  // every lane acquires
+          pk = ld_cl(pa);
+#pragma unroll
+          for (int k = 0; k < NW; ++k) pv[k] = ld_cl(pa + (1 + k) * 32 * 4);
+        }
       } else {  // V_INTER: per-(region, warp) queue of S records
         const size_t fi = slot_index(j);
         unsigned* fl = c.flags + fi;
@@ -412,7 +525,7 @@ struct Rep {
       // warp ballot over the compare results: completes every lane's loads
       const unsigned mb = __ballot_sync(FULL, mism);
       if (mb != 0u && lane == __ffs(mb) - 1) atomicAdd(c.err, (unsigned long long)__popc(mb));
-      if constexpr (INTER) {
+      if constexpr (INTER || CLUSTER) {
         ++j;
         ++pend;
         if (!defer) flush();  // publish (producer) / free the buffers (consumer)
@@ -425,7 +538,9 @@ struct Rep {
 template <int V>
 struct Geom {
   static constexpr int DUP = (V == V_INTRA_SMEM || V == V_INTRA_REG) ? 2 : 1;
-  static __host__ __device__ unsigned grid(unsigned lblocks) { return V == V_INTER ? 2u * lblocks : lblocks; }
+  static __host__ __device__ unsigned grid(unsigned lblocks) {
+    return (V == V_INTER || V == V_CLUSTER) ? 2u * lblocks : lblocks;
+  }
   static __host__ __device__ unsigned block(unsigned lthreads) { return lthreads * DUP; }
 };
 

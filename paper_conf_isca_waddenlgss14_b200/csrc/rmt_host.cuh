@@ -63,6 +63,10 @@ int dispatch(int v, int m, F&& f) {
       return m == M_FAULT ? f(VM<V_INTER, M_FAULT>{})
            : m == M_NOCOMM ? f(VM<V_INTER, M_NOCOMM>{})
                            : f(VM<V_INTER, M_NORMAL>{});
+    case V_CLUSTER:
+      return m == M_FAULT ? f(VM<V_CLUSTER, M_FAULT>{})
+           : m == M_NOCOMM ? f(VM<V_CLUSTER, M_NOCOMM>{})
+                           : f(VM<V_CLUSTER, M_NORMAL>{});
   }
   return RMT_EINVAL;
 }
@@ -130,11 +134,27 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
     int occ = 0;
     if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kr, Geom<V>::block(BL), smem);
-    int target = V == V_INTER ? (occ / 2 > 1 ? occ / 2 : 1) : (occ > 1 ? occ : 1);
+    int target = (V == V_INTER || V == V_CLUSTER) ? (occ / 2 > 1 ? occ / 2 : 1) : (occ > 1 ? occ : 1);
     size_t pad = pad_for_occupancy(kn, BL, smem, target);
     if (smem + pad > 48 * 1024)
       cudaFuncSetAttribute(kn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem + pad));
     kn<<<G, BL, smem + pad, L.stream>>>(a, c);
+  } else if constexpr (V == V_CLUSTER) {
+    if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(Geom<V>::grid(G));
+    cfg.blockDim = dim3(Geom<V>::block(BL));
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = L.stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;  // the replica pair
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kr, a, c);
+    if (e != cudaSuccess) return cuda_check(e, what);
   } else {
     if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     kr<<<Geom<V>::grid(G), Geom<V>::block(BL), smem, L.stream>>>(a, c);

@@ -5,7 +5,7 @@ import torch
 from paper_conf_isca_waddenlgss14_b200 import rmt
 
 SENTINEL = 0xFFFFFFFF
-VARIANTS = ("none", "intra_smem", "intra_reg", "inter_group")
+VARIANTS = ("none",) + rmt.RMT_VARIANTS
 
 
 def dev(a: np.ndarray) -> torch.Tensor:

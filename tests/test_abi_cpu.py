@@ -44,6 +44,7 @@ def test_workspace_sizes(L):
     from paper_conf_isca_waddenlgss14_b200 import rmt
     assert rmt.workspace_size("blackscholes", "none", 1 << 16) == 0
     assert rmt.workspace_size("blackscholes", "intra_reg", 1 << 16) == 0
+    assert rmt.workspace_size("blackscholes", "inter_cluster", 1 << 16) == 0  # mailbox lives in DSMEM
     inter = rmt.workspace_size("blackscholes", "inter_group", 1 << 16)
     assert inter > 0 and inter % 256 == 0
     assert rmt.workspace_size("reduction", "none", 1 << 20) >= 148 * 8 * 8

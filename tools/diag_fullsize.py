@@ -12,7 +12,7 @@ for j in workloads.config_jobs(cfg):
     bufs = j.device_buffers()
     outs = [i for i, h in enumerate(j.host_in) if h is None]
     ref = None
-    for v in ("none", "intra_smem", "intra_reg", "inter_group"):
+    for v in ("none", "intra_smem", "intra_reg", "inter_group", "inter_cluster"):
         ws = rmt.make_workspace(j.kernel, v, j.n, j.dims)
         for r in range(reps):
             err = torch.zeros(1, dtype=torch.int64, device="cuda")

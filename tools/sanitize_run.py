@@ -14,7 +14,7 @@ for c in cases:
     if only and c.kernel not in only:
         continue
     ref = None
-    for v in ("none", "intra_smem", "intra_reg", "inter_group"):
+    for v in ("none", "intra_smem", "intra_reg", "inter_group", "inter_cluster"):
         b = c.buffers()
         e = run(c.kernel, v, b, c.n, c.dims)
         o = c.outputs(b)

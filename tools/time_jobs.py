@@ -7,7 +7,7 @@ from paper_conf_isca_waddenlgss14_b200 import rmt, workloads
 
 cfg = sys.argv[1]
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
-variants = sys.argv[3].split(",") if len(sys.argv) > 3 else ["none", "intra_smem", "intra_reg", "inter_group"]
+variants = sys.argv[3].split(",") if len(sys.argv) > 3 else ["none", "intra_smem", "intra_reg", "inter_group", "inter_cluster"]
 for j in workloads.config_jobs(cfg):
     b = j.device_buffers()
     base = None
