@@ -42,6 +42,13 @@
  *                   its store records into the consumer CTA's shared memory
  *                   through distributed shared memory (DSMEM) with cluster-scope
  *                   release/acquire flags, instead of an L2/HBM queue.
+ *   RMT_INTRA_NOLDS Intra-Group RMT -LDS:
+ *                   pairs as in INTRA_REG, but the kernel's shared memory is NOT
+ *                   duplicated: both replicas read one copy, and every kernel
+ *                   shared-memory store is exchanged (registers), compared and
+ *                   performed once by the consumer.  Shared memory is outside
+ *                   this variant's sphere of replication (a fault in the copy
+ *                   is read by both replicas and is not detected).
  *
  * Thread-safety: launches on different streams must use different workspaces.
  * The fault-injection and ablation state is process-global (test/bench use).
@@ -61,7 +68,8 @@ typedef enum {
     RMT_INTRA_SMEM = 1,
     RMT_INTRA_REG = 2,
     RMT_INTER_GROUP = 3,
-    RMT_INTER_CLUSTER = 4
+    RMT_INTER_CLUSTER = 4,
+    RMT_INTRA_NOLDS = 5
 } rmt_variant_t;
 
 /* The AMD APP SDK-style kernels the paper evaluates (Fig. 2 axis

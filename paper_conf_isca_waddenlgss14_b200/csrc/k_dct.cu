@@ -35,7 +35,7 @@ template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ __align__(16) float Zs[DUP == 2 ? PLANE + ZWORDS : ZWORDS];
+  __shared__ __align__(16) float Zs[Geom<V>::SMDUP == 2 ? PLANE + ZWORDS : ZWORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
@@ -67,8 +67,12 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c
     z[v] = s;
   }
   float* zrow = &rep.template smp<PLANE>(Zs, b * BSTRIDE + r * 8);
-  reinterpret_cast<float4*>(zrow)[0] = make_float4(z[0], z[1], z[2], z[3]);
-  reinterpret_cast<float4*>(zrow)[1] = make_float4(z[4], z[5], z[6], z[7]);
+  const unsigned zw[8] = {__float_as_uint(z[0]), __float_as_uint(z[1]), __float_as_uint(z[2]), __float_as_uint(z[3]),
+                          __float_as_uint(z[4]), __float_as_uint(z[5]), __float_as_uint(z[6]), __float_as_uint(z[7])};
+  if (rep.template sts_ok<8>(zw, b * BSTRIDE + r * 8)) {
+    reinterpret_cast<float4*>(zrow)[0] = make_float4(z[0], z[1], z[2], z[3]);
+    reinterpret_cast<float4*>(zrow)[1] = make_float4(z[4], z[5], z[6], z[7]);
+  }
   __syncthreads();
   // column pass: thread (b, u) produces output row u of block b
   const int u = r;

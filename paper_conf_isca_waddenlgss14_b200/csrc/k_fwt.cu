@@ -71,13 +71,18 @@ __device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int 
         v[k + h] = __fsub_rn(x0, x1);
       }
     }
+    unsigned vw[G];
 #pragma unroll
     for (int k = 0; k < G; ++k) {
       if constexpr (R::FAULT) {
         if (a.s0 == 0 && round_no == 0)
           v[k] = rep.faultf(SITE_COMPUTE, (long long)gindex(a, tileid, ebase | (k << q)), v[k]);
       }
-      rep.template smp<PLANE>(tile, phys(ebase | (k << q))) = v[k];
+      vw[k] = __float_as_uint(v[k]);
+    }
+    if (rep.template sts_ok<G>(vw, (unsigned)ebase)) {
+#pragma unroll
+      for (int k = 0; k < G; ++k) rep.template smp<PLANE>(tile, phys(ebase | (k << q))) = v[k];
     }
   }
 }
@@ -119,13 +124,18 @@ __device__ __forceinline__ void fwt_round_ct(const R& rep, float* tile, const Fw
         v[k + h] = __fsub_rn(x0, x1);
       }
     }
+    unsigned vw[G];
 #pragma unroll
     for (int k = 0; k < G; ++k) {
       if constexpr (R::FAULT) {
         if (a.s0 == 0 && round_no == 0)
           v[k] = rep.faultf(SITE_COMPUTE, (long long)gindex(a, tileid, ebase | (k << Q)), v[k]);
       }
-      pb[coff<NB, Q>(k)] = v[k];
+      vw[k] = __float_as_uint(v[k]);
+    }
+    if (rep.template sts_ok<G>(vw, (unsigned)ebase)) {
+#pragma unroll
+      for (int k = 0; k < G; ++k) pb[coff<NB, Q>(k)] = v[k];
     }
   }
 }
@@ -137,7 +147,7 @@ template <int V, int M, int KIND>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ float tile[DUP == 2 ? PLANE + SM_WORDS : SM_WORDS];
+  __shared__ float tile[Geom<V>::SMDUP == 2 ? PLANE + SM_WORDS : SM_WORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned tileid = (unsigned)rep.lblock;
@@ -153,15 +163,20 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
 #pragma unroll
       for (int k = 0; k < 4; ++k) w[k] = e0 + k < te ? a.src[g + k] : 0.0f;
     }
+    unsigned xw[4];
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      if (e0 + k < te) {
-        float x = w[k];
-        if constexpr (M == M_FAULT) {
-          if (a.s0 == 0) x = rep.faultf(SITE_LOAD, (long long)g + k, x);
-        }
-        rep.template smp<PLANE>(tile, phys(e0 + k)) = x;
+      float x = w[k];
+      if constexpr (M == M_FAULT) {
+        if (a.s0 == 0 && e0 + k < te) x = rep.faultf(SITE_LOAD, (long long)g + k, x);
       }
+      w[k] = x;
+      xw[k] = __float_as_uint(x);
+    }
+    if (rep.template sts_ok<4>(xw, (unsigned)e0)) {
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        if (e0 + k < te) rep.template smp<PLANE>(tile, phys(e0 + k)) = w[k];
     }
   }
   __syncthreads();

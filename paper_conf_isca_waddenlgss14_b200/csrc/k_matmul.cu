@@ -37,7 +37,7 @@ constexpr int ECHUNK = 64;                   // epilogue columns per chunk
 template <int V>
 struct MmCfg {
   static constexpr int COPIES = (V == V_INTRA_SMEM) ? 2 : 1;       // operand copies in smem
-  static constexpr int ACCS = (V == V_INTRA_SMEM || V == V_INTRA_REG) ? 2 : 1;
+  static constexpr int ACCS = (V == V_INTRA_SMEM || V == V_INTRA_REG || V == V_INTRA_NOLDS) ? 2 : 1;
   static constexpr int COPY_BYTES = TILE_A + TILE_B;
   static constexpr int STAGE_BYTES = COPY_BYTES * COPIES;
   static constexpr int NSTAGE = COPIES == 2 ? 2 : 4;               // 192 KiB of operand ring
@@ -219,7 +219,9 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 1) mm_kernel(const __grid_c
     for (int i = 0; i < BM * ECHUNK / 4 / BL; ++i) {
       const int vi = rep.ltid + BL * i;
       const int r = vi / (ECHUNK / 4), c4 = (vi % (ECHUNK / 4)) * 4;
-      const float4 f = *reinterpret_cast<const float4*>(&rep.template smp<SPLANE>(stg, r * SPITCH + c4));
+      // replica r reads the staging of its own accumulator (also under -LDS: the
+      // two accumulators are the replicas' state, not kernel-written shared data)
+      const float4 f = *reinterpret_cast<const float4*>(stg + (Cfg::ACCS == 2 ? rep.r : 0) * SPLANE + r * SPITCH + c4);
       unsigned w[4] = {__float_as_uint(f.x), __float_as_uint(f.y), __float_as_uint(f.z), __float_as_uint(f.w)};
       const unsigned idx = (tm * BM + r) * a.N + tn * BN + ch * ECHUNK + c4;
       rep.template commit<4, 0>(0xFu, idx, w, a.M * a.N, [&](unsigned e, unsigned m, const unsigned* x) {

@@ -41,7 +41,7 @@ __device__ __forceinline__ unsigned block_sum_u32(const Rep<V, M>& rep, unsigned
   constexpr int NLW = BL / LW;
 #pragma unroll
   for (int m = LW / 2; m >= 1; m >>= 1) s += rep.lshfl_xor(s, m);
-  if (rep.llane == 0) rep.sm(sw, rep.ltid / LW) = s;
+  if (rep.llane == 0 && rep.sts_ok1(s, rep.ltid / LW)) rep.sm(sw, rep.ltid / LW) = s;
   __syncthreads();
   unsigned t = rep.llane < NLW ? rep.sm(sw, rep.llane) : 0u;
 #pragma unroll
@@ -54,7 +54,7 @@ template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_reduce_kernel(PsArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned sw[(BL / (32 / DUP)) * DUP];
+  __shared__ unsigned sw[(BL / (32 / DUP)) * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned ch = (unsigned)rep.lblock;
@@ -103,7 +103,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ct
   constexpr int LW = 32 / DUP;
   constexpr int NLW = BL / LW;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned sw[NLW * DUP];
+  __shared__ unsigned sw[NLW * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned ch = a.nch - 1u - (unsigned)rep.lblock;  // reverse order: L2-hot chunks first
@@ -150,7 +150,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ct
       const unsigned u = rep.lshfl_up(ws, d);
       if (rep.llane >= d) ws += u;
     }
-    if (rep.llane == LW - 1) rep.sm(sw, lw) = ws;
+    if (rep.llane == LW - 1 && rep.sts_ok1(ws, lw)) rep.sm(sw, lw) = ws;
     __syncthreads();
     unsigned wt = rep.llane < NLW ? rep.sm(sw, rep.llane) : 0u;  // every warp scans the warp totals
     if constexpr (M == M_FAULT) wt = rep.fault(SITE_SMEM, (long long)ch * BL + rep.llane * LW, wt);

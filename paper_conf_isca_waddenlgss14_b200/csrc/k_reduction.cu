@@ -29,7 +29,10 @@ __device__ __forceinline__ unsigned long long block_sum(const Rep<V, M>& rep, un
 #pragma unroll
   for (int m = LW / 2; m >= 1; m >>= 1) s += rep.lshfl_xor64(s, m);
   const int lw = rep.ltid / LW;
-  if (rep.llane == 0) rep.sm(sm_warp, lw) = s;
+  if (rep.llane == 0) {
+    const unsigned sw2[2] = {(unsigned)s, (unsigned)(s >> 32)};
+    if (rep.template sts_ok<2>(sw2, (unsigned)lw)) rep.sm(sm_warp, lw) = s;
+  }
   __syncthreads();
   unsigned long long t = 0;
   if (rep.warp == 0) {
@@ -50,7 +53,7 @@ template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) red_partial_kernel(RedArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * DUP];
+  __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned T = (unsigned)c.nblocks * BL;  // logical threads in the grid
@@ -92,7 +95,7 @@ template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) red_final_kernel(RedArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * DUP];
+  __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
   unsigned long long s = 0;

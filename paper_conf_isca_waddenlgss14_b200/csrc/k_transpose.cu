@@ -33,7 +33,7 @@ template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) tr_kernel(TrArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned tile[DUP == 2 ? PLANE + SWORDS : SWORDS];
+  __shared__ unsigned tile[Geom<V>::SMDUP == 2 ? PLANE + SWORDS : SWORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned ty = (unsigned)rep.lblock / a.nsx, sx = (unsigned)rep.lblock % a.nsx;
@@ -51,10 +51,13 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) tr_kernel(TrArgs a, Ctx c) 
   for (int t = 0; t < NT; ++t) {
     unsigned w[4] = {v[t].x, v[t].y, v[t].z, v[t].w};
     const unsigned gj = sx * (NT * TS) + t * TS + l4;
+    if constexpr (M == M_FAULT) {
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      if constexpr (M == M_FAULT) w[k] = rep.fault(SITE_LOAD, (long long)gi * a.W + gj + k, w[k]);
-      rep.template smp<PLANE>(tile, t * TWORDS + r * PITCH + l4 + k) = w[k];
+      for (int k = 0; k < 4; ++k) w[k] = rep.fault(SITE_LOAD, (long long)gi * a.W + gj + k, w[k]);
+    }
+    if (rep.template sts_ok<4>(w, t * TWORDS + r * PITCH + l4)) {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) rep.template smp<PLANE>(tile, t * TWORDS + r * PITCH + l4 + k) = w[k];
     }
   }
   __syncthreads();

@@ -42,7 +42,7 @@ const KEntry kTable[RMT_K_COUNT] = {
     KE(matmul, 2, 0, 1, 1, 2, 0),
 };
 
-const char* kVariantNames[5] = {"none", "intra_smem", "intra_reg", "inter_group", "inter_cluster"};
+const char* kVariantNames[6] = {"none", "intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds"};
 
 int check_device() {
   static int ok_dev = -1;
@@ -91,7 +91,7 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
                void* workspace, size_t ws_bytes, void* stream) {
   g_last_launches = 0;
   if (kernel < 0 || kernel >= RMT_K_COUNT) { set_error("bad kernel id"); return RMT_EINVAL; }
-  if (variant < 0 || variant > RMT_INTER_CLUSTER) { set_error("bad variant id"); return RMT_EINVAL; }
+  if (variant < 0 || variant > RMT_INTRA_NOLDS) { set_error("bad variant id"); return RMT_EINVAL; }
   if (!bufs || !err_count) { set_error("bufs and err_count must be non-NULL"); return RMT_EINVAL; }
   int rc = check_device();
   if (rc) return rc;
@@ -138,7 +138,7 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
 }
 
 size_t rmt_workspace_size(int kernel, int variant, int64_t n, const int64_t* dims) {
-  if (kernel < 0 || kernel >= RMT_K_COUNT || variant < 0 || variant > RMT_INTER_CLUSTER) return 0;
+  if (kernel < 0 || kernel >= RMT_K_COUNT || variant < 0 || variant > RMT_INTRA_NOLDS) return 0;
   int64_t zero[4] = {0, 0, 0, 0};
   return ws_size(kernel, variant, n, dims ? dims : zero, nullptr);
 }
@@ -229,7 +229,7 @@ const char* rmt_kernel_name(int kernel) {
 }
 
 const char* rmt_variant_name(int variant) {
-  return (variant >= 0 && variant <= RMT_INTER_CLUSTER) ? kVariantNames[variant] : "?";
+  return (variant >= 0 && variant <= RMT_INTRA_NOLDS) ? kVariantNames[variant] : "?";
 }
 
 }  // extern "C"

@@ -1,7 +1,7 @@
 // rmt_device.cuh -- device-side RMT policies for sm_100a.
 //
 // One kernel body is written once and instantiated per variant V and mode MODE:
-//   V    = V_NONE | V_INTRA_SMEM | V_INTRA_REG | V_INTER      (include/rmt.h)
+//   V    = V_NONE | V_INTRA_SMEM | V_INTRA_REG | V_INTER | V_CLUSTER | V_INTRA_NOLDS  (include/rmt.h)
 //   MODE = M_NORMAL | M_FAULT (single-bit fault hooks compiled in) | M_NOCOMM
 //          (ablation: replicas run, no exchange/compare)
 //
@@ -33,7 +33,7 @@
 
 namespace rmt {
 
-constexpr int V_NONE = 0, V_INTRA_SMEM = 1, V_INTRA_REG = 2, V_INTER = 3, V_CLUSTER = 4;
+constexpr int V_NONE = 0, V_INTRA_SMEM = 1, V_INTRA_REG = 2, V_INTER = 3, V_CLUSTER = 4, V_INTRA_NOLDS = 5;
 constexpr int M_NORMAL = 0, M_FAULT = 1, M_NOCOMM = 2;
 constexpr int SITE_LOAD = 0, SITE_COMPUTE = 1, SITE_SMEM = 2, SITE_STORE_VAL = 3, SITE_STORE_ADDR = 4;
 constexpr int MAXW = 4;               // max value words per commit
@@ -42,8 +42,11 @@ constexpr int MBOX_WORDS = RING_WORDS * 16;  // intra_smem mailbox words per war
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int CTRL_TURN = 64;         // ctrl[64 ..) = per-region turn counters
 constexpr unsigned long long WATCHDOG_CYCLES = 1ull << 32;  // ~2 s at 2 GHz
-constexpr int CL_S = 4;     // inter_cluster: mailbox slots per warp (in the consumer CTA's smem)
-constexpr int CL_MAXW = 8;  // inter_cluster: max warps per CTA
+// inter_cluster: record slots per warp in the consumer CTA's shared memory
+// (Ctx::S, a power of two chosen by the launcher): 8 lets the producer fill one
+// deferred batch (<= 4 records) while the consumer drains the previous one; 4
+// when a larger mailbox would cost occupancy (CTAs of more than 4 warps).
+constexpr int CL_S_SMALL = 4, CL_S_LARGE = 8;
 
 struct FaultDesc {
   int replica, site, bit, sid;
@@ -172,7 +175,11 @@ __device__ __forceinline__ bool spin_cl(unsigned addr, unsigned want, const Ctx&
 // ---------------------------------------------------------------- replica state
 template <int V, int MODE>
 struct Rep {
-  static constexpr bool INTRA = (V == V_INTRA_SMEM || V == V_INTRA_REG);
+  static constexpr bool INTRA = (V == V_INTRA_SMEM || V == V_INTRA_REG || V == V_INTRA_NOLDS);
+  // +LDS: kernel-written shared memory duplicated per replica;
+  // -LDS (intra_nolds): one copy, every kernel st.shared compared
+  static constexpr bool SMDUP = (V == V_INTRA_SMEM || V == V_INTRA_REG);
+  static constexpr bool NOLDS = (V == V_INTRA_NOLDS);
   static constexpr bool INTER = (V == V_INTER);
   static constexpr bool CLUSTER = (V == V_CLUSTER);
   static constexpr int DUP = INTRA ? 2 : 1;  // physical threads per logical thread
@@ -230,17 +237,22 @@ struct Rep {
       // "co-scheduling" remark); rank 0 = producer, rank 1 = consumer.  Records go
       // into a mailbox in the CONSUMER's shared memory through distributed
       // shared memory (DSMEM), not through L2.
-      __shared__ __align__(16) unsigned cl_payload[CL_MAXW * CL_S * RING_WORDS * 32];
-      __shared__ unsigned cl_flags[CL_MAXW * CL_S];
+      // The mailbox is appended to the dynamic shared memory at byte offset c.R
+      // (launch_std): per warp c.S records of RING_WORDS x 32 words, then c.S flags.
+      extern __shared__ __align__(16) unsigned char rmt_dyn_smem[];
       r = (int)cluster_ctarank();
       consumer = (r == 1);
       lblock = (int)cluster_id_x();
       ltid = threadIdx.x;
       llane = lane;
       if constexpr (!NOCOMM) {
-        for (int i = threadIdx.x; i < CL_MAXW * CL_S; i += blockDim.x) cl_flags[i] = 0u;
-        unsigned pb = (unsigned)__cvta_generic_to_shared(cl_payload) + (unsigned)(warp * CL_S * RING_WORDS * 32) * 4u;
-        unsigned fb = (unsigned)__cvta_generic_to_shared(cl_flags) + (unsigned)(warp * CL_S) * 4u;
+        const unsigned nw = blockDim.x >> 5;
+        const unsigned base = (unsigned)__cvta_generic_to_shared(rmt_dyn_smem) + (unsigned)c.R;
+        const unsigned fl0 = base + nw * (unsigned)(c.S * RING_WORDS * 32) * 4u;
+        unsigned* flp = (unsigned*)__cvta_shared_to_generic(fl0);
+        for (unsigned i = threadIdx.x; i < nw * (unsigned)c.S; i += blockDim.x) flp[i] = 0u;
+        unsigned pb = base + (unsigned)(warp * c.S * RING_WORDS * 32) * 4u;
+        unsigned fb = fl0 + (unsigned)(warp * c.S) * 4u;
         cl_pay = consumer ? pb : mapa_rank(pb, 1u);
         cl_full = consumer ? fb : mapa_rank(fb, 1u);
         cluster_sync_all();  // both mailboxes initialised before any record
@@ -270,10 +282,10 @@ struct Rep {
       if (!consumer) {
         asm volatile("fence.acq_rel.cluster;" ::: "memory");
         __syncwarp();
-        if ((unsigned)lane < pend) st_relaxed_cl(cl_full + ((first + lane) % CL_S) * 4u, 1u);
+        if ((unsigned)lane < pend) st_relaxed_cl(cl_full + ((first + lane) & (unsigned)(c.S - 1)) * 4u, 1u);
       } else {
         __syncwarp();
-        if ((unsigned)lane < pend) st_release_cl(cl_full + ((first + lane) % CL_S) * 4u, 0u);
+        if ((unsigned)lane < pend) st_release_cl(cl_full + ((first + lane) & (unsigned)(c.S - 1)) * 4u, 0u);
       }
       pend = 0u;
     }
@@ -322,7 +334,7 @@ struct Rep {
   // ---- duplicated shared memory (+LDS): replica r owns its interleaved copy
   template <class T>
   __device__ __forceinline__ T& sm(T* base, int i) const {
-    if constexpr (INTRA) return base[2 * i + r];
+    if constexpr (SMDUP) return base[2 * i + r];
     else return base[i];
   }
 
@@ -331,8 +343,34 @@ struct Rep {
   // banks for that kernel's access patterns (interleaving conflicts otherwise).
   template <int PLANE, class T>
   __device__ __forceinline__ T& smp(T* base, int i) const {
-    if constexpr (INTRA) return base[PLANE * r + i];
+    if constexpr (SMDUP) return base[PLANE * r + i];
     else return base[i];
+  }
+
+  // ---- -LDS shared stores (intra_nolds).  The pair shares one copy of the
+  // kernel's shared memory, so a shared store leaves the sphere of replication
+  // ("-LDS ... communicate ... on every LDS write"): the replicas
+  // exchange (index, words) through registers and compare; a mismatch counts one
+  // error; the store is performed once, by the consumer, with its own value.
+  // Returns whether this lane performs the store (every other variant: true).
+  // Both lanes of the pair must call it together (they always share control flow).
+  template <int NW>
+  __device__ __forceinline__ bool sts_ok(const unsigned (&w)[NW], unsigned i) const {
+    if constexpr (!NOLDS) {
+      return true;
+    } else {
+      if constexpr (NOCOMM) return consumer;
+      const unsigned pm = 3u << (lane & ~1);
+      bool mism = __shfl_xor_sync(pm, i, 1) != i;
+#pragma unroll
+      for (int k = 0; k < NW; ++k) mism |= __shfl_xor_sync(pm, w[k], 1) != w[k];
+      if (mism && consumer) atomicAdd(c.err, 1ull);
+      return consumer;
+    }
+  }
+  __device__ __forceinline__ bool sts_ok1(unsigned w, unsigned i) const {
+    const unsigned a[1] = {w};
+    return sts_ok<1>(a, i);
   }
 
   // ---- logical-warp shuffles (replica-private: lanes keep their role bit)
@@ -367,7 +405,10 @@ struct Rep {
   // ---- fault hooks (compiled out unless MODE == M_FAULT)
   __device__ __forceinline__ unsigned fault(int site, long long elem, unsigned x) const {
     if constexpr (FAULT) {
-      if (c.f.site == site && c.f.elem == elem && c.f.replica == r) x ^= 1u << c.f.bit;
+      // -LDS: a SMEM-site fault corrupts the single shared copy, i.e. what both
+      // replicas read (shared memory is outside this variant's SoR)
+      if (c.f.site == site && c.f.elem == elem && (c.f.replica == r || (NOLDS && site == SITE_SMEM)))
+        x ^= 1u << c.f.bit;
     }
     return x;
   }
@@ -444,7 +485,7 @@ struct Rep {
       else key = mask ? (((idx / NW) << NW) | mask) : 0u;
       unsigned pk = 0, pv[NW];
       bool have = true;  // consumer got the producer's record
-      if constexpr (V == V_INTRA_REG) {
+      if constexpr (V == V_INTRA_REG || V == V_INTRA_NOLDS) {
         pk = __shfl_xor_sync(FULL, key, 1);
 #pragma unroll
         for (int k = 0; k < NW; ++k) pv[k] = __shfl_xor_sync(FULL, v[k], 1);
@@ -463,11 +504,11 @@ struct Rep {
         }
         __syncwarp();
       } else if constexpr (V == V_CLUSTER) {  // DSMEM mailbox in the consumer CTA
-        const unsigned slot = j % CL_S;
+        const unsigned slot = j & (unsigned)(c.S - 1);
         const unsigned pa = cl_pay + (slot * RING_WORDS * 32 + lane) * 4u;
         const unsigned fa = cl_full + slot * 4u;
         if (!consumer) {
-          if (j >= (unsigned)CL_S) {  // publish ours first, then wait for a free slot
+          if (j >= (unsigned)c.S) {  // publish ours first, then wait for a free slot
             flush();
             spin_cl(fa, 0u, c, lane == 0);
           }
@@ -537,7 +578,8 @@ struct Rep {
 // ---------------------------------------------------------------- launch geometry
 template <int V>
 struct Geom {
-  static constexpr int DUP = (V == V_INTRA_SMEM || V == V_INTRA_REG) ? 2 : 1;
+  static constexpr int DUP = (V == V_INTRA_SMEM || V == V_INTRA_REG || V == V_INTRA_NOLDS) ? 2 : 1;
+  static constexpr int SMDUP = (V == V_INTRA_SMEM || V == V_INTRA_REG) ? 2 : 1;  // kernel smem copies
   static __host__ __device__ unsigned grid(unsigned lblocks) {
     return (V == V_INTER || V == V_CLUSTER) ? 2u * lblocks : lblocks;
   }

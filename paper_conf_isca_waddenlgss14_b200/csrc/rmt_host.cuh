@@ -63,6 +63,10 @@ int dispatch(int v, int m, F&& f) {
       return m == M_FAULT ? f(VM<V_INTER, M_FAULT>{})
            : m == M_NOCOMM ? f(VM<V_INTER, M_NOCOMM>{})
                            : f(VM<V_INTER, M_NORMAL>{});
+    case V_INTRA_NOLDS:
+      return m == M_FAULT ? f(VM<V_INTRA_NOLDS, M_FAULT>{})
+           : m == M_NOCOMM ? f(VM<V_INTRA_NOLDS, M_NOCOMM>{})
+                           : f(VM<V_INTRA_NOLDS, M_NORMAL>{});
     case V_CLUSTER:
       return m == M_FAULT ? f(VM<V_CLUSTER, M_FAULT>{})
            : m == M_NOCOMM ? f(VM<V_CLUSTER, M_NOCOMM>{})
@@ -140,11 +144,19 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
       cudaFuncSetAttribute(kn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem + pad));
     kn<<<G, BL, smem + pad, L.stream>>>(a, c);
   } else if constexpr (V == V_CLUSTER) {
-    if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    // the DSMEM mailbox (rmt_device.cuh, Rep::init) follows the kernel's own
+    // dynamic shared memory
+    size_t dyn = smem;
+    if (L.mode != M_NOCOMM) {
+      c.R = (int)align_up(smem, 16);
+      c.S = BL <= 128 ? CL_S_LARGE : CL_S_SMALL;
+      dyn = (size_t)c.R + (size_t)(BL / 32) * c.S * (RING_WORDS * 32 + 1) * 4;
+    }
+    cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(Geom<V>::grid(G));
     cfg.blockDim = dim3(Geom<V>::block(BL));
-    cfg.dynamicSmemBytes = smem;
+    cfg.dynamicSmemBytes = dyn;
     cfg.stream = L.stream;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;

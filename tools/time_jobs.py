@@ -6,6 +6,8 @@ import torch
 from paper_conf_isca_waddenlgss14_b200 import rmt, workloads
 
 cfg = sys.argv[1]
+if os.environ.get("RMT_ABL"):  # full | nocomm | inflate
+    rmt.set_ablation(os.environ["RMT_ABL"])
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 variants = sys.argv[3].split(",") if len(sys.argv) > 3 else ["none", "intra_smem", "intra_reg", "inter_group", "inter_cluster"]
 for j in workloads.config_jobs(cfg):
