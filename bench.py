@@ -4,7 +4,7 @@
 
 One step = one pass of the whole hot path over one batch of synthetic input:
 every kernel of the config launched once under each variant
-(none, intra_smem, intra_reg, inter_group, inter_cluster) through the C ABI (librmt.so).
+(none, intra_smem, intra_reg, inter_group) through the C ABI (librmt.so).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config suite] [--impl rmt|reference]
 
@@ -31,7 +31,9 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "RMT slowdown vs unprotected kernel per variant; baseline HBM GB/s vs peak"
-VARIANTS = ("none", "intra_smem", "intra_reg", "inter_group", "inter_cluster")
+VARIANTS = ("none", "intra_smem", "intra_reg", "inter_group")
+# B200 extensions: measured after the timed step, not part of it
+EXTRA_VARIANTS = ("inter_cluster", "intra_nolds")
 
 
 def parse():
@@ -44,6 +46,8 @@ def parse():
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--variants", default=",".join(VARIANTS))
+    p.add_argument("--extra-variants", default=",".join(EXTRA_VARIANTS),
+                   help="variants timed per launch after the timed region (reported, not in the step)")
     p.add_argument("--ablations", action="store_true",
                    help="also time the INFLATE and NOCOMM ablations per kernel x RMT variant (cost attribution)")
     p.add_argument("--dist-backend", default="nccl",
@@ -397,6 +401,37 @@ def main():
             attribution[j.kernel] = d
         err.zero_()
 
+    # B200-native extension variants: per-launch medians outside the timed step
+    extra = None
+    xvars = [v for v in args.extra_variants.split(",") if v and v not in variants]
+    if xvars and "none" in variants:
+        extra = {"kernels": {}, "slowdown_geomean": {}}
+        xs = {v: [] for v in xvars}
+        err.zero_()
+        for j in jobs:
+            d = {}
+            for v in xvars:
+                wsx = rmt.make_workspace(j.kernel, v, j.n, j.dims)
+                ts = []
+                for r in range(5):
+                    a = torch.cuda.Event(enable_timing=True)
+                    b = torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
+                    rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=wsx, stream=stream.cuda_stream)
+                    b.record(stream)
+                    torch.cuda.synchronize()
+                    if r:
+                        ts.append(a.elapsed_time(b))
+                ms = statistics.median(ts)
+                sd = ms / per[(j.kernel, "none")]
+                d[v] = {"ms": round(ms, 4), "slowdown": round(sd, 3)}
+                xs[v].append(sd)
+                del wsx
+            extra["kernels"][j.kernel] = d
+        extra["slowdown_geomean"] = {v: round(math.exp(sum(math.log(x) for x in s_) / len(s_)), 3)
+                                     for v, s_ in xs.items()}
+        extra["err_count"] = int(err.item())
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rate, secs, cores, desc = oracle_sample_rate(jobs)
@@ -416,7 +451,7 @@ def main():
                                "gbs": kernels[best_none.kernel]["none"]["gbs"],
                                "frac": kernels[best_none.kernel]["none"]["frac"]} if best_none else None),
             "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
-            "attribution": attribution,
+            "attribution": attribution, "extra_variants": extra,
             "gpu_launches": counts["gpu_launches"], "err_count": errs,
             "clocks": clk.summary(),
         }

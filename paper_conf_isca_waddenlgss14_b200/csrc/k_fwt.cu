@@ -19,10 +19,24 @@ namespace {
 constexpr int BL = 256;
 constexpr int TB_MAX = 12;
 constexpr int TE_MAX = 1 << TB_MAX;
-constexpr int SM_WORDS = TE_MAX + TE_MAX / 32;  // pad32 swizzle: <=2-way conflicts for all rounds
-constexpr int PLANE = SM_WORDS + 16;            // intra replica plane: 16 banks apart (fewest conflicts over all rounds)
-
-__device__ __forceinline__ int phys(int e) { return e + (e >> 5); }
+// Tile swizzle.  One replica per warp lane (none, inter): pad one word per 32
+// ("pad32"), conflict-free for the 32-thread patterns of every round.  Two
+// replicas per warp (+LDS intra variants, P16): each replica has 16 logical
+// threads; pad one word per 16 makes every round's 16-thread pattern hit 16
+// banks whose complement is the same set + 16, so the replica planes sit 16
+// banks apart (PLANE = 16 mod 32) and a pair never conflicts.
+template <bool P16>
+struct Swz {
+  static constexpr int WORDS = TE_MAX + TE_MAX / (P16 ? 16 : 32);
+  static constexpr int PLANE = WORDS + 16;  // replica plane offset (== 16 mod 32)
+  static __device__ __forceinline__ int phys(int e) { return e + (e >> (P16 ? 4 : 5)); }
+  // phys(ebase | k << Q) - phys(ebase) for ebase with zeros in bits Q..Q+3
+  template <int Q>
+  static __device__ __forceinline__ constexpr int coff(int k) {
+    if constexpr (P16) return (k << Q) + ((k << Q) >> 4);
+    else return (k << Q) + ((Q >= 5) ? (k << (Q - 5)) : ((k << Q) >> 5));
+  }
+};
 
 struct FwtArgs {
   const float* src;
@@ -42,11 +56,28 @@ __device__ __forceinline__ unsigned gindex(const FwtArgs& a, unsigned tile, unsi
   return (hi << (a.s0 + a.b)) | (st << a.s0) | (mid << a.c) | col;
 }
 
+// gindex with the pass shape known at compile time (KIND 1: s0 = 0, tb = 12;
+// KIND 2: b = 7, c = 5)
+template <int KIND>
+__device__ __forceinline__ unsigned gindex_k(const FwtArgs& a, unsigned tile, unsigned e) {
+  if constexpr (KIND == 1) {
+    return (tile << TB_MAX) | e;
+  } else if constexpr (KIND == 2) {
+    const unsigned col = e & 31u, st = e >> 5;
+    const int midb = a.s0 - 5;
+    const unsigned mid = tile & ((1u << midb) - 1u), hi = tile >> midb;
+    return (hi << (a.s0 + 7)) | (st << a.s0) | (mid << 5) | col;
+  } else {
+    return gindex(a, tile, e);
+  }
+}
+
 // One register round: NB consecutive stages at tile-bit q on groups of 2^NB.
 template <int NB, class R>
-__device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int te, const FwtArgs& a, unsigned tileid,
+__device__ __forceinline__ void fwt_round(const R& rep, float* tp, int q, int te, const FwtArgs& a, unsigned tileid,
                                           int round_no) {
   constexpr int G = 1 << NB;
+  using S = Swz<R::SMDUP>;
   const int groups = te >> NB;
   for (int gi = rep.ltid; gi < groups; gi += BL) {
     const int lowmask = (1 << q) - 1;
@@ -54,7 +85,7 @@ __device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int 
     float v[G];
 #pragma unroll
     for (int k = 0; k < G; ++k) {
-      v[k] = rep.template smp<PLANE>(tile, phys(ebase | (k << q)));
+      v[k] = tp[S::phys(ebase | (k << q))];
       if constexpr (R::FAULT) {
         if (a.s0 == 0 && round_no == 1)
           v[k] = rep.faultf(SITE_SMEM, (long long)gindex(a, tileid, ebase | (k << q)), v[k]);
@@ -82,7 +113,7 @@ __device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int 
     }
     if (rep.template sts_ok<G>(vw, (unsigned)ebase)) {
 #pragma unroll
-      for (int k = 0; k < G; ++k) rep.template smp<PLANE>(tile, phys(ebase | (k << q))) = v[k];
+      for (int k = 0; k < G; ++k) tp[S::phys(ebase | (k << q))] = v[k];
     }
   }
 }
@@ -90,24 +121,21 @@ __device__ __forceinline__ void fwt_round(const R& rep, float* tile, int q, int 
 // Compile-time round (full 4096-element tile): with Q known, phys(ebase | k<<Q)
 // = phys(ebase) + C(k) with a constant C(k) (ebase has zeros in bits Q..Q+NB),
 // so every element costs one LDS and one STS with an immediate offset.
-template <int NB, int Q>
-__device__ __forceinline__ constexpr int coff(int k) {
-  return (k << Q) + ((Q >= 5) ? (k << (Q - 5)) : ((k << Q) >> 5));
-}
 template <int NB, int Q, class R>
-__device__ __forceinline__ void fwt_round_ct(const R& rep, float* tile, const FwtArgs& a, unsigned tileid,
+__device__ __forceinline__ void fwt_round_ct(const R& rep, float* tp, const FwtArgs& a, unsigned tileid,
                                              int round_no) {
   constexpr int G = 1 << NB;
   constexpr int GPT = (TE_MAX >> NB) / BL;  // groups per thread
+  using S = Swz<R::SMDUP>;
 #pragma unroll
   for (int w = 0; w < GPT; ++w) {
     const int gi = rep.ltid + BL * w;
     const int ebase = (gi & ((1 << Q) - 1)) | ((gi >> Q) << (Q + NB));
-    float* pb = &rep.template smp<PLANE>(tile, phys(ebase));
+    float* pb = tp + S::phys(ebase);
     float v[G];
 #pragma unroll
     for (int k = 0; k < G; ++k) {
-      v[k] = pb[coff<NB, Q>(k)];
+      v[k] = pb[S::template coff<Q>(k)];
       if constexpr (R::FAULT) {
         if (a.s0 == 0 && round_no == 1)
           v[k] = rep.faultf(SITE_SMEM, (long long)gindex(a, tileid, ebase | (k << Q)), v[k]);
@@ -135,7 +163,7 @@ __device__ __forceinline__ void fwt_round_ct(const R& rep, float* tile, const Fw
     }
     if (rep.template sts_ok<G>(vw, (unsigned)ebase)) {
 #pragma unroll
-      for (int k = 0; k < G; ++k) pb[coff<NB, Q>(k)] = v[k];
+      for (int k = 0; k < G; ++k) pb[S::template coff<Q>(k)] = v[k];
     }
   }
 }
@@ -146,15 +174,18 @@ __device__ __forceinline__ void fwt_round_ct(const R& rep, float* tile, const Fw
 template <int V, int M, int KIND>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
+  using S = Swz<Rep<V, M>::SMDUP>;
+  constexpr int PLANE = S::PLANE;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ float tile[Geom<V>::SMDUP == 2 ? PLANE + SM_WORDS : SM_WORDS];
+  __shared__ float tile[Geom<V>::SMDUP == 2 ? PLANE + S::WORDS : S::WORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned tileid = (unsigned)rep.lblock;
-  const int te = 1 << a.tb;
+  const int te = KIND != 0 ? TE_MAX : 1 << a.tb;  // full tiles in the specialised passes
+  float* const tp = &rep.template smp<PLANE>(tile, 0);  // this replica's plane
   // load: 16-B vectors, contiguous in both the tile and global memory
   for (int e0 = 4 * rep.ltid; e0 < te; e0 += 4 * BL) {
-    const unsigned g = gindex(a, tileid, (unsigned)e0);
+    const unsigned g = gindex_k<KIND>(a, tileid, (unsigned)e0);
     float w[4];
     if (te >= 4) {
       float4 f = *reinterpret_cast<const float4*>(a.src + g);
@@ -176,32 +207,32 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
     if (rep.template sts_ok<4>(xw, (unsigned)e0)) {
 #pragma unroll
       for (int k = 0; k < 4; ++k)
-        if (e0 + k < te) rep.template smp<PLANE>(tile, phys(e0 + k)) = w[k];
+        if (e0 + k < te) tp[S::phys(e0 + k)] = w[k];
     }
   }
   __syncthreads();
   // stages [s0, s0 + b) live at tile bits [c, c + b); rounds of <= 4 stages
   if constexpr (KIND == 1) {
-    fwt_round_ct<4, 0>(rep, tile, a, tileid, 0);
+    fwt_round_ct<4, 0>(rep, tp, a, tileid, 0);
     __syncthreads();
-    fwt_round_ct<4, 4>(rep, tile, a, tileid, 1);
+    fwt_round_ct<4, 4>(rep, tp, a, tileid, 1);
     __syncthreads();
-    fwt_round_ct<4, 8>(rep, tile, a, tileid, 2);
+    fwt_round_ct<4, 8>(rep, tp, a, tileid, 2);
     __syncthreads();
   } else if constexpr (KIND == 2) {
-    fwt_round_ct<4, 5>(rep, tile, a, tileid, 0);
+    fwt_round_ct<4, 5>(rep, tp, a, tileid, 0);
     __syncthreads();
-    fwt_round_ct<3, 9>(rep, tile, a, tileid, 1);
+    fwt_round_ct<3, 9>(rep, tp, a, tileid, 1);
     __syncthreads();
   } else {
     int round_no = 0;
     for (int q = a.c; q < a.c + a.b; q += 4, ++round_no) {
       const int nb = min(4, a.c + a.b - q);
       switch (nb) {
-        case 4: fwt_round<4>(rep, tile, q, te, a, tileid, round_no); break;
-        case 3: fwt_round<3>(rep, tile, q, te, a, tileid, round_no); break;
-        case 2: fwt_round<2>(rep, tile, q, te, a, tileid, round_no); break;
-        default: fwt_round<1>(rep, tile, q, te, a, tileid, round_no); break;
+        case 4: fwt_round<4>(rep, tp, q, te, a, tileid, round_no); break;
+        case 3: fwt_round<3>(rep, tp, q, te, a, tileid, round_no); break;
+        case 2: fwt_round<2>(rep, tp, q, te, a, tileid, round_no); break;
+        default: fwt_round<1>(rep, tp, q, te, a, tileid, round_no); break;
       }
       __syncthreads();
     }
@@ -214,11 +245,11 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
     unsigned mask = 0;
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      const bool in = e0 + k < te;
-      w[k] = in ? __float_as_uint(rep.template smp<PLANE>(tile, phys(e0 + k))) : 0u;
+      const bool in = KIND != 0 || e0 + k < te;  // specialised passes: full tiles
+      w[k] = in ? __float_as_uint(tp[S::phys(e0 + k)]) : 0u;
       mask |= (in ? 1u : 0u) << k;
     }
-    const unsigned g = e0 < te ? gindex(a, tileid, (unsigned)e0) : 0u;
+    const unsigned g = e0 < te ? gindex_k<KIND>(a, tileid, (unsigned)e0) : 0u;
     rep.template commit<4, 0>(mask, g, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
       if (m == 0xFu)
         *reinterpret_cast<float4*>(a.dst + idx) =

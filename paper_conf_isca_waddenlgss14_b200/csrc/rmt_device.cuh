@@ -551,9 +551,11 @@ struct Rep {
       }
       bool mism = false;
       if (consumer) {
-        bool eq = have && (pk == key);
+        // bitwise difference of key (address + predicate) and of the stored words
+        unsigned d = pk ^ key;
 #pragma unroll
-        for (int k = 0; k < NW; ++k) eq = eq && (!((mask >> k) & 1u) || pv[k] == v[k]);
+        for (int k = 0; k < NW; ++k) d |= (pv[k] ^ v[k]) & (0u - ((mask >> k) & 1u));
+        const bool eq = have && d == 0u;
         if (eq) {
           if (mask != 0u) store(idx, mask, v);
         } else {
