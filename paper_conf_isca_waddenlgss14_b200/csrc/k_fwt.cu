@@ -184,30 +184,46 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
   const int te = KIND != 0 ? TE_MAX : 1 << a.tb;  // full tiles in the specialised passes
   float* const tp = &rep.template smp<PLANE>(tile, 0);  // this replica's plane
   // load: 16-B vectors, contiguous in both the tile and global memory
-  for (int e0 = 4 * rep.ltid; e0 < te; e0 += 4 * BL) {
-    const unsigned g = gindex_k<KIND>(a, tileid, (unsigned)e0);
-    float w[4];
-    if (te >= 4) {
-      float4 f = *reinterpret_cast<const float4*>(a.src + g);
-      w[0] = f.x; w[1] = f.y; w[2] = f.z; w[3] = f.w;
-    } else {
-#pragma unroll
-      for (int k = 0; k < 4; ++k) w[k] = e0 + k < te ? a.src[g + k] : 0.0f;
-    }
+  auto put4 = [&](int e0, unsigned g, float (&w)[4]) {
     unsigned xw[4];
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      float x = w[k];
       if constexpr (M == M_FAULT) {
-        if (a.s0 == 0 && e0 + k < te) x = rep.faultf(SITE_LOAD, (long long)g + k, x);
+        if (a.s0 == 0 && e0 + k < te) w[k] = rep.faultf(SITE_LOAD, (long long)g + k, w[k]);
       }
-      w[k] = x;
-      xw[k] = __float_as_uint(x);
+      xw[k] = __float_as_uint(w[k]);
     }
     if (rep.template sts_ok<4>(xw, (unsigned)e0)) {
 #pragma unroll
       for (int k = 0; k < 4; ++k)
-        if (e0 + k < te) tp[S::phys(e0 + k)] = w[k];
+        if (KIND != 0 || e0 + k < te) tp[S::phys(e0 + k)] = w[k];
+    }
+  };
+  if constexpr (KIND != 0) {
+    // full tile: all of this thread's loads in flight before the first use
+    constexpr int IT = TE_MAX / (4 * BL);
+    float4 f[IT];
+#pragma unroll
+    for (int it = 0; it < IT; ++it)
+      f[it] = *reinterpret_cast<const float4*>(a.src + gindex_k<KIND>(a, tileid, (unsigned)(4 * rep.ltid + it * 4 * BL)));
+#pragma unroll
+    for (int it = 0; it < IT; ++it) {
+      const int e0 = 4 * rep.ltid + it * 4 * BL;
+      float w[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
+      put4(e0, gindex_k<KIND>(a, tileid, (unsigned)e0), w);
+    }
+  } else {
+    for (int e0 = 4 * rep.ltid; e0 < te; e0 += 4 * BL) {
+      const unsigned g = gindex(a, tileid, (unsigned)e0);
+      float w[4];
+      if (te >= 4) {
+        float4 f = *reinterpret_cast<const float4*>(a.src + g);
+        w[0] = f.x; w[1] = f.y; w[2] = f.z; w[3] = f.w;
+      } else {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) w[k] = e0 + k < te ? a.src[g + k] : 0.0f;
+      }
+      put4(e0, g, w);
     }
   }
   __syncthreads();
