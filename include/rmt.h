@@ -195,6 +195,13 @@ int rmt_set_ablation(int mode);
 /* Kernel launches the last rmt_launch issued (for the bench's launch count). */
 int rmt_last_launch_count(void);
 
+/* Diagnostic: launch `pairs` 2-CTA clusters and
+ * report in *same_sm_pairs how many had both CTAs on the same SM (read from
+ * %smid).  0 means every inter_cluster pair spans two SMs, so the SM-private
+ * structures (L1, LSU, schedulers) are inside that variant's sphere of
+ * replication.  Synchronous; allocates and frees its own device buffer. */
+int rmt_probe_cluster_placement(int64_t pairs, int64_t* same_sm_pairs);
+
 const char* rmt_strerror(int code);
 const char* rmt_last_error(void); /* thread-local detail of the last failure */
 const char* rmt_kernel_name(int kernel);

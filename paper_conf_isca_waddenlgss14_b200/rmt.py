@@ -84,6 +84,8 @@ def lib() -> ctypes.CDLL:
         L.rmt_kernel_name.restype = ctypes.c_char_p
         L.rmt_variant_name.argtypes = [I32]
         L.rmt_variant_name.restype = ctypes.c_char_p
+        L.rmt_probe_cluster_placement.argtypes = [I64, ctypes.POINTER(ctypes.c_int64)]
+        L.rmt_probe_cluster_placement.restype = I32
         _lib = L
     return _lib
 
@@ -184,3 +186,10 @@ def set_ablation(mode):
 
 def last_launch_count() -> int:
     return lib().rmt_last_launch_count()
+
+
+def probe_cluster_placement(pairs: int = 4096) -> int:
+    """Pairs (of `pairs` 2-CTA clusters) whose two CTAs shared one SM."""
+    out = ctypes.c_int64(-1)
+    _check(lib().rmt_probe_cluster_placement(int(pairs), ctypes.byref(out)), "rmt_probe_cluster_placement")
+    return out.value

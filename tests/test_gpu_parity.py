@@ -107,3 +107,11 @@ def test_prefixsum_carry_in(variant):
     y = c.outputs(b)[0].astype(np.uint64)
     ref = (oracle.prefixsum_u32(c.x).astype(np.uint64) + carry) % 2**32
     assert np.array_equal(y, ref)
+
+
+def test_cluster_placement_probe():
+    """inter_cluster SoR: how often do the two CTAs of a pair share an SM?"""
+    pairs = 4096
+    same = rmt.probe_cluster_placement(pairs)
+    assert 0 <= same <= pairs
+    print(f"cluster pairs sharing an SM: {same}/{pairs}")
