@@ -62,6 +62,13 @@ def lib():
         L.orc_dct8x8_absbound.argtypes = [P, I, I, P]
         L.orc_matmul_bf16.argtypes = [P, P, I, I, I, P]
         L.orc_matmul_bf16_sampled.argtypes = [P, P, I, I, P, P, P, P]
+        L.orc_sort_u32.argtypes = [P, I, P]
+        L.orc_dwthaar1d_f64.argtypes = [P, I, P]
+        L.orc_dwthaar1d_f32dag.argtypes = [P, I, P]
+        L.orc_crr_price.argtypes = [D, D, D, D, D, I, ctypes.c_int]
+        L.orc_crr_price.restype = D
+        L.orc_bo_params.argtypes = [D, P, P, P]
+        L.orc_binomialoption.argtypes = [P, I, P]
         _lib = L
     return _lib
 
@@ -199,3 +206,44 @@ def matmul_bf16_sampled(A: np.ndarray, Bt: np.ndarray, rows: np.ndarray, cols: n
     lib().orc_matmul_bf16_sampled(_p(A), _p(Bt), A.shape[1], rows.size, _p(rows), _p(cols),
                                   _p(out), _p(absout))
     return out, absout
+
+
+def sort_u32(keys: np.ndarray) -> np.ndarray:
+    keys = np.ascontiguousarray(keys, dtype=np.uint32)
+    out = np.empty_like(keys)
+    lib().orc_sort_u32(_p(keys), keys.size, _p(out))
+    return out
+
+
+def dwthaar1d_f64(x: np.ndarray) -> np.ndarray:
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    y = np.empty(x.size, np.float64)
+    lib().orc_dwthaar1d_f64(_p(x), x.size, _p(y))
+    return y
+
+
+def dwthaar1d_f32dag(x: np.ndarray) -> np.ndarray:
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    y = np.empty(x.size, np.float32)
+    lib().orc_dwthaar1d_f32dag(_p(x), x.size, _p(y))
+    return y
+
+
+BO_STEPS, BO_R, BO_V = 254, 0.02, 0.30
+
+
+def crr_price(S, K, T, R, V, N, call=True) -> float:
+    return lib().orc_crr_price(float(S), float(K), float(T), float(R), float(V), int(N), 1 if call else 0)
+
+
+def bo_params(r: float):
+    S, K, T = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+    lib().orc_bo_params(float(r), ctypes.byref(S), ctypes.byref(K), ctypes.byref(T))
+    return S.value, K.value, T.value
+
+
+def binomialoption(r: np.ndarray) -> np.ndarray:
+    r = np.ascontiguousarray(r, dtype=np.float32)
+    call = np.empty(r.size, np.float64)
+    lib().orc_binomialoption(_p(r), r.size, _p(call))
+    return call

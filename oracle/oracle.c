@@ -333,3 +333,115 @@ void orc_matmul_bf16_sampled(const uint16_t* A, const uint16_t* Bt, int64_t K, i
         absout[s] = aacc;
     }
 }
+
+/* ======================================================================== */
+/* the paper's communication-stress kernels              */
+/* ======================================================================== */
+
+/* ------------------------------------------------------------------------ */
+/* BitonicSort (P:157 / Fig.2 "BitS"; memory-bound P:567, Inter 9.48x P:695, */
+/* P:807; reading R-BIT1: ascending u32 keys, N a power of two).  A sorting  */
+/* network's result is the sorted sequence, which is unique for keys, so the */
+/* oracle is that definition: a library sort of a copy.                      */
+/* ------------------------------------------------------------------------ */
+static int orc_cmp_u32(const void* a, const void* b) {
+    uint32_t x = *(const uint32_t*)a, y = *(const uint32_t*)b;
+    return (x > y) - (x < y);
+}
+void orc_sort_u32(const uint32_t* keys, int64_t n, uint32_t* out) {
+    memcpy(out, keys, (size_t)n * sizeof(uint32_t));
+    qsort(out, (size_t)n, sizeof(uint32_t), orc_cmp_u32);
+}
+
+/* ------------------------------------------------------------------------ */
+/* DwtHaar1D (P:157 / Fig.2 "DWT"; memory-bound yet communication-heavy,     */
+/* P:571-575).  Readings R-DWT1/2: full orthonormal Haar decomposition of N = */
+/* 2^L samples, level by level: a_i = (c_{2i} + c_{2i+1}) / sqrt2,            */
+/* d_i = (c_{2i} - c_{2i+1}) / sqrt2 of the previous level's approximation c. */
+/* Layout: y[0] = final approximation a_L, y[2^(L-k) .. 2^(L-k+1)) = level-k */
+/* details (k = 1 finest: y[N/2 .. N)).                                      */
+/* ------------------------------------------------------------------------ */
+void orc_dwthaar1d_f64(const float* x, int64_t N, double* y) {
+    double* c = (double*)malloc((size_t)N * sizeof(double));
+    for (int64_t i = 0; i < N; ++i) c[i] = (double)x[i];
+    for (int64_t len = N; len > 1; len >>= 1) {
+        int64_t half = len >> 1;
+        for (int64_t i = 0; i < half; ++i) {
+            double a = (c[2 * i] + c[2 * i + 1]) * M_SQRT1_2;
+            double d = (c[2 * i] - c[2 * i + 1]) * M_SQRT1_2;
+            y[half + i] = d;
+            c[i] = a; /* i < 2i: the in-place overwrite reads nothing later needed */
+        }
+    }
+    if (N >= 1) y[0] = c[0];
+    free(c);
+}
+
+/* Same DAG in fp32 (R-DWT2: per level a = RN(RN(c0 + c1) * s), d = RN(RN(c0 -
+ * c1) * s), s = RN32(1/sqrt2); the level order fixes every rounding, so the GPU
+ * is checked bit for bit against this). */
+void orc_dwthaar1d_f32dag(const float* x, int64_t N, float* y) {
+    float* c = (float*)malloc((size_t)N * sizeof(float));
+    const float s = (float)M_SQRT1_2;
+    memcpy(c, x, (size_t)N * sizeof(float));
+    for (int64_t len = N; len > 1; len >>= 1) {
+        int64_t half = len >> 1;
+        for (int64_t i = 0; i < half; ++i) {
+            volatile float sum = c[2 * i] + c[2 * i + 1];
+            volatile float dif = c[2 * i] - c[2 * i + 1];
+            volatile float a = sum * s;
+            volatile float d = dif * s;
+            y[half + i] = d;
+            c[i] = a;
+        }
+    }
+    if (N >= 1) y[0] = c[0];
+    free(c);
+}
+
+/* ------------------------------------------------------------------------ */
+/* BinomialOption (P:157 / Fig.2 "BO"; LDS-bound, -LDS trades compute for    */
+/* communication P:575; FAST swizzle beneficiary P:853).  Readings R-BO1/2:   */
+/* European call on a Cox-Ross-Rubinstein lattice of NSTEPS = 254 steps,     */
+/* R = 0.02, sigma = 0.30; one U[0,1) draw r per option mapped to            */
+/* S = 5(1-r) + 30r, K = (1-r) + 100r, T = 0.25(1-r) + 10r [APP-SDK?].        */
+/* dt = T/N, u = e^{sigma sqrt dt}, d = 1/u, p = (e^{R dt} - d)/(u - d);      */
+/* leaves V_i = max(S u^{2i-N} - K, 0), i = 0..N; N backward steps           */
+/* V_i <- e^{-R dt} (p V_{i+1} + (1-p) V_i); the price is V_0.               */
+/* ------------------------------------------------------------------------ */
+#define ORC_BO_STEPS 254
+#define ORC_BO_R 0.02
+#define ORC_BO_V 0.30
+
+double orc_crr_price(double S, double K, double T, double R, double V, int64_t N, int call) {
+    double dt = T / (double)N;
+    double u = exp(V * sqrt(dt)), d = 1.0 / u;
+    double p = (exp(R * dt) - d) / (u - d);
+    double disc = exp(-R * dt);
+    double* v = (double*)malloc((size_t)(N + 1) * sizeof(double));
+    for (int64_t i = 0; i <= N; ++i) {
+        double price = S * pow(u, (double)(2 * i - N));
+        double pay = call ? price - K : K - price;
+        v[i] = pay > 0.0 ? pay : 0.0;
+    }
+    for (int64_t j = N; j > 0; --j)
+        for (int64_t i = 0; i < j; ++i) v[i] = disc * (p * v[i + 1] + (1.0 - p) * v[i]);
+    double out = v[0];
+    free(v);
+    return out;
+}
+
+void orc_bo_params(double r, double* S, double* K, double* T) {
+    *S = 5.0 * (1.0 - r) + 30.0 * r;
+    *K = 1.0 * (1.0 - r) + 100.0 * r;
+    *T = 0.25 * (1.0 - r) + 10.0 * r;
+}
+
+void orc_binomialoption(const float* r, int64_t n, double* call) {
+#pragma omp parallel for schedule(dynamic, 64)
+    for (int64_t i = 0; i < n; ++i) {
+        double S, K, T;
+        orc_bo_params((double)r[i], &S, &K, &T);
+        call[i] = orc_crr_price(S, K, T, ORC_BO_R, ORC_BO_V, ORC_BO_STEPS, 1);
+    }
+}

@@ -152,3 +152,23 @@ def matmul_bf16_int(seed: int, rows: int, cols: int, stream: int, lo: int = -4, 
     n = rows * cols
     v = (u32(seed, n, row_offset * cols, stream=stream) % np.uint32(hi - lo + 1)).astype(np.int64) + lo
     return f32_to_bf16_bits(v.astype(np.float32)).reshape(rows, cols)
+
+
+# ---- SURVEY 8(f) rank 2 kernels ----
+
+def bitonic_keys(seed: int, n: int, offset: int = 0, bits: int = 32) -> np.ndarray:
+    """u32 keys, uniform over [0, 2^bits) (bits < 32: duplicate-heavy)."""
+    k = u32(seed, n, offset, stream=10)
+    if bits < 32:
+        k &= np.uint32((1 << bits) - 1)
+    return k
+
+
+def dwt_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """f32 U[-1,1) signal (exact: 2*k*2^-24 - 1)."""
+    return (uniform_f32(seed, n, offset, stream=11) * np.float32(2.0) - np.float32(1.0)).astype(np.float32)
+
+
+def binomial_r(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """One U[0,1) draw per option (APP-SDK style; the kernel maps r -> S, K, T)."""
+    return uniform_f32(seed, n, offset, stream=12)

@@ -361,3 +361,148 @@ def test_bf16_rounding_is_rne():
     assert back[0] == 1.0 and back[1] == 1.0  # tie -> even
     assert back[2] == 1.0 + 2**-7  # above half -> up
     assert back[3] == -2.5
+
+
+# ---------------------------------------------------------------- BitonicSort (R-BIT1)
+
+
+def test_sort_vs_library_and_invariants():
+    for bits in (32, 8, 1):
+        k = inputs.bitonic_keys(21, 1 << 14, bits=bits)
+        s = oracle.sort_u32(k)
+        assert np.array_equal(s, np.sort(k))                      # library routine
+        assert np.all(s[1:] >= s[:-1])                            # sorted
+        assert np.array_equal(np.unique(s, return_counts=True)[1],  # same multiset
+                              np.unique(k, return_counts=True)[1])
+    assert np.array_equal(oracle.sort_u32(np.arange(1024, dtype=np.uint32)[::-1].copy()),
+                          np.arange(1024, dtype=np.uint32))
+    assert np.array_equal(oracle.sort_u32(np.array([7], np.uint32)), np.array([7], np.uint32))
+    assert np.array_equal(oracle.sort_u32(np.full(64, 0xFFFFFFFF, np.uint32)), np.full(64, 0xFFFFFFFF, np.uint32))
+
+
+def test_sort_brute_force_permutations():
+    base = [0, 1, 1, 2, 3, 5, 8, 0xFFFFFFFF]
+    for perm in itertools.islice(itertools.permutations(base), 0, 40320, 17):
+        assert list(oracle.sort_u32(np.array(perm, np.uint32))) == sorted(base)
+
+
+# ---------------------------------------------------------------- DwtHaar1D (R-DWT1/2)
+
+
+def _haar_basis(N):
+    """Rows = the orthonormal Haar functions in the R-DWT1 output layout."""
+    L = N.bit_length() - 1
+    H = np.zeros((N, N))
+    H[0, :] = 2.0 ** (-L / 2)
+    for k in range(1, L + 1):
+        w = 1 << k
+        for j in range(N >> k):
+            row = (N >> k) + j
+            H[row, j * w: j * w + w // 2] = 2.0 ** (-k / 2)
+            H[row, j * w + w // 2: (j + 1) * w] = -(2.0 ** (-k / 2))
+    return H
+
+
+def test_dwt_haar_basis_closed_form():
+    for N in (1, 2, 4, 8, 64, 256):
+        x = inputs.dwt_x(3, N)
+        y = oracle.dwthaar1d_f64(x)
+        assert np.allclose(y, _haar_basis(N) @ x.astype(np.float64), rtol=0, atol=1e-12), N
+
+
+def test_dwt_parseval_constant_and_inverse():
+    N = 1 << 12
+    x = inputs.dwt_x(4, N)
+    y = oracle.dwthaar1d_f64(x)
+    assert abs(np.dot(y, y) - np.dot(x.astype(np.float64), x)) < 1e-9 * np.dot(x.astype(np.float64), x)
+    c = oracle.dwthaar1d_f64(np.full(N, 0.5, np.float32))
+    assert abs(c[0] - 0.5 * math.sqrt(N)) < 1e-12 and np.all(np.abs(c[1:]) < 1e-12)
+    # inverse, written independently: coarse to fine, c_{2i} = (a+d)/sqrt2, c_{2i+1} = (a-d)/sqrt2
+    a = y[:1].copy()
+    n = 1
+    while n < N:
+        d = y[n:2 * n]
+        nxt = np.empty(2 * n)
+        nxt[0::2] = (a + d) / math.sqrt(2.0)
+        nxt[1::2] = (a - d) / math.sqrt(2.0)
+        a, n = nxt, 2 * n
+    assert np.allclose(a, x.astype(np.float64), rtol=0, atol=1e-12)
+
+
+def test_dwt_f32dag_within_rounding_bound():
+    N = 1 << 14
+    x = inputs.dwt_x(5, N)
+    y64 = oracle.dwthaar1d_f64(x)
+    y32 = oracle.dwthaar1d_f32dag(x).astype(np.float64)
+    # every coefficient is a signed sum over its support scaled by 2^{-k/2}; each
+    # level adds <= 2 roundings: |err| <= 2 L u * (same transform of |x| with + only)
+    L = N.bit_length() - 1
+    absb = oracle.dwthaar1d_f64(np.abs(x))  # a-path of |x| bounds |a|; details bounded by the same a
+    bound = np.empty(N)
+    bound[0] = absb[0]
+    for k in range(1, L + 1):
+        lo, hi = N >> k, N >> (k - 1)
+        # level-k |coefficient| <= 2^{-k/2} * sum |x| over 2^k samples = level-k a of |x|
+        ax = np.abs(x.astype(np.float64)).reshape(-1, 1 << k).sum(axis=1) * 2.0 ** (-k / 2)
+        bound[lo:hi] = ax
+    assert np.all(np.abs(y32 - y64) <= 2 * L * 2.0 ** -24 * bound + 1e-30)
+
+
+# ---------------------------------------------------------------- BinomialOption (R-BO1/2)
+
+
+def _crr_closed_form(S, K, T, R, V, N, call=True):
+    """Independent form: discounted binomial expectation of the payoff."""
+    dt = T / N
+    u = math.exp(V * math.sqrt(dt))
+    d = 1 / u
+    p = (math.exp(R * dt) - d) / (u - d)
+    tot = 0.0
+    for k in range(N + 1):
+        ST = S * u ** (2 * k - N)
+        pay = max(ST - K, 0.0) if call else max(K - ST, 0.0)
+        if pay > 0:
+            lw = (math.lgamma(N + 1) - math.lgamma(k + 1) - math.lgamma(N - k + 1)
+                  + k * math.log(p) + (N - k) * math.log1p(-p))
+            tot += math.exp(lw) * pay
+    return math.exp(-R * T) * tot
+
+
+def test_bo_lattice_vs_closed_form_sum():
+    for r in (0.0, 0.13, 0.5, 0.77, 1.0):
+        S, K, T = oracle.bo_params(r)
+        for call in (True, False):
+            a = oracle.crr_price(S, K, T, oracle.BO_R, oracle.BO_V, oracle.BO_STEPS, call)
+            b = _crr_closed_form(S, K, T, oracle.BO_R, oracle.BO_V, oracle.BO_STEPS, call)
+            assert abs(a - b) <= 1e-9 * max(1.0, abs(b)), (r, call, a, b)
+    # N = 1 by hand
+    S, K, T, R, V = 20.0, 21.0, 1.0, 0.05, 0.3
+    u = math.exp(V); d = 1 / u; p = (math.exp(R) - d) / (u - d)
+    hand = math.exp(-R) * (p * max(S * u - K, 0) + (1 - p) * max(S * d - K, 0))
+    assert abs(oracle.crr_price(S, K, T, R, V, 1, True) - hand) < 1e-12
+
+
+def test_bo_put_call_parity_bounds_and_bs_limit():
+    for r in np.linspace(0, 1, 11):
+        S, K, T = oracle.bo_params(r)
+        C = oracle.crr_price(S, K, T, oracle.BO_R, oracle.BO_V, oracle.BO_STEPS, True)
+        P = oracle.crr_price(S, K, T, oracle.BO_R, oracle.BO_V, oracle.BO_STEPS, False)
+        disc = K * math.exp(-oracle.BO_R * T)
+        assert abs((C - P) - (S - disc)) < 1e-9 * S          # exact on the lattice
+        assert max(0.0, S - disc) - 1e-12 <= C <= S
+        bs_c, _ = oracle.bs_price(S, K, T, oracle.BO_R, oracle.BO_V)
+        assert abs(C - bs_c) < 5e-3 * S                       # CRR -> Black-Scholes, O(1/N)
+    # the error shrinks with N (first-order convergence, at-the-money)
+    e1 = abs(oracle.crr_price(100, 100, 1, 0.05, 0.2, 64, True) - 10.450575619322287)
+    e2 = abs(oracle.crr_price(100, 100, 1, 0.05, 0.2, 1024, True) - 10.450575619322287)
+    assert e2 < e1 / 4
+
+
+def test_bo_workload_mapping():
+    assert oracle.bo_params(0.0) == (5.0, 1.0, 0.25)
+    assert oracle.bo_params(1.0) == (30.0, 100.0, 10.0)
+    r = inputs.binomial_r(7, 64)
+    v = oracle.binomialoption(r)
+    for i in (0, 17, 63):
+        S, K, T = oracle.bo_params(float(r[i]))
+        assert v[i] == oracle.crr_price(S, K, T, oracle.BO_R, oracle.BO_V, oracle.BO_STEPS, True)
