@@ -162,6 +162,15 @@ def oracle_sample_rate(jobs, min_seconds=1.0):
         elif j.kernel == "blackscholes":
             r = j.host_in[0][: 1 << 22]
             fn, units, what = (lambda: oracle.blackscholes(r)), r.size, f"n={r.size}"
+        elif j.kernel == "dwthaar1d":
+            x = j.host_in[0][: 1 << 22]
+            fn, units, what = (lambda: oracle.dwthaar1d_f64(x)), x.size, "N=2^22"
+        elif j.kernel == "bitonicsort":
+            k = j.host_in[0][: 1 << 22]
+            fn, units, what = (lambda: oracle.sort_u32(k)), k.size, "N=2^22"
+        elif j.kernel == "binomialoption":
+            r = j.host_in[0][: 1 << 12]
+            fn, units, what = (lambda: oracle.binomialoption(r)), r.size, "n=2^12"
         else:
             continue
         reps, t0 = 0, time.perf_counter()

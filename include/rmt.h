@@ -73,7 +73,8 @@ typedef enum {
 } rmt_variant_t;
 
 /* The AMD APP SDK-style kernels the paper evaluates (Fig. 2 axis
- * P:237-255) plus MatrixTranspose (BASELINE.json configs[1]). */
+ * P:237-255) plus MatrixTranspose (BASELINE.json configs[1]); ids >= 10 are
+ * the paper's communication-stress kernels. */
 typedef enum {
     RMT_K_BLACKSCHOLES = 0,
     RMT_K_BINARYSEARCH = 1,
@@ -85,7 +86,8 @@ typedef enum {
     RMT_K_FLOYDWARSHALL = 7,
     RMT_K_DCT = 8,
     RMT_K_MATMUL = 9,
-    RMT_K_COUNT = 10
+    RMT_K_DWTHAAR1D = 10,
+    RMT_K_COUNT = 11
 } rmt_kernel_t;
 
 typedef enum { RMT_F32 = 0, RMT_U32 = 1, RMT_U64 = 2, RMT_U8X4 = 3, RMT_BF16 = 4 } rmt_dtype_t;
@@ -113,6 +115,9 @@ typedef struct {
  *   DCT           buf {X:F32[H*W], Y:F32[H*W]}                      n = H*W, dims {H, W}, H%8 = W%8 = 0
  *   MATMUL        buf {A:BF16[M*K], Bt:BF16[N*K], C:F32[M*N]}       n = M*N, dims {M, N, K}
  *                 C = A * Bt^T (both operands K-major); M%128 = N%256 = 0, K%64 = 0
+ *   DWTHAAR1D     buf {x:F32[N], y:F32[N]}                          n = N = 2^L <= 2^30
+ *                 full orthonormal Haar decomposition: y[0] = a_L, y[N>>k + i] = level-k
+ *                 detail i (DESIGN.md R-DWT1/2)
  * Vector-committed buffers must have < 2^30 elements.
  */
 typedef struct {

@@ -97,6 +97,7 @@ RMT_DECLARE_KERNEL(sobel)
 RMT_DECLARE_KERNEL(floydwarshall)
 RMT_DECLARE_KERNEL(dct)
 RMT_DECLARE_KERNEL(matmul)
+RMT_DECLARE_KERNEL(dwthaar1d)
 
 }  // namespace rmt
 

@@ -133,6 +133,11 @@ def job_floydwarshall(n, seed=8):
                note="per pass: 4 B/elem read of D (L2-resident) + conditional writes; n passes + init")
 
 
+def job_dwthaar1d(N, seed=11, rank=0):
+    return Job("dwthaar1d", N, (), [inputs.dwt_x(seed, N, rank * N), None], [(1, 4 * N)],
+               alg_bytes=8 * N, unit="samples", note="read x once, write y once (+N/256 B of approximations)")
+
+
 # ---------------------------------------------------------------- BASELINE.json configs
 
 def config_jobs(name: str, rank: int = 0):
@@ -154,6 +159,8 @@ def config_jobs(name: str, rank: int = 0):
         return [job_matmul(8192, 8192, 8192, rank=rank)]
     if name == "fwdct":      # configs[3]
         return [job_floydwarshall(4096), job_dct(8192, 8192, rank=rank)]
+    if name == "comm":       # the paper's communication-stress kernels
+        return [job_dwthaar1d(1 << 26, rank=rank)]
     if name == "small":      # smoke-sized
         return [job_binarysearch(1 << 16, 1 << 14, rank=rank), job_fwt(1 << 14, rank=rank),
                 job_prefixsum(1 << 16, rank=rank), job_reduction(1 << 16, rank=rank),
@@ -171,4 +178,5 @@ CONFIG_TITLES = {
     "mm16k": "MatrixMultiplication 16384^3 bf16 -> fp32 (tcgen05)",
     "mm8k": "MatrixMultiplication 8192^3 bf16 -> fp32 (tcgen05)",
     "fwdct": "FloydWarshall 4096 nodes + DCT 8192^2",
+    "comm": "communication-stress kernels (SURVEY 8(f) rank 2): DwtHaar1D 2^26",
 }

@@ -400,6 +400,37 @@ class MatMul(Case):
         return 2, self.n
 
 
+class DWT(Case):
+    kernel = "dwthaar1d"
+
+    def __init__(self, n, seed=11):
+        self.n = n
+        self.x = inputs.dwt_x(seed, n)
+
+    @functools.cached_property
+    def x_d(self):
+        return dev(self.x)
+
+    def buffers(self):
+        return [self.x_d, out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32)]
+
+    def check(self, outs, x=None):
+        x = self.x if x is None else x
+        # R-DWT2: bit-exact vs the fp32 DAG in level order
+        assert np.array_equal(outs[0], oracle.dwthaar1d_f32dag(x).view(np.uint32))
+        # and within 1e-5 of the fp64 definition, scaled by the coefficient's support norm
+        y64 = oracle.dwthaar1d_f64(x)
+        got = outs[0].view(np.float32).astype(np.float64)
+        scale = max(1.0, float(np.sqrt(np.dot(x.astype(np.float64), x))))
+        assert np.max(np.abs(got - y64)) <= 1e-5 * scale
+
+    def out_elems(self):
+        return 1, self.n
+
+
 def small_cases():
     """Sizes the oracle finishes in seconds that still span several tiles and a ragged tail."""
     return [
@@ -414,4 +445,5 @@ def small_cases():
         DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8),
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
         MatMul(128, 256, 64), MatMul(256, 512, 192, integer=True), MatMul(384, 256, 1024),
+        DWT(1), DWT(2), DWT(4), DWT(8), DWT(64), DWT(4096), DWT(8192), DWT(1 << 20), DWT(1 << 23),
     ]
