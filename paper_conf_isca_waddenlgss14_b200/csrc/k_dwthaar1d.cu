@@ -125,9 +125,12 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dwt_kernel(DwtArgs a, Ctx c
       }
     }
     __syncthreads();  // every read of this level precedes the first write-back
+    // a warp none of whose logical threads has a group this level skips the
+    // commit: the decision is the same in both replicas (a function of ltid, k)
+    const int lw0 = rep.ltid - rep.llane;  // first logical thread of this warp
 #pragma unroll
     for (int u = 0; u < 2; ++u) {
-      if (u < nu) {
+      if (u < nu && lw0 + u * BL < ng) {
         const int g = rep.ltid + u * BL;
         const bool act = g < ng;
         if (act) {
@@ -141,7 +144,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dwt_kernel(DwtArgs a, Ctx c
         const unsigned idx = (a.M >> k) + tile * (unsigned)half + 4u * (unsigned)g;
         rep.template commit<4, 0>(act ? 0xFu : 0u, act ? idx : 0u, dw, a.M,
                                   [&](unsigned i, unsigned m, const unsigned* w) { st_y(a.y, i, m, w); },
-                                  /*defer=*/u + 1 < nu);
+                                  /*defer=*/u + 1 < nu && lw0 + (u + 1) * BL < ng);
       }
     }
     __syncthreads();
