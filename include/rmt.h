@@ -87,7 +87,8 @@ typedef enum {
     RMT_K_DCT = 8,
     RMT_K_MATMUL = 9,
     RMT_K_DWTHAAR1D = 10,
-    RMT_K_COUNT = 11
+    RMT_K_BITONICSORT = 11,
+    RMT_K_COUNT = 12
 } rmt_kernel_t;
 
 typedef enum { RMT_F32 = 0, RMT_U32 = 1, RMT_U64 = 2, RMT_U8X4 = 3, RMT_BF16 = 4 } rmt_dtype_t;
@@ -118,6 +119,8 @@ typedef struct {
  *   DWTHAAR1D     buf {x:F32[N], y:F32[N]}                          n = N = 2^L <= 2^30
  *                 full orthonormal Haar decomposition: y[0] = a_L, y[N>>k + i] = level-k
  *                 detail i (DESIGN.md R-DWT1/2)
+ *   BITONICSORT   buf {keys:U32[N], sorted:U32[N]}                  n = N = 2^n <= 2^30, ascending
+ *                 (DESIGN.md R-BIT1)
  * Vector-committed buffers must have < 2^30 elements.
  */
 typedef struct {

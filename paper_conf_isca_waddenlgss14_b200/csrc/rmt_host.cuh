@@ -98,6 +98,7 @@ RMT_DECLARE_KERNEL(floydwarshall)
 RMT_DECLARE_KERNEL(dct)
 RMT_DECLARE_KERNEL(matmul)
 RMT_DECLARE_KERNEL(dwthaar1d)
+RMT_DECLARE_KERNEL(bitonicsort)
 
 }  // namespace rmt
 

@@ -138,6 +138,18 @@ def job_dwthaar1d(N, seed=11, rank=0):
                alg_bytes=8 * N, unit="samples", note="read x once, write y once (+N/256 B of approximations)")
 
 
+def bitonic_launches(N):
+    n = max(0, N.bit_length() - 1)
+    return 1 + sum(-(-(s - 11) // 7) + 1 for s in range(12, n))
+
+
+def job_bitonicsort(N, seed=21, rank=0):
+    L = bitonic_launches(N)
+    return Job("bitonicsort", N, (), [inputs.bitonic_keys(seed, N, rank * N), None], [(1, 4 * N)],
+               alg_bytes=8 * N * L, unit="keys", note=f"{L} tile launches x 8 B/key (bitonic network, "
+                                                      f"{(N.bit_length() - 1) * N.bit_length() // 2} passes)")
+
+
 # ---------------------------------------------------------------- BASELINE.json configs
 
 def config_jobs(name: str, rank: int = 0):
@@ -160,7 +172,7 @@ def config_jobs(name: str, rank: int = 0):
     if name == "fwdct":      # configs[3]
         return [job_floydwarshall(4096), job_dct(8192, 8192, rank=rank)]
     if name == "comm":       # the paper's communication-stress kernels
-        return [job_dwthaar1d(1 << 26, rank=rank)]
+        return [job_dwthaar1d(1 << 26, rank=rank), job_bitonicsort(1 << 26, rank=rank)]
     if name == "small":      # smoke-sized
         return [job_binarysearch(1 << 16, 1 << 14, rank=rank), job_fwt(1 << 14, rank=rank),
                 job_prefixsum(1 << 16, rank=rank), job_reduction(1 << 16, rank=rank),
@@ -178,5 +190,5 @@ CONFIG_TITLES = {
     "mm16k": "MatrixMultiplication 16384^3 bf16 -> fp32 (tcgen05)",
     "mm8k": "MatrixMultiplication 8192^3 bf16 -> fp32 (tcgen05)",
     "fwdct": "FloydWarshall 4096 nodes + DCT 8192^2",
-    "comm": "communication-stress kernels (SURVEY 8(f) rank 2): DwtHaar1D 2^26",
+    "comm": "communication-stress kernels (SURVEY 8(f) rank 2): DwtHaar1D 2^26, BitonicSort 2^26",
 }

@@ -431,6 +431,32 @@ class DWT(Case):
         return 1, self.n
 
 
+class BitonicSort(Case):
+    kernel = "bitonicsort"
+
+    def __init__(self, n, seed=21, bits=32):
+        self.n = n
+        self.multipass = n > 4096
+        self.keys = inputs.bitonic_keys(seed, n, bits=bits)
+
+    @functools.cached_property
+    def k_d(self):
+        return dev(self.keys)
+
+    def buffers(self):
+        return [self.k_d, out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32)]
+
+    def check(self, outs, keys=None):
+        keys = self.keys if keys is None else keys
+        assert np.array_equal(outs[0], oracle.sort_u32(keys))  # R-BIT1: the unique sorted sequence
+
+    def out_elems(self):
+        return 1, self.n
+
+
 def small_cases():
     """Sizes the oracle finishes in seconds that still span several tiles and a ragged tail."""
     return [
@@ -446,4 +472,6 @@ def small_cases():
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
         MatMul(128, 256, 64), MatMul(256, 512, 192, integer=True), MatMul(384, 256, 1024),
         DWT(1), DWT(2), DWT(4), DWT(8), DWT(64), DWT(4096), DWT(8192), DWT(1 << 20), DWT(1 << 23),
+        BitonicSort(1), BitonicSort(2), BitonicSort(8), BitonicSort(16), BitonicSort(64, bits=3),
+        BitonicSort(4096), BitonicSort(8192, bits=8), BitonicSort(1 << 17), BitonicSort(1 << 20, bits=12),
     ]

@@ -14,7 +14,7 @@ import numpy as np
 import pytest
 
 from paper_conf_isca_waddenlgss14_b200 import rmt
-from cases import (DCT, DWT, FWT, BinarySearch, BlackScholes, FloydWarshall, MatMul, PrefixSum, Reduction, Sobel,
+from cases import (DCT, DWT, FWT, BitonicSort, BinarySearch, BlackScholes, FloydWarshall, MatMul, PrefixSum, Reduction, Sobel,
                    Transpose)
 from helpers import run
 
@@ -43,6 +43,8 @@ CAMPAIGN = [
                                  "store_val": lambda c: c.n ** 3, "store_addr": lambda c: c.n ** 3}),
     (lambda: MatMul(256, 256, 128), {"compute": lambda c: c.n, "store_val": lambda c: c.n,
                                      "store_addr": lambda c: c.n}),
+    (lambda: BitonicSort(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n, "smem": lambda c: c.n,
+                                    "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
     (lambda: DWT(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n // 2, "smem": lambda c: c.n // 2,
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
 ]
