@@ -12,9 +12,10 @@
 // Schedule: one contiguous launch sorts every tile (stages 0..11, 78 passes);
 // then per stage s >= 12, strided launches cover pass bits s..12 (<= 7 per
 // launch) and one contiguous launch the passes 11..0.  Inside a launch, passes
-// run as register rounds: each thread takes the 16 keys that differ only in 4
-// tile bits and applies every consecutive pass on those bits (up to 10) before
-// writing back -- one LDS + one STS per key per round, min/max per pair.
+// run as register rounds: each thread takes the 16 keys that differ only in a
+// window of 4 consecutive tile bits [q, q+4) and applies every consecutive
+// pass on those bits (up to 10) before writing back -- one LDS + one STS per
+// key per round (compile-time window: immediate smem offsets), min/max per pair.
 // HBM: 8 B/key per launch.  The result is the unique sorted sequence, so every
 // variant is bitwise equal to `none` and to the oracle.
 #include "rmt_host.cuh"
@@ -32,8 +33,10 @@ constexpr int MAXR = 40, MAXP = 96;
 __device__ __forceinline__ int phys(int e) { return e + (e >> 5); }
 
 struct BitRound {
-  unsigned char bits[4];  // tile bits of the 16-key group, ascending
+  unsigned char q;          // the round's tile bits are [q, q+4)
   unsigned char np, first;  // passes [first, first + np) of `ops`
+  unsigned char run;        // 1: passes are local bits l0, l0-1, .. of ONE stage with a uniform direction
+  unsigned char l0, g;      // run: first local bit, direction bit (global)
 };
 struct BitArgs {
   const unsigned* src;
@@ -72,6 +75,22 @@ __device__ __forceinline__ void cmpx(unsigned (&v)[16], bool asc) {
   }
 }
 
+// Ascending compare-exchange on local bits L0, L0-1, ..., L0-NP+1.
+template <int L0, int NP>
+__device__ __forceinline__ void cmpx_run(unsigned (&v)[16]) {
+#pragma unroll
+  for (int i = 0; i < NP; ++i) {
+    const int L = L0 - i;
+#pragma unroll
+    for (int k = 0; k < 16; ++k) {
+      if (k & (1 << L)) continue;
+      const unsigned x = v[k], y = v[k | (1 << L)];
+      v[k] = min(x, y);
+      v[k | (1 << L)] = max(x, y);
+    }
+  }
+}
+
 template <int L>
 __device__ __forceinline__ void cmpx_l(unsigned (&v)[16], int ld, bool asc) {
   switch (ld) {
@@ -80,6 +99,81 @@ __device__ __forceinline__ void cmpx_l(unsigned (&v)[16], int ld, bool asc) {
     case 2: if constexpr (L != 2) cmpx<L, 2>(v, asc); break;
     case 3: if constexpr (L != 3) cmpx<L, 3>(v, asc); break;
     default: cmpx<L, -1>(v, asc); break;
+  }
+}
+
+// phys(ebase | k << Q-window) - phys(ebase), for ebase with zeros in bits Q..Q+3
+template <int Q>
+__device__ __forceinline__ constexpr int coff(int k) {
+  return (k << Q) + ((Q >= 5) ? (k << (Q - 5)) : ((k << Q) >> 5));
+}
+
+// One round on the 4-bit window [Q, Q+4): thread = one 16-key group.
+template <int Q, class R_>
+__device__ __forceinline__ void bit_round(const R_& rep, const BitArgs& a, unsigned* tp, unsigned tile,
+                                          const BitRound& R, int ri) {
+  const int groups = (1 << a.tb) >> 4;
+  if (rep.ltid >= groups) return;
+  const unsigned gi = (unsigned)rep.ltid;
+  const unsigned ebase = (gi & ((1u << Q) - 1u)) | ((gi >> Q) << (Q + 4));
+  unsigned* pb = tp + phys((int)ebase);
+  unsigned v[16];
+#pragma unroll
+  for (int k = 0; k < 16; ++k) v[k] = pb[coff<Q>(k)];
+  if constexpr (R_::FAULT) {
+    if (a.first && ri == 1) {
+#pragma unroll
+      for (int k = 0; k < 16; ++k) v[k] = rep.fault(SITE_SMEM, (long long)gidx(a, tile, ebase | (k << Q)), v[k]);
+    }
+  }
+  const unsigned gbase = gidx(a, tile, ebase);
+  if (R.run) {
+    // one stage, uniform direction: a descending pass sorts the complemented
+    // keys ascending, so flip once and run pure min/max
+    const unsigned flip = ((gbase >> R.g) & 1u) ? 0xFFFFFFFFu : 0u;
+#pragma unroll
+    for (int k = 0; k < 16; ++k) v[k] ^= flip;
+    switch (R.l0 * 4 + R.np - 1) {
+      case 0: cmpx_run<0, 1>(v); break;
+      case 4: cmpx_run<1, 1>(v); break;
+      case 5: cmpx_run<1, 2>(v); break;
+      case 8: cmpx_run<2, 1>(v); break;
+      case 9: cmpx_run<2, 2>(v); break;
+      case 10: cmpx_run<2, 3>(v); break;
+      case 12: cmpx_run<3, 1>(v); break;
+      case 13: cmpx_run<3, 2>(v); break;
+      case 14: cmpx_run<3, 3>(v); break;
+      default: cmpx_run<3, 4>(v); break;
+    }
+#pragma unroll
+    for (int k = 0; k < 16; ++k) v[k] ^= flip;
+  } else {
+    for (int pi = 0; pi < R.np; ++pi) {
+      const unsigned op = a.ops[R.first + pi];
+      const int l = op & 3, ld = (op >> 2) & 7, g = (op >> 5) & 31;
+      const bool asc = ((gbase >> g) & 1u) == 0u;
+      switch (l) {
+        case 0: cmpx_l<0>(v, ld, asc); break;
+        case 1: cmpx_l<1>(v, ld, asc); break;
+        case 2: cmpx_l<2>(v, ld, asc); break;
+        default: cmpx_l<3>(v, ld, asc); break;
+      }
+    }
+  }
+  if constexpr (R_::FAULT) {
+    if (a.first && ri == 0) {
+#pragma unroll
+      for (int k = 0; k < 16; ++k) v[k] = rep.fault(SITE_COMPUTE, (long long)gidx(a, tile, ebase | (k << Q)), v[k]);
+    }
+  }
+  // -LDS: the group's keys are compared as four 4-word records
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const unsigned w4[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
+    if (rep.template sts_ok<4>(w4, ebase + (unsigned)q)) {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) pb[coff<Q>(4 * q + k)] = v[4 * q + k];
+    }
   }
 }
 
@@ -133,62 +227,18 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bitonic_kernel(BitArgs a, C
   __syncthreads();
 
   // ---- register rounds
-  const int groups = te >> 4;
   for (int ri = 0; ri < a.nr; ++ri) {
     const BitRound R = a.r[ri];
-    if (rep.ltid < groups) {
-      // deposit the thread's group id into the tile bits outside the round
-      unsigned ebase = 0, gid = (unsigned)rep.ltid;
-      const unsigned inb = (1u << R.bits[0]) | (1u << R.bits[1]) | (1u << R.bits[2]) | (1u << R.bits[3]);
-      for (int t = 0; t < a.tb; ++t) {
-        if (inb & (1u << t)) continue;
-        ebase |= (gid & 1u) << t;
-        gid >>= 1;
-      }
-      auto elem = [&](int k) -> unsigned {  // tile index of group key k
-        return ebase | ((k & 1) << R.bits[0]) | (((k >> 1) & 1) << R.bits[1]) | (((k >> 2) & 1) << R.bits[2]) |
-               (((k >> 3) & 1) << R.bits[3]);
-      };
-      int off[16];
-      unsigned v[16];
-#pragma unroll
-      for (int k = 0; k < 16; ++k) {
-        off[k] = phys((int)elem(k));
-        v[k] = tp[off[k]];
-      }
-      if constexpr (M == M_FAULT) {
-        if (a.first && ri == 1) {
-#pragma unroll
-          for (int k = 0; k < 16; ++k) v[k] = rep.fault(SITE_SMEM, (long long)gidx(a, tile, elem(k)), v[k]);
-        }
-      }
-      const unsigned gbase = gidx(a, tile, ebase);
-      for (int pi = 0; pi < R.np; ++pi) {
-        const unsigned op = a.ops[R.first + pi];
-        const int l = op & 3, ld = (op >> 2) & 7, g = (op >> 5) & 31;
-        const bool asc = ((gbase >> g) & 1u) == 0u;
-        switch (l) {
-          case 0: cmpx_l<0>(v, ld, asc); break;
-          case 1: cmpx_l<1>(v, ld, asc); break;
-          case 2: cmpx_l<2>(v, ld, asc); break;
-          default: cmpx_l<3>(v, ld, asc); break;
-        }
-      }
-      if constexpr (M == M_FAULT) {
-        if (a.first && ri == 0) {
-#pragma unroll
-          for (int k = 0; k < 16; ++k) v[k] = rep.fault(SITE_COMPUTE, (long long)gidx(a, tile, elem(k)), v[k]);
-        }
-      }
-      // -LDS: the whole group's keys are compared as four 4-word records
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const unsigned w4[4] = {v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]};
-        if (rep.template sts_ok<4>(w4, ebase + (unsigned)q)) {
-#pragma unroll
-          for (int k = 0; k < 4; ++k) tp[off[4 * q + k]] = v[4 * q + k];
-        }
-      }
+    switch (R.q) {
+      case 0: bit_round<0>(rep, a, tp, tile, R, ri); break;
+      case 1: bit_round<1>(rep, a, tp, tile, R, ri); break;
+      case 2: bit_round<2>(rep, a, tp, tile, R, ri); break;
+      case 3: bit_round<3>(rep, a, tp, tile, R, ri); break;
+      case 4: bit_round<4>(rep, a, tp, tile, R, ri); break;
+      case 5: bit_round<5>(rep, a, tp, tile, R, ri); break;
+      case 6: bit_round<6>(rep, a, tp, tile, R, ri); break;
+      case 7: bit_round<7>(rep, a, tp, tile, R, ri); break;
+      default: bit_round<8>(rep, a, tp, tile, R, ri); break;
     }
     __syncthreads();
   }
@@ -235,43 +285,43 @@ int tile_bit(const BitArgs& a, int g) {
   return -1;
 }
 
-// Group consecutive passes into register rounds of <= 4 distinct tile bits.
+// Group consecutive passes into rounds on 4-bit windows [q, q+4): a round
+// starts at the next pass (tile bit t, window q = clamp(t - 3, 0, tb - 4)) and
+// takes every following pass whose bit stays inside the window.
 bool build_rounds(BitArgs& a, const Op* ops, int nops) {
   a.nr = 0;
   int np = 0, i = 0;
   while (i < nops) {
     if (a.nr >= MAXR) return false;
-    unsigned set = 0;
-    int cnt = 0, j = i;
+    const int t0 = tile_bit(a, ops[i].p);
+    int q = t0 - 3;
+    if (q > a.tb - 4) q = a.tb - 4;
+    if (q < 0) q = 0;
+    BitRound& R = a.r[a.nr++];
+    R.q = (unsigned char)q;
+    R.first = (unsigned char)np;
+    int j = i;
     while (j < nops) {
       const int t = tile_bit(a, ops[j].p);
-      if (!(set & (1u << t))) {
-        if (cnt == 4) break;
-        set |= 1u << t;
-        ++cnt;
-      }
+      if (t < q || t >= q + 4) break;
+      if (np >= MAXP) return false;
+      const int g = ops[j].s + 1;
+      const int tg = tile_bit(a, g);
+      const int ld = (tg >= q && tg < q + 4) ? tg - q : 4;
+      a.ops[np++] = (unsigned short)((t - q) | (ld << 2) | ((g & 31) << 5));
       ++j;
     }
-    for (int t = 0; cnt < 4 && t < a.tb; ++t)  // pad the group to 4 bits
-      if (!(set & (1u << t))) { set |= 1u << t; ++cnt; }
-    BitRound& R = a.r[a.nr++];
-    int q = 0;
-    for (int t = 0; t < a.tb; ++t)
-      if (set & (1u << t)) R.bits[q++] = (unsigned char)t;
-    R.first = (unsigned char)np;
     R.np = (unsigned char)(j - i);
-    for (int k = i; k < j; ++k) {
-      if (np >= MAXP) return false;
-      const int t = tile_bit(a, ops[k].p);
-      int l = 0;
-      while (R.bits[l] != t) ++l;
-      const int g = ops[k].s + 1;
-      const int tg = tile_bit(a, g);
-      int ld = 4;
-      for (int z = 0; z < 4; ++z)
-        if (tg >= 0 && R.bits[z] == tg) ld = z;
-      a.ops[np++] = (unsigned short)(l | (ld << 2) | ((g & 31) << 5));
+    // a run: one stage, uniform direction, local bits l0, l0-1, ...
+    bool run = R.np >= 1 && R.np <= 4;
+    const int l0 = a.ops[R.first] & 3;
+    for (int k = 0; run && k < R.np; ++k) {
+      const unsigned op = a.ops[R.first + k];
+      run = ((op >> 2) & 7) == 4 && (int)(op & 3) == l0 - k && ops[i + k].s == ops[i].s;
     }
+    R.run = run ? 1 : 0;
+    R.l0 = (unsigned char)l0;
+    R.g = (unsigned char)(ops[i].s + 1);
     i = j;
   }
   return true;
