@@ -88,7 +88,8 @@ typedef enum {
     RMT_K_MATMUL = 9,
     RMT_K_DWTHAAR1D = 10,
     RMT_K_BITONICSORT = 11,
-    RMT_K_COUNT = 12
+    RMT_K_BINOMIALOPTION = 12,
+    RMT_K_COUNT = 13
 } rmt_kernel_t;
 
 typedef enum { RMT_F32 = 0, RMT_U32 = 1, RMT_U64 = 2, RMT_U8X4 = 3, RMT_BF16 = 4 } rmt_dtype_t;
@@ -121,6 +122,9 @@ typedef struct {
  *                 detail i (DESIGN.md R-DWT1/2)
  *   BITONICSORT   buf {keys:U32[N], sorted:U32[N]}                  n = N = 2^n <= 2^30, ascending
  *                 (DESIGN.md R-BIT1)
+ *   BINOMIALOPTION buf {r:F32[n], call:F32[n]}                      n = options <= 2^28
+ *                 CRR European call, 254 steps, R = 0.02, sigma = 0.30, (S, K, T) from r
+ *                 (DESIGN.md R-BO1/2)
  * Vector-committed buffers must have < 2^30 elements.
  */
 typedef struct {

@@ -42,6 +42,7 @@ const KEntry kTable[RMT_K_COUNT] = {
     KE(matmul, 2, 0, 1, 1, 2, 0),
     KE(dwthaar1d, 1, 0, 0, 1, 1, 0),
     KE(bitonicsort, 1, 0, 0, 1, 1, 0),
+    KE(binomialoption, 1, 0, 0, 1, 1, 0),
 };
 
 const char* kVariantNames[6] = {"none", "intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds"};

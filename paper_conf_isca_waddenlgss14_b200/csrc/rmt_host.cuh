@@ -99,6 +99,7 @@ RMT_DECLARE_KERNEL(dct)
 RMT_DECLARE_KERNEL(matmul)
 RMT_DECLARE_KERNEL(dwthaar1d)
 RMT_DECLARE_KERNEL(bitonicsort)
+RMT_DECLARE_KERNEL(binomialoption)
 
 }  // namespace rmt
 

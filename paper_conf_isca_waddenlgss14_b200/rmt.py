@@ -18,7 +18,7 @@ LIB_PATH = os.path.join(_HERE, "librmt.so")
 KERNELS = {
     "blackscholes": 0, "binarysearch": 1, "fwt": 2, "prefixsum": 3, "reduction": 4,
     "transpose": 5, "sobel": 6, "floydwarshall": 7, "dct": 8, "matmul": 9,
-    "dwthaar1d": 10, "bitonicsort": 11,
+    "dwthaar1d": 10, "bitonicsort": 11, "binomialoption": 12,
 }
 VARIANTS = {"none": 0, "intra_smem": 1, "intra_reg": 2, "inter_group": 3, "inter_cluster": 4, "intra_nolds": 5}
 RMT_VARIANTS = ("intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds")
@@ -41,6 +41,7 @@ SCHEMA = {
     "matmul": (BF16, BF16, F32),
     "dwthaar1d": (F32, F32),
     "bitonicsort": (U32, U32),
+    "binomialoption": (F32, F32),
 }
 
 

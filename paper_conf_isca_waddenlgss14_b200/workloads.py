@@ -150,6 +150,12 @@ def job_bitonicsort(N, seed=21, rank=0):
                                                       f"{(N.bit_length() - 1) * N.bit_length() // 2} passes)")
 
 
+def job_binomialoption(n, seed=12, rank=0):
+    return Job("binomialoption", n, (), [inputs.binomial_r(seed, n, rank * n), None], [(1, 4 * n)],
+               alg_bytes=8 * n, unit="options", bound="alu",
+               note="254-step CRR lattice in registers: ~64.8k flop/option (2 flop/node/step); HBM 8 B/option")
+
+
 # ---------------------------------------------------------------- BASELINE.json configs
 
 def config_jobs(name: str, rank: int = 0):
@@ -172,7 +178,8 @@ def config_jobs(name: str, rank: int = 0):
     if name == "fwdct":      # configs[3]
         return [job_floydwarshall(4096), job_dct(8192, 8192, rank=rank)]
     if name == "comm":       # the paper's communication-stress kernels
-        return [job_dwthaar1d(1 << 26, rank=rank), job_bitonicsort(1 << 26, rank=rank)]
+        return [job_dwthaar1d(1 << 26, rank=rank), job_bitonicsort(1 << 26, rank=rank),
+                job_binomialoption(1 << 17, rank=rank)]
     if name == "small":      # smoke-sized
         return [job_binarysearch(1 << 16, 1 << 14, rank=rank), job_fwt(1 << 14, rank=rank),
                 job_prefixsum(1 << 16, rank=rank), job_reduction(1 << 16, rank=rank),
@@ -190,5 +197,6 @@ CONFIG_TITLES = {
     "mm16k": "MatrixMultiplication 16384^3 bf16 -> fp32 (tcgen05)",
     "mm8k": "MatrixMultiplication 8192^3 bf16 -> fp32 (tcgen05)",
     "fwdct": "FloydWarshall 4096 nodes + DCT 8192^2",
-    "comm": "communication-stress kernels (SURVEY 8(f) rank 2): DwtHaar1D 2^26, BitonicSort 2^26",
+    "comm": "communication-stress kernels (SURVEY 8(f) rank 2): DwtHaar1D 2^26, BitonicSort 2^26, "
+            "BinomialOption 2^17 options",
 }

@@ -457,6 +457,36 @@ class BitonicSort(Case):
         return 1, self.n
 
 
+class BinomialOption(Case):
+    kernel = "binomialoption"
+
+    def __init__(self, n, seed=12):
+        self.n = n
+        self.r = inputs.binomial_r(seed, n)
+
+    @functools.cached_property
+    def r_d(self):
+        return dev(self.r)
+
+    def buffers(self):
+        return [self.r_d, out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32)]
+
+    def check(self, outs, r=None):
+        r = self.r if r is None else r
+        ref = oracle.binomialoption(r)
+        S = 5.0 * (1 - r.astype(np.float64)) + 30.0 * r.astype(np.float64)
+        got = outs[0].view(np.float32).astype(np.float64)
+        # reading R-BO2: relative 1e-4 (transcendental + 254-step recurrence, as BlackScholes), floored at 1e-2*S
+        bad = ~(np.abs(got - ref) <= 1e-4 * np.maximum(np.abs(ref), 1e-2 * S))
+        assert not bad.any(), f"{bad.sum()} mismatches, first at {np.argmax(bad)}"
+
+    def out_elems(self):
+        return 1, self.n
+
+
 def small_cases():
     """Sizes the oracle finishes in seconds that still span several tiles and a ragged tail."""
     return [
@@ -474,4 +504,5 @@ def small_cases():
         DWT(1), DWT(2), DWT(4), DWT(8), DWT(64), DWT(4096), DWT(8192), DWT(1 << 20), DWT(1 << 23),
         BitonicSort(1), BitonicSort(2), BitonicSort(8), BitonicSort(16), BitonicSort(64, bits=3),
         BitonicSort(4096), BitonicSort(8192, bits=8), BitonicSort(1 << 17), BitonicSort(1 << 20, bits=12),
+        BinomialOption(1), BinomialOption(5), BinomialOption(100), BinomialOption(4096 + 3),
     ]

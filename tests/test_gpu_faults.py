@@ -14,7 +14,7 @@ import numpy as np
 import pytest
 
 from paper_conf_isca_waddenlgss14_b200 import rmt
-from cases import (DCT, DWT, FWT, BitonicSort, BinarySearch, BlackScholes, FloydWarshall, MatMul, PrefixSum, Reduction, Sobel,
+from cases import (DCT, DWT, FWT, BinomialOption, BitonicSort, BinarySearch, BlackScholes, FloydWarshall, MatMul, PrefixSum, Reduction, Sobel,
                    Transpose)
 from helpers import run
 
@@ -45,6 +45,8 @@ CAMPAIGN = [
                                      "store_addr": lambda c: c.n}),
     (lambda: BitonicSort(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n, "smem": lambda c: c.n,
                                     "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
+    (lambda: BinomialOption(2000), {"load": lambda c: c.n, "compute": lambda c: c.n, "store_val": lambda c: c.n,
+                                    "store_addr": lambda c: c.n}),
     (lambda: DWT(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n // 2, "smem": lambda c: c.n // 2,
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
 ]
