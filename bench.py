@@ -33,7 +33,41 @@ sys.path.insert(0, ROOT)
 METRIC = "RMT slowdown vs unprotected kernel per variant; baseline HBM GB/s vs peak"
 VARIANTS = ("none", "intra_smem", "intra_reg", "inter_group")
 # B200 extensions: measured after the timed step, not part of it
-EXTRA_VARIANTS = ("inter_cluster", "intra_nolds")
+EXTRA_VARIANTS = ("inter_cluster", "intra_nolds", "dup_kernel")
+
+
+# ---------------------------------------------------------------- energy (NVML; Fig. 5)
+def measure_energy(dev_index, launch, seconds=0.25):
+    """Back-to-back launches for >= `seconds`: average board power (W) from the
+    NVML total-energy counter (mJ) over the device time, and energy per launch."""
+    import torch
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+        pynvml.nvmlDeviceGetTotalEnergyConsumption(h)
+    except Exception:
+        return None
+    launch()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    launch()
+    torch.cuda.synchronize()
+    one = max(time.perf_counter() - t0, 1e-5)
+    reps = max(3, int(seconds / one))
+    e0 = pynvml.nvmlDeviceGetTotalEnergyConsumption(h)
+    a = torch.cuda.Event(enable_timing=True)
+    b = torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(reps):
+        launch()
+    b.record()
+    torch.cuda.synchronize()
+    e1 = pynvml.nvmlDeviceGetTotalEnergyConsumption(h)
+    secs = a.elapsed_time(b) * 1e-3
+    joules = (e1 - e0) * 1e-3
+    return {"avg_w": round(joules / secs, 1), "j_per_launch": round(joules / reps, 6), "launches": reps,
+            "ms_per_launch": round(1e3 * secs / reps, 4)}
 
 
 def parse():
@@ -48,6 +82,8 @@ def parse():
     p.add_argument("--variants", default=",".join(VARIANTS))
     p.add_argument("--extra-variants", default=",".join(EXTRA_VARIANTS),
                    help="variants timed per launch after the timed region (reported, not in the step)")
+    p.add_argument("--energy-seconds", type=float, default=0.25,
+                   help="per (kernel, variant) NVML energy window; 0 disables the energy table")
     p.add_argument("--ablations", action="store_true",
                    help="also time the INFLATE and NOCOMM ablations per kernel x RMT variant (cost attribution)")
     p.add_argument("--dist-backend", default="nccl",
@@ -441,6 +477,30 @@ def main():
                                      for v, s_ in xs.items()}
         extra["err_count"] = int(err.item())
 
+    # average power and energy per launch for every kernel x variant
+    energy = None
+    if args.energy_seconds > 0 and world == 1:
+        energy = {}
+        allv = variants + [v for v in args.extra_variants.split(",") if v and v not in variants]
+        for j in jobs:
+            d = {}
+            for v in allv:
+                wsx = ws.get((j.kernel, v))
+                if wsx is None:
+                    wsx = rmt.make_workspace(j.kernel, v, j.n, j.dims)
+                r = measure_energy(dev_index, lambda: rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims,
+                                                                 workspace=wsx, stream=stream.cuda_stream),
+                                   args.energy_seconds)
+                if r is None:
+                    d = None
+                    break
+                d[v] = r
+            if d is None:
+                energy = None
+                break
+            energy[j.kernel] = d
+        err.zero_()
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         rate, secs, cores, desc = oracle_sample_rate(jobs)
@@ -460,7 +520,7 @@ def main():
                                "gbs": kernels[best_none.kernel]["none"]["gbs"],
                                "frac": kernels[best_none.kernel]["none"]["frac"]} if best_none else None),
             "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
-            "attribution": attribution, "extra_variants": extra,
+            "attribution": attribution, "extra_variants": extra, "energy": energy,
             "gpu_launches": counts["gpu_launches"], "err_count": errs,
             "clocks": clk.summary(),
         }

@@ -49,6 +49,13 @@
  *                   performed once by the consumer.  Shared memory is outside
  *                   this variant's sphere of replication (a fault in the copy
  *                   is read by both replicas and is not detected).
+ *   RMT_DUP_KERNEL  naive kernel-level duplication (SURVEY 8(f) rank
+ *                   4): the unprotected kernel runs twice, each replica into its
+ *                   own shadow outputs (and scratch) in the workspace, then one
+ *                   compare kernel commits every aligned 4-word output group the
+ *                   two agree on and counts the others in *err_count (the paper
+ *                   compares on the host and re-executes; here the comparison
+ *                   stays on the device and the library only detects).
  *
  * Thread-safety: launches on different streams must use different workspaces.
  * The fault-injection and ablation state is process-global (test/bench use).
@@ -69,7 +76,8 @@ typedef enum {
     RMT_INTRA_REG = 2,
     RMT_INTER_GROUP = 3,
     RMT_INTER_CLUSTER = 4,
-    RMT_INTRA_NOLDS = 5
+    RMT_INTRA_NOLDS = 5,
+    RMT_DUP_KERNEL = 6
 } rmt_variant_t;
 
 /* The AMD APP SDK-style kernels the paper evaluates (Fig. 2 axis

@@ -45,7 +45,8 @@ const KEntry kTable[RMT_K_COUNT] = {
     KE(binomialoption, 1, 0, 0, 1, 1, 0),
 };
 
-const char* kVariantNames[6] = {"none", "intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds"};
+const char* kVariantNames[7] = {"none",        "intra_smem",  "intra_reg", "inter_group",
+                                "inter_cluster", "intra_nolds", "dup_kernel"};
 
 int check_device() {
   static int ok_dev = -1;
@@ -67,12 +68,85 @@ int check_device() {
 
 size_t dtype_bytes(int dt) { return dt == RMT_U64 ? 8 : dt == RMT_BF16 ? 2 : 4; }
 
+// 32-bit words of output buffer `which` (in kTable order) as a function of n:
+// every schema's outputs hold n elements, except FloydWarshall (n*n) and
+// Reduction (one u64).
+size_t out_words(int kernel, int64_t n) {
+  if (kernel == RMT_K_FLOYDWARSHALL) return (size_t)n * (size_t)n;
+  if (kernel == RMT_K_REDUCTION) return 2;
+  return (size_t)n;
+}
+
+// dup_kernel workspace: [scratch A][scratch B] then, per output buffer, the
+// two replicas' shadows.
+size_t dup_bytes(int kernel, int64_t n, const int64_t* dims, size_t* scr) {
+  const KEntry& e = kTable[kernel];
+  const size_t s = align_up(e.scratch(n, dims), 256);
+  if (scr) *scr = s;
+  return 2 * s + (size_t)e.nout * 2 * align_up(out_words(kernel, n) * 4, 256);
+}
+
 size_t ws_size(int kernel, int variant, int64_t n, const int64_t* dims, size_t* inter_part) {
   const KEntry& e = kTable[kernel];
   size_t ip = 0;
+  if (variant == RMT_DUP_KERNEL) {
+    if (inter_part) *inter_part = 0;
+    return dup_bytes(kernel, n, dims, nullptr);
+  }
   if (variant == RMT_INTER_GROUP) ip = align_up(inter_bytes(e.inter_warps(n, dims)), 256);
   if (inter_part) *inter_part = ip;
   return ip + align_up(e.scratch(n, dims), 256);
+}
+
+// Kernel-level duplication: two runs of the unprotected kernel into
+// shadows, then the on-device compare-and-commit.
+int run_dup(Launch& L0, const KEntry& e, char* ws, bool armed, const FaultDesc& f) {
+  const rmt_bufs_t* bufs = L0.bufs;
+  size_t scr = 0;
+  dup_bytes(L0.kernel, L0.n, bufs->dims, &scr);
+  const size_t ow = out_words(L0.kernel, L0.n);
+  const size_t sh = align_up(ow * 4, 256);
+  char* shadows = ws + 2 * scr;
+  rmt_bufs_t rb[2] = {*bufs, *bufs};
+  for (int r = 0; r < 2; ++r) {
+    for (int i = 0; i < e.nout; ++i) {
+      void* p = shadows + ((size_t)i * 2 + r) * sh;
+      const int bi = e.out[i];
+      bool inout = false;
+      for (int k = 0; k < e.nin; ++k) inout = inout || e.in[k] == bi;
+      // an in/out buffer: the replica starts from its own copy of the input;
+      // otherwise the shadows are poisoned differently (0xA5.. / 0x5A..) so that
+      // a word one replica failed to write (e.g. a flipped store address) differs
+      // from the other replica's value unless that value is the poison itself
+      int rc = inout ? cuda_check(cudaMemcpyAsync(p, bufs->buf[bi].ptr, ow * 4, cudaMemcpyDeviceToDevice, L0.stream),
+                                  "dup: copy in/out input")
+                     : cuda_check(cudaMemsetAsync(p, r ? 0x5A : 0xA5, ow * 4, L0.stream), "dup: poison shadow");
+      if (rc) return rc;
+      rb[r].buf[bi].ptr = p;
+    }
+  }
+  for (int r = 0; r < 2; ++r) {
+    Launch L = L0;
+    L.variant = RMT_NONE;
+    L.bufs = &rb[r];
+    L.scratch = ws + (size_t)r * scr;
+    L.scratch_bytes = scr;
+    L.launches = 0;
+    const bool hit = armed && f.replica == r;
+    L.mode = hit ? M_FAULT : M_NORMAL;
+    L.ctx.f = f;
+    L.ctx.f.replica = 0;  // the unprotected kernel is replica 0 of itself
+    int rc = e.run(L);
+    L0.launches += L.launches;
+    if (rc) return rc;
+  }
+  for (int i = 0; i < e.nout; ++i) {
+    const int bi = e.out[i];
+    int rc = dup_compare_launch(rb[0].buf[bi].ptr, rb[1].buf[bi].ptr, bufs->buf[bi].ptr, ow, L0.ctx.err, L0.stream);
+    if (rc) return rc;
+    L0.launches += 1;
+  }
+  return RMT_OK;
 }
 }  // namespace
 
@@ -94,7 +168,7 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
                void* workspace, size_t ws_bytes, void* stream) {
   g_last_launches = 0;
   if (kernel < 0 || kernel >= RMT_K_COUNT) { set_error("bad kernel id"); return RMT_EINVAL; }
-  if (variant < 0 || variant > RMT_INTRA_NOLDS) { set_error("bad variant id"); return RMT_EINVAL; }
+  if (variant < 0 || variant > RMT_DUP_KERNEL) { set_error("bad variant id"); return RMT_EINVAL; }
   if (!bufs || !err_count) { set_error("bufs and err_count must be non-NULL"); return RMT_EINVAL; }
   int rc = check_device();
   if (rc) return rc;
@@ -106,6 +180,23 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
   if (need > 0 && (workspace == nullptr || ws_bytes < need)) {
     set_error("workspace too small: need " + std::to_string(need) + " bytes");
     return RMT_EWORKSPACE;
+  }
+  if (variant == RMT_DUP_KERNEL) {
+    if (g_ablation != RMT_ABL_FULL && !g_armed) {
+      set_error("dup_kernel has no ablation modes");
+      return RMT_EUNSUPPORTED;
+    }
+    Launch L{};
+    L.kernel = kernel;
+    L.variant = variant;
+    L.bufs = bufs;
+    L.n = n;
+    L.stream = (cudaStream_t)stream;
+    L.ctx.err = err_count;
+    rc = run_dup(L, e, (char*)workspace, g_armed, g_fault);
+    g_last_launches = L.launches;
+    if (rc == RMT_OK) rc = cuda_check(cudaGetLastError(), "kernel launch");
+    return rc;
   }
   if (g_armed && variant == RMT_NONE && g_fault.replica != 0) {
     set_error("variant none has a single replica: fault replica must be 0");
@@ -141,7 +232,7 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
 }
 
 size_t rmt_workspace_size(int kernel, int variant, int64_t n, const int64_t* dims) {
-  if (kernel < 0 || kernel >= RMT_K_COUNT || variant < 0 || variant > RMT_INTRA_NOLDS) return 0;
+  if (kernel < 0 || kernel >= RMT_K_COUNT || variant < 0 || variant > RMT_DUP_KERNEL) return 0;
   int64_t zero[4] = {0, 0, 0, 0};
   return ws_size(kernel, variant, n, dims ? dims : zero, nullptr);
 }
@@ -232,7 +323,7 @@ const char* rmt_kernel_name(int kernel) {
 }
 
 const char* rmt_variant_name(int variant) {
-  return (variant >= 0 && variant <= RMT_INTRA_NOLDS) ? kVariantNames[variant] : "?";
+  return (variant >= 0 && variant <= RMT_DUP_KERNEL) ? kVariantNames[variant] : "?";
 }
 
 }  // extern "C"

@@ -101,6 +101,10 @@ RMT_DECLARE_KERNEL(dwthaar1d)
 RMT_DECLARE_KERNEL(bitonicsort)
 RMT_DECLARE_KERNEL(binomialoption)
 
+// dup_kernel: commit agreeing 4-word groups of shadows a, b to out; count the others.
+int dup_compare_launch(const void* a, const void* b, void* out, unsigned long long nwords, unsigned long long* err,
+                       cudaStream_t s);
+
 }  // namespace rmt
 
 namespace rmt {

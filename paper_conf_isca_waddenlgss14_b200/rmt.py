@@ -20,8 +20,9 @@ KERNELS = {
     "transpose": 5, "sobel": 6, "floydwarshall": 7, "dct": 8, "matmul": 9,
     "dwthaar1d": 10, "bitonicsort": 11, "binomialoption": 12,
 }
-VARIANTS = {"none": 0, "intra_smem": 1, "intra_reg": 2, "inter_group": 3, "inter_cluster": 4, "intra_nolds": 5}
-RMT_VARIANTS = ("intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds")
+VARIANTS = {"none": 0, "intra_smem": 1, "intra_reg": 2, "inter_group": 3, "inter_cluster": 4, "intra_nolds": 5,
+            "dup_kernel": 6}
+RMT_VARIANTS = ("intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds", "dup_kernel")
 SITES = {"load": 0, "compute": 1, "smem": 2, "store_val": 3, "store_addr": 4}
 ABLATIONS = {"full": 0, "nocomm": 1, "inflate": 2}
 

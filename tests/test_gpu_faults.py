@@ -97,7 +97,11 @@ def test_fault_campaign(idx):
                         continue
                     assert err >= 1, (f"{case.kernel}: live {site} fault (elem {elem}, bit {bit}) in replica "
                                       f"{replica} NOT detected by {variant}")
-                    if site.startswith("store") and case.kernel not in ("floydwarshall",):
+                    if variant == "dup_kernel" and site == "store_addr":
+                        # output comparison sees an address flip as two differing groups (the
+                        # skipped one, left poisoned, and the overwritten one), not as one commit
+                        assert err <= 2 or case.kernel == "floydwarshall"
+                    elif site.startswith("store") and case.kernel not in ("floydwarshall",):
                         assert err == 1, f"{case.kernel}/{variant}: {site} flip must corrupt exactly one commit"
                     detected += 1
         report[site] = (live, detected)

@@ -9,7 +9,7 @@ cfg = sys.argv[1]
 if os.environ.get("RMT_ABL"):  # full | nocomm | inflate
     rmt.set_ablation(os.environ["RMT_ABL"])
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
-variants = sys.argv[3].split(",") if len(sys.argv) > 3 else ["none", "intra_smem", "intra_reg", "inter_group", "inter_cluster"]
+variants = sys.argv[3].split(",") if len(sys.argv) > 3 else ["none", "intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds", "dup_kernel"]
 for j in workloads.config_jobs(cfg):
     b = j.device_buffers()
     base = None
