@@ -82,7 +82,7 @@ def parse():
     p.add_argument("--variants", default=",".join(VARIANTS))
     p.add_argument("--extra-variants", default=",".join(EXTRA_VARIANTS),
                    help="variants timed per launch after the timed region (reported, not in the step)")
-    p.add_argument("--energy-seconds", type=float, default=0.25,
+    p.add_argument("--energy-seconds", type=float, default=0.5,
                    help="per (kernel, variant) NVML energy window; 0 disables the energy table")
     p.add_argument("--ablations", action="store_true",
                    help="also time the INFLATE and NOCOMM ablations per kernel x RMT variant (cost attribution)")
