@@ -493,7 +493,7 @@ def small_cases():
         BlackScholes(1), BlackScholes(7), BlackScholes(1024 * 3 + 5), BlackScholes(1 << 16),
         Reduction(0), Reduction(3), Reduction(1000003), Reduction(1 << 22),
         Transpose(4, 4), Transpose(68, 132), Transpose(256, 512, index_coded=True), Transpose(1000, 764),
-        PrefixSum(1), PrefixSum(4095), PrefixSum(4096 * 37 + 11), PrefixSum(1 << 22),
+        PrefixSum(1), PrefixSum(4095), PrefixSum(4096 * 37 + 11), PrefixSum(1 << 22), PrefixSum((1 << 25) + 12347),
         FWT(1), FWT(2), FWT(64), FWT(4096), FWT(1 << 13), FWT(1 << 20), FWT(1 << 16, ternary=True),
         BinarySearch(0, 16), BinarySearch(1, 7), BinarySearch(1000, 1003), BinarySearch(1 << 16, 50000, odd=True),
         BinarySearch(1 << 22, 1 << 18),
