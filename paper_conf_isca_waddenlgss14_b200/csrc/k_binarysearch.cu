@@ -31,6 +31,8 @@ struct Levels {
   unsigned off[MAXLEV + 1];      // word offset of level k (k >= 1) in the scratch
   unsigned padded[MAXLEV + 1];   // entries rounded up to a multiple of 16
   unsigned vecs_before[MAXLEV + 2];  // index-build vector ranges
+  unsigned N16;                  // N rounded down to a multiple of 16
+  unsigned tail_off;             // word offset of the padded copy of A[N16, N) (16 words)
 };
 
 struct BsArgs {
@@ -59,10 +61,43 @@ Levels make_levels(unsigned N) {
   L.T = k;
   L.vecs_before[1] = 0;
   for (int i = 1; i <= L.T; ++i) L.vecs_before[i + 1] = L.vecs_before[i] + L.padded[i] / 4;
+  L.N16 = N & ~15u;
+  L.tail_off = off;
   return L;
 }
 
-// ---- index build: logical thread v writes 4 consecutive entries of one level
+// #{w_i >= k} over the 4 words: each unsigned compare is the carry of w - k
+// (sub.cc: carry = no borrow = w >= k), summed with addc -- two integer-pipe
+// instructions per key instead of a compare, a select and a bit-combine.
+__device__ __forceinline__ unsigned count_ge(uint4 w, unsigned k) {
+  unsigned c, t;
+  asm("{\n\t"
+      "sub.cc.u32 %1, %2, %6;\n\t"
+      "addc.u32 %0, 0, 0;\n\t"
+      "sub.cc.u32 %1, %3, %6;\n\t"
+      "addc.u32 %0, %0, 0;\n\t"
+      "sub.cc.u32 %1, %4, %6;\n\t"
+      "addc.u32 %0, %0, 0;\n\t"
+      "sub.cc.u32 %1, %5, %6;\n\t"
+      "addc.u32 %0, %0, 0;\n\t"
+      "}"
+      : "=r"(c), "=&r"(t)
+      : "r"(w.x), "r"(w.y), "r"(w.z), "r"(w.w), "r"(k));
+  return c;
+}
+
+// p + i (u32 elements) as one wide multiply-add (keeps nvcc from widening the
+// index sum with carries)
+__device__ __forceinline__ const unsigned* wide_addr(const unsigned* p, unsigned i) {
+  const unsigned* r;
+  asm("mad.wide.u32 %0, %1, 4, %2;" : "=l"(r) : "r"(i), "l"(p));
+  return r;
+}
+
+// ---- index build: logical thread v writes 4 consecutive entries of one level,
+// or (the last 4 vectors) 4 words of the padded tail block T[i] = A[N16 + i]
+// (0xFFFFFFFF past N), so the final level's 64-B block loads need no bounds
+// checks (branch-free: all of a thread's block loads are in flight together).
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
@@ -73,8 +108,9 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
   int k = 1;
 #pragma unroll 1
   while (k < a.L.T && v >= a.L.vecs_before[k + 1]) ++k;
-  const bool active = v < total;
-  const unsigned j0 = active ? (v - a.L.vecs_before[k]) * 4 : 0u;
+  const bool tail = v >= total && v < total + 4u;
+  const bool active = v < total || tail;
+  const unsigned j0 = tail ? (v - total) * 4 : active ? (v - a.L.vecs_before[k]) * 4 : 0u;
   unsigned stride = 1;
 #pragma unroll 1
   for (int i = 0; i < k; ++i) stride *= FAN;
@@ -82,10 +118,15 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
     const unsigned j = j0 + q;
-    const unsigned long long src = (unsigned long long)j * stride;
-    w[q] = (active && j < a.L.n[k]) ? __ldcs(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[16^k j] (A: evict-first)
+    if (tail) {
+      w[q] = a.L.N16 + j < a.N ? __ldg(a.A + a.L.N16 + j) : 0xFFFFFFFFu;
+    } else {
+      const unsigned long long src = (unsigned long long)j * stride;
+      w[q] = (active && j < a.L.n[k]) ? __ldcs(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[16^k j] (A: evict-first)
+    }
   }
-  rep.template commit<4, 1>(active ? 0xFu : 0u, active ? a.L.off[k] + j0 : 0u, w, 0xFFFFFFF0u,
+  const unsigned dst = tail ? a.L.tail_off + j0 : active ? a.L.off[k] + j0 : 0u;
+  rep.template commit<4, 1>(active ? 0xFu : 0u, dst, w, 0xFFFFFFF0u,
                             [&](unsigned i, unsigned m, const unsigned* x) {
                               if (m == 0xFu) *reinterpret_cast<uint4*>(a.lev + i) = make_uint4(x[0], x[1], x[2], x[3]);
                             });
@@ -134,32 +175,30 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 3 : 4) 
   for (int s = 0; s < VEC; ++s) jj[s] = a.N ? 1u : 0u;  // "block 0" of the top level
   // one level: J <- 16 (max(J,1) - 1) + #{block < key}.  When J = 0 (key <= every
   // entry) block 0 counts 0, so J stays 0 with no special case.
-  auto level = [&](const unsigned* P, unsigned lim, bool tail) {
+  const unsigned* tailp = a.lev + a.L.tail_off - a.L.N16;  // tailp[N16 + i] = T[i]
+  // per-lane quarter pointers: element (base + 4 gm) of level P is Pq + 16 base bytes
+  auto level = [&](const unsigned* P, bool last) {
+    const unsigned* Pq = P + 4 * gm;
+    const unsigned* Tq = tailp + 4 * gm;
 #pragma unroll
     for (int s = 0; s < VEC; ++s) {
       const unsigned mybase = (max(jj[s], 1u) - 1u) * FAN;
       unsigned packed = 0;
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
-        const unsigned base = rep.lshfl_idx(mybase, g0 + i) + 4u * gm;
+        const unsigned base = rep.lshfl_idx(mybase, g0 + i);
         uint4 w;
-        if (!tail) {  // sample levels: keep them L2-resident (default policy)
-          w = __ldg(reinterpret_cast<const uint4*>(P + base));
-        } else if (base + 4u <= lim) {  // the caller's A: random 64-B blocks, evict-first
-          w = __ldcs(reinterpret_cast<const uint4*>(P + base));
-        } else {  // tail of the caller's A: element-wise, never past lim
-          w.x = base + 0 < lim ? __ldcs(P + base + 0) : 0xFFFFFFFFu;
-          w.y = base + 1 < lim ? __ldcs(P + base + 1) : 0xFFFFFFFFu;
-          w.z = base + 2 < lim ? __ldcs(P + base + 2) : 0xFFFFFFFFu;
-          w.w = base + 3 < lim ? __ldcs(P + base + 3) : 0xFFFFFFFFu;
+        if (!last) {  // sample levels: keep them L2-resident (default policy)
+          w = __ldg(reinterpret_cast<const uint4*>(wide_addr(Pq, base)));
+        } else {  // the caller's A: random 64-B blocks, evict-first; the ragged
+                  // last block comes from the padded copy (a block never straddles N16)
+          w = __ldcs(reinterpret_cast<const uint4*>(wide_addr(base >= a.L.N16 ? Tq : Pq, base)));
         }
-        const unsigned k = K[i][s];
-        const unsigned bits = (w.x < k ? 1u : 0u) | (w.y < k ? 2u : 0u) | (w.z < k ? 4u : 0u) | (w.w < k ? 8u : 0u);
-        packed += (unsigned)__popc(bits) << (8 * i);
+        packed += count_ge(w, K[i][s]) << (8 * i);
       }
       packed += rep.lshfl_xor(packed, 1);  // sum the 4 quarters (bytes <= 16: no carries)
       packed += rep.lshfl_xor(packed, 2);
-      jj[s] = mybase + ((packed >> (8 * gm)) & 0xFFu);
+      jj[s] = mybase + FAN - ((packed >> (8 * gm)) & 0xFFu);  // #{block < key} = 16 - #{block >= key}
     }
   };
   for (int lv = a.L.T; lv >= 1; --lv) {  // padded sample levels: no bounds checks
@@ -172,7 +211,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 3 : 4) 
         }
       }
     }
-    level(a.lev + a.L.off[lv], a.L.padded[lv], false);
+    level(a.lev + a.L.off[lv], false);
   }
   if constexpr (M == M_FAULT) {
     if (a.L.T == 1) {
@@ -183,7 +222,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 3 : 4) 
       }
     }
   }
-  level(a.A, a.N, true);  // the caller's A
+  level(a.A, true);  // the caller's A
   rep.template commit<VEC, 0>(mask, j0, jj, a.Q, [&](unsigned i, unsigned m, const unsigned* w) {
     if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.idx + i), make_uint4(w[0], w[1], w[2], w[3]));
     else
@@ -208,7 +247,7 @@ size_t binarysearch_scratch(int64_t, const int64_t* dims) {
   Levels L = make_levels((unsigned)dims[0]);
   size_t words = 0;
   for (int k = 1; k <= L.T; ++k) words += L.padded[k];
-  return words * 4 + 64;
+  return (words + 16) * 4 + 64;  // + the padded tail block
 }
 int binarysearch_inter_warps(int64_t, const int64_t*) { return BL / 32; }
 
@@ -223,12 +262,12 @@ int binarysearch_run(Launch& L) {
   a.Q = Q;
   a.L = make_levels(N);
   a.top_iters = 0;
-  const unsigned Gi = (a.L.vecs_before[a.L.T + 1] + BL - 1) / BL;
+  const unsigned Gi = (a.L.vecs_before[a.L.T + 1] + 4 + BL - 1) / BL;
   const unsigned G = (Q + BL * VEC - 1) / (BL * VEC);
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     int rc = RMT_OK;
-    if (a.L.T > 0 && Q > 0)
+    if (Q > 0)
       rc = launch_std<V>(L, bins_index_kernel<V, M>, bins_index_kernel<V_NONE, M_NORMAL>, Gi, BL, 0, a,
                          "binarysearch/index");
     if (rc) return rc;

@@ -496,7 +496,8 @@ def small_cases():
         PrefixSum(1), PrefixSum(4095), PrefixSum(4096 * 37 + 11), PrefixSum(1 << 22), PrefixSum((1 << 25) + 12347),
         FWT(1), FWT(2), FWT(64), FWT(4096), FWT(1 << 13), FWT(1 << 20), FWT(1 << 16, ternary=True),
         BinarySearch(0, 16), BinarySearch(1, 7), BinarySearch(1000, 1003), BinarySearch(1 << 16, 50000, odd=True),
-        BinarySearch(1 << 22, 1 << 18),
+        BinarySearch(1 << 22, 1 << 18), BinarySearch(15, 100, odd=True), BinarySearch(17, 999),
+        BinarySearch((1 << 20) + 13, 70001), BinarySearch(4096 + 9, 5000, odd=True),
         Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
         DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8),
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
