@@ -11,7 +11,9 @@
 // separable Sobel (vertical smooth / difference per column, then horizontal).
 // isqrt: floor(sqrt(s)/2) = isqrt(s/4); computed as floor(sqrt_approx(s/4 + 1/8))
 // which is exact for every s whose result is < 256 (margin >= 9.6e-7 relative
-// vs approx error < 2^-22); larger results saturate to 255 anyway.
+// vs approx error < 2^-22); larger results saturate to 255 anyway.  floor is
+// one FADD2 with the magic 2^23 - 1/2; saturation one VIMNMX.U16x2 per two
+// channels.
 #include "rmt_host.cuh"
 
 namespace rmt {
@@ -60,9 +62,9 @@ __device__ __forceinline__ f2_t fma2(f2_t a, f2_t b, f2_t c) {
 }
 
 // Two channels at once: gw, yw hold two biased 16-bit lanes (value + 1024) of
-// Gx and Gy.  Returns two words whose low byte is the output of the low / high
-// lane channel.  s = Gx^2 + Gy^2 < 2^21 is exact in fp32; out = min(255,
-// floor(sqrt_approx(s/4 + 1/8))) (exact: see the header).  The 16-bit lanes
+// Gx and Gy.  Returns two words 2^23 + floor(sqrt_approx(s/4 + 1/8)) (as fp32
+// bits; the low 10 bits hold the unsaturated output of the low / high lane
+// channel).  s = Gx^2 + Gy^2 < 2^21 is exact in fp32 (exact: see the header).  The 16-bit lanes
 // become floats through the 2^23 magic (PRMT + FADD2), no conversion pipe.
 __device__ __forceinline__ void sobel_mag2(unsigned gw, unsigned yw, unsigned& out_lo, unsigned& out_hi) {
   const unsigned MAG = 0x4B000000u;
@@ -75,10 +77,11 @@ __device__ __forceinline__ void sobel_mag2(unsigned gw, unsigned yw, unsigned& o
                       f2(__float_as_uint(0.125f), __float_as_uint(0.125f)));  // s/4 + 1/8, exact
   unsigned f0, f1;
   f2_split(f, f0, f1);
-  const float r0 = fminf(sqrt_approx(__uint_as_float(f0)), 255.25f);
-  const float r1 = fminf(sqrt_approx(__uint_as_float(f1)), 255.25f);
-  f2_t r = add2(f2(__float_as_uint(r0), __float_as_uint(r1)), f2(__float_as_uint(-0.5f), __float_as_uint(-0.5f)));
-  r = add2(r, f2(__float_as_uint(12582912.0f), __float_as_uint(12582912.0f)));  // RN(r - 1/2) = floor(r)
+  const float r0 = sqrt_approx(__uint_as_float(f0));
+  const float r1 = sqrt_approx(__uint_as_float(f1));
+  // RN(r + 2^23 - 1/2) = 2^23 + floor(r) for r >= sqrt(1/8): r is never a
+  // half-integer (2 (2k+1)^2 != 2 s + 1); the caller saturates at 255
+  const f2_t r = add2(f2(__float_as_uint(r0), __float_as_uint(r1)), f2(__float_as_uint(8388607.5f), __float_as_uint(8388607.5f)));
   f2_split(r, out_lo, out_hi);
 }
 
@@ -148,7 +151,10 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) sobel_kernel(SobArgs a, Ctx
       unsigned m0, m2, m1, m3;
       sobel_mag2(gx_lo, gy_lo, m0, m2);  // channels 0, 2
       sobel_mag2(gx_hi, gy_hi, m1, m3);  // channels 1, 3
-      const unsigned px = __byte_perm(__byte_perm(m0, m1, 0x0040), __byte_perm(m2, m3, 0x0040), 0x5410);
+      // two channels per 16-bit lane pair, saturated with one VIMNMX.U16x2 each
+      const unsigned h01 = __vminu2(__byte_perm(m0, m1, 0x5410), 0x00FF00FFu);
+      const unsigned h23 = __vminu2(__byte_perm(m2, m3, 0x5410), 0x00FF00FFu);
+      const unsigned px = __byte_perm(h01, h23, 0x6420);
       out[p] = (yin && ((xin >> p) & 1u)) ? px : 0u;
     }
     const unsigned mask = (active && y < (int)a.H) ? 0xFu : 0u;

@@ -75,9 +75,10 @@ def _to_dev(a: np.ndarray) -> torch.Tensor:
 def job_binarysearch(N, Q, seed=6, rank=0):
     A, _ = inputs.binarysearch_inputs(seed, N, 1)
     q = inputs.u32(seed, Q, rank * Q, stream=2)
-    return Job("binarysearch", Q, (N, Q), [A, q, None], [(2, 4 * Q)], alg_bytes=40 * Q, unit="queries",
-               bound="latency", note="40 B/query compulsory: q + idx + the one 32-B sector of A holding the answer "
-                                     "(any comparison search must touch it); upper levels are L2-resident")
+    return Job("binarysearch", Q, (N, Q), [A, q, None], [(2, 4 * Q)], alg_bytes=136 * Q, unit="queries",
+               note="136 B/query compulsory: q + idx + the 128-B DRAM line of A holding the answer (any comparison "
+                    "search must touch it; a random access of 4..128 B moves one ~128-B line on B200, measured by "
+                    "tools/gather_probe.cu); upper levels are L2-resident")
 
 
 def job_fwt(N, seed=5, rank=0):
