@@ -89,17 +89,27 @@ struct Row {
   unsigned lo[6], hi[6];  // columns x0-1 .. x0+4, channels (0,2) and (1,3)
 };
 
+// Raw words of one input row (columns x0-1 .. x0+4); zeros outside the image.
 template <int V, int M>
-__device__ __forceinline__ void load_row(const Rep<V, M>& rep, const SobArgs& a, int y, unsigned x0, bool active,
-                                         Row& R) {
-  unsigned p[6] = {0, 0, 0, 0, 0, 0};
+__device__ __forceinline__ void load_raw(const Rep<V, M>& rep, const SobArgs& a, int y, unsigned x0, bool active,
+                                         unsigned (&p)[6]) {
+#pragma unroll
+  for (int k = 0; k < 6; ++k) p[k] = 0u;
   if (active && y >= 0 && y < (int)a.H) {
     const unsigned* row = a.I + (size_t)y * a.W;
     uint4 c = __ldg(reinterpret_cast<const uint4*>(row + x0));
     p[1] = c.x; p[2] = c.y; p[3] = c.z; p[4] = c.w;
     if (x0 >= 1) p[0] = __ldg(row + x0 - 1);
     if (x0 + 4 < a.W) p[5] = __ldg(row + x0 + 4);
-    if constexpr (M == M_FAULT) {
+  }
+}
+
+// Apply the LOAD-site fault hook and split into 16-bit channel lanes.
+template <int V, int M>
+__device__ __forceinline__ void unpack_row(const Rep<V, M>& rep, const SobArgs& a, int y, unsigned x0,
+                                           unsigned (&p)[6], Row& R) {
+  if constexpr (M == M_FAULT) {
+    if (y >= 0 && y < (int)a.H) {
 #pragma unroll
       for (int k = 0; k < 6; ++k) {
         long long e = (long long)y * a.W + x0 + k - 1;
@@ -167,12 +177,21 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) sobel_kernel(SobArgs a, Ctx
                                     if ((mm >> k) & 1u) a.O[idx + k] = w[k];
                               });
   };
+  // rolling 3-row window; the raw words of the row after next are in flight
+  // while the current row is filtered (one row of prefetch distance)
   Row top, mid, bot;
-  load_row(rep, a, y0 - 1, x0, active, top);
-  load_row(rep, a, y0, x0, active, mid);
+  unsigned raw[6], nxt[6];
+  load_raw(rep, a, y0 - 1, x0, active, raw);
+  unpack_row(rep, a, y0 - 1, x0, raw, top);
+  load_raw(rep, a, y0, x0, active, raw);
+  load_raw(rep, a, y0 + 1, x0, active, nxt);
+  unpack_row(rep, a, y0, x0, raw, mid);
 #pragma unroll 1
   for (int y = y0; y < y0 + RY; ++y) {
-    load_row(rep, a, y + 1, x0, active, bot);
+#pragma unroll
+    for (int k = 0; k < 6; ++k) raw[k] = nxt[k];
+    load_raw(rep, a, y + 2, x0, active, nxt);
+    unpack_row(rep, a, y + 1, x0, raw, bot);
     row_out(y, top, mid, bot);
     top = mid;
     mid = bot;
