@@ -278,6 +278,183 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
   rep.finish();
 }
 
+// ---------------------------------------------------------------- specialised passes
+// Tiles of 4096 elements, BLS = 128 logical threads x 32 elements.  Register
+// rounds of up to 5 stages; the first round of each pass runs on the loaded
+// registers and the last writes straight to global memory, so a pass touches
+// shared memory only between rounds:
+//   pass 1  (stages 0..11, contiguous tile):  float4 load -> stages 0,1 in
+//           registers -> STS -> round A (stages 2..6, 32 elements at stride 4)
+//           -> round B (stages 7..11, 32 elements at stride 128) -> STG
+//           (2 STS + 2 LDS per element instead of 4 + 4);
+//   strided (7 stages on the 128 rows of a 128 x 32 tile): 32 row loads per
+//           thread (each warp load = one 128-B row) -> stages on row bits 0..4 in
+//           registers -> STS -> stages on row bits 5, 6 (4 elements) -> STG
+//           (1 STS + 1 LDS per element instead of 3 + 3).
+// Stores are 4-word commits of elements at a fixed stride (each warp store
+// instruction covers 128 contiguous bytes).
+constexpr int BLS = 128;
+
+// Pass-1 layout: phys(e) = e + (e >> 5) (one pad word per 32) makes each of the
+// three access patterns (float4 staging: e = 4t + c + 512 it; round A:
+// e = (t & 3) + 4k + 128 (t >> 2); round B: e = t + 128 k) hit 32 distinct banks
+// over a warp, and it is additive over the disjoint bit fields of a thread's
+// base and the compile-time k, so every access is one LDS/STS with an
+// immediate offset.  +LDS replica planes sit P1_PLANE (== 16 mod 32) words
+// apart: disjoint banks in rounds A and B (a warp's 16 logical lanes cover 16
+// consecutive banks); the staging stores of a pair share banks (2-way).
+constexpr int P1_WORDS = TE_MAX + TE_MAX / 32;
+constexpr int P1_PLANE = P1_WORDS + 16;
+__device__ __forceinline__ constexpr int p1_phys(int e) { return e + (e >> 5); }
+
+template <int NB>
+__device__ __forceinline__ void butterflies(float (&v)[1 << NB]) {
+#pragma unroll
+  for (int s = 0; s < NB; ++s) {
+    const int h = 1 << s;
+#pragma unroll
+    for (int k = 0; k < (1 << NB); ++k) {
+      if (k & h) continue;
+      const float x0 = v[k], x1 = v[k + h];
+      v[k] = __fadd_rn(x0, x1);
+      v[k + h] = __fsub_rn(x0, x1);
+    }
+  }
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, Ctx c) {
+  using R = Rep<V, M>;
+  constexpr bool DUPL = R::SMDUP;
+  __shared__ unsigned mb[mbox_words<V>(BLS * Geom<V>::DUP)];
+  __shared__ float tile[DUPL ? P1_PLANE + P1_WORDS : P1_WORDS];
+  R rep(c);
+  rep.init(mb);
+  const unsigned tileid = (unsigned)rep.lblock;
+  const unsigned gbase = tileid << TB_MAX;
+  float* const tp = tile + (DUPL ? P1_PLANE * rep.r : 0);  // this replica's plane
+  const int t = rep.ltid;
+  // load: 8 coalesced float4 per thread, all in flight before the first use
+  float4 f[8];
+#pragma unroll
+  for (int it = 0; it < 8; ++it) f[it] = *reinterpret_cast<const float4*>(a.src + gbase + 4 * t + 512 * it);
+  float* const ps = tp + p1_phys(4 * t);  // + p1_phys(512 it) + k: compile-time offsets
+#pragma unroll
+  for (int it = 0; it < 8; ++it) {
+    const int e0 = 4 * t + 512 * it;
+    float v[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
+    if constexpr (M == M_FAULT) {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) v[k] = rep.faultf(SITE_LOAD, (long long)gbase + e0 + k, v[k]);
+    }
+    butterflies<2>(v);  // stages 0, 1 (element bits 0, 1)
+    unsigned w[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_COMPUTE, (long long)gbase + e0 + k, v[k]);
+      w[k] = __float_as_uint(v[k]);
+    }
+    if (rep.template sts_ok<4>(w, (unsigned)e0)) {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) ps[p1_phys(512 * it) + k] = v[k];
+    }
+  }
+  __syncthreads();
+  {  // round A: stages 2..6 on elements ebase + 4k
+    const int ebase = (t & 3) | ((t >> 2) << 7);
+    float* const pb = tp + p1_phys(ebase);  // + p1_phys(4k): compile-time offsets
+    float v[32];
+#pragma unroll
+    for (int k = 0; k < 32; ++k) {
+      v[k] = pb[p1_phys(4 * k)];
+      if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_SMEM, (long long)gbase + ebase + 4 * k, v[k]);
+    }
+    butterflies<5>(v);
+    unsigned w[32];
+#pragma unroll
+    for (int k = 0; k < 32; ++k) w[k] = __float_as_uint(v[k]);
+    // each thread reads and rewrites its own 32 elements: no barrier inside the round
+    if (rep.template sts_ok<32>(w, (unsigned)ebase)) {
+#pragma unroll
+      for (int k = 0; k < 32; ++k) pb[p1_phys(4 * k)] = v[k];
+    }
+  }
+  __syncthreads();
+  // round B: stages 7..11 on elements t + 128k, then 8 strided commits
+  float* const pt = tp + p1_phys(t);
+  float v[32];
+#pragma unroll
+  for (int k = 0; k < 32; ++k) v[k] = pt[p1_phys(128 * k)];
+  butterflies<5>(v);
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    unsigned w[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) w[u] = __float_as_uint(v[4 * j + u]);
+    rep.template commit<4, 0>(0xFu, gbase + t + 512 * j, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if ((m >> u) & 1u) a.dst[idx + 128 * u] = __uint_as_float(x[u]);
+    }, /*defer=*/j < 7, /*stride=*/128u);
+  }
+  rep.finish();
+}
+
+// Strided pass: stages [s0, s0 + 7) on tiles of 128 rows (global stride 2^s0)
+// x 32 contiguous columns.  Layout e = col | row << 5 (bank = col), replica
+// planes XOR bank bit 4 (a warp's 16 logical lanes share it).
+template <int V, int M>
+__global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_ps_kernel(FwtArgs a, Ctx c) {
+  using R = Rep<V, M>;
+  constexpr bool DUPL = R::SMDUP;
+  __shared__ unsigned mb[mbox_words<V>(BLS * Geom<V>::DUP)];
+  __shared__ float tile[TE_MAX * Geom<V>::SMDUP];
+  R rep(c);
+  rep.init(mb);
+  const unsigned tileid = (unsigned)rep.lblock;
+  const int t = rep.ltid;
+  const int col = t & 31, g = t >> 5;
+  // this replica's plane, column pre-applied (bank bit 4 flipped for replica 1):
+  // element (col, row) is tc[row << 5], a compile-time offset from a per-thread base
+  float* const tc = tile + (DUPL ? TE_MAX * rep.r : 0) + (col ^ (DUPL && rep.r ? 16 : 0));
+  // global index of tile element (col, row): row bits land at s0.. (gindex_k<2>)
+  const int midb = a.s0 - 5;
+  const unsigned gcol = ((tileid >> midb) << (a.s0 + 7)) | ((tileid & ((1u << midb) - 1u)) << 5) | (unsigned)col;
+  // rows 32 g + i, i = 0..31: one 128-B row per warp load
+  float v[32];
+#pragma unroll
+  for (int i = 0; i < 32; ++i) v[i] = a.src[gcol + ((unsigned)(32 * g + i) << a.s0)];
+  butterflies<5>(v);  // stages s0 .. s0+4 (row bits 0..4)
+  unsigned w[32];
+#pragma unroll
+  for (int i = 0; i < 32; ++i) w[i] = __float_as_uint(v[i]);
+  if (rep.template sts_ok<32>(w, (unsigned)(col | (32 * g) << 5))) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) tc[(32 * g + i) << 5] = v[i];
+  }
+  __syncthreads();
+  // stages s0+5, s0+6 (row bits 5, 6): 8 groups of 4 rows {rlo + 32 k}
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const int rlo = g + 4 * j;
+    float q[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) q[k] = tc[(rlo + 32 * k) << 5];
+    butterflies<2>(q);
+    unsigned x[4];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) x[k] = __float_as_uint(q[k]);
+    const unsigned stride = 1u << (a.s0 + 5);
+    rep.template commit<4, 0>(0xFu, gcol + ((unsigned)rlo << a.s0), x, a.N,
+                              [&](unsigned idx, unsigned m, const unsigned* y) {
+#pragma unroll
+                                for (int k = 0; k < 4; ++k)
+                                  if ((m >> k) & 1u) a.dst[idx + stride * k] = __uint_as_float(y[k]);
+                              }, /*defer=*/j < 7, stride);
+  }
+  rep.finish();
+}
+
 int log2u(int64_t n) {
   int m = 0;
   while ((1LL << m) < n) ++m;
@@ -311,13 +488,13 @@ int fwt_run(Launch& L) {
     L.ctx.f.sid = (tb < m) ? -1 : sid;
     FwtArgs a{x, y, (unsigned)L.n, tb, 0, tb, 0};
     int rc = tb == TB_MAX
-                 ? launch_std<V>(L, fwt_kernel<V, M, 1>, fwt_kernel<V_NONE, M_NORMAL, 1>, tiles, BL, 0, a, "fwt/pass1")
+                 ? launch_std<V>(L, fwt_p1_kernel<V, M>, fwt_p1_kernel<V_NONE, M_NORMAL>, tiles, BLS, 0, a, "fwt/pass1")
                  : launch_std<V>(L, fwt_kernel<V, M, 0>, fwt_kernel<V_NONE, M_NORMAL, 0>, tiles, BL, 0, a, "fwt/pass1");
     for (int s = tb; s < m && rc == RMT_OK; ) {  // strided passes, in place on y
       const int b = (m - s) < 7 ? (m - s) : 7;
       L.ctx.f.sid = (s + b < m) ? -1 : sid;
       FwtArgs p{y, y, (unsigned)L.n, TB_MAX, s, b, TB_MAX - b};
-      rc = b == 7 ? launch_std<V>(L, fwt_kernel<V, M, 2>, fwt_kernel<V_NONE, M_NORMAL, 2>, tiles, BL, 0, p, "fwt/pass")
+      rc = b == 7 ? launch_std<V>(L, fwt_ps_kernel<V, M>, fwt_ps_kernel<V_NONE, M_NORMAL>, tiles, BLS, 0, p, "fwt/pass")
                   : launch_std<V>(L, fwt_kernel<V, M, 0>, fwt_kernel<V_NONE, M_NORMAL, 0>, tiles, BL, 0, p, "fwt/pass");
       s += b;
     }

@@ -23,7 +23,9 @@
 //       - INTER     : bounded per-(pair, warp) queue in global memory with
 //         release/acquire flags (P:691 two-tier locking, P:693 L2-coherent reads),
 //         region ownership handed over by a per-region turn counter;
-//   * warp-aggregated error counting (one atomicAdd per warp with mismatches).
+//   * error counting: inter variants one atomicAdd per warp with mismatches
+//     (warp ballot at every commit); intra variants a per-lane count added once
+//     at finish().
 //
 // Determinism rule for bodies: everything that feeds a commit must be computed
 // identically in every variant.
@@ -194,12 +196,13 @@ struct Rep {
   int lblock;     // logical CTA id
   int lane, warp, llane;
   unsigned j;     // records this warp has committed (inter)
+  unsigned nerr;  // intra: mismatching commits of this (consumer) lane, added to *err at finish()
   unsigned pend;  // inter: records not yet published (producer) / freed (consumer)
   unsigned region, epoch;
   unsigned* mbox;  // intra_smem: this warp's mailbox
   unsigned cl_pay, cl_full;  // inter_cluster: this warp's mailbox / flags in the consumer CTA (shared::cluster)
 
-  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), pend(0), region(0), epoch(0), mbox(nullptr), cl_pay(0), cl_full(0) {}
+  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), nerr(0), pend(0), region(0), epoch(0), mbox(nullptr), cl_pay(0), cl_full(0) {}
 
   // Must be called by every thread of the CTA, first thing (may __syncthreads).
   // mbox_smem: MBOX_WORDS * (blockDim/32) words of shared memory (intra_smem only).
@@ -305,6 +308,9 @@ struct Rep {
   }
 
   __device__ __forceinline__ void finish() {
+    if constexpr (INTRA) {  // deferred error count (mismatches are rare: one atomic per faulty lane)
+      if (nerr != 0u) atomicAdd(c.err, (unsigned long long)nerr);
+    }
     if constexpr (CLUSTER && !NOCOMM) {
       flush();
       cluster_sync_all();  // no DSMEM access of either CTA is in flight when they exit
@@ -438,16 +444,19 @@ struct Rep {
   //         before any CTA-wide barrier, and a run of deferred commits plus its
   //         closing commit must not exceed INTER_S records (deadlock freedom,
   //         DESIGN.md "Inter-Group queue").
+  //   stride element distance between consecutive words (1: a contiguous vector;
+  //         the store functor places word k at idx + k * stride)
   template <int NW, int SID = 0, bool LIVE = false, class Store>
   __device__ __forceinline__ void commit(unsigned mask, unsigned idx, unsigned (&v)[NW], unsigned limit,
-                                         Store&& store, bool defer = false) {
+                                         Store&& store, bool defer = false, unsigned stride = 1) {
     static_assert(NW >= 1 && NW <= MAXW, "commit width");
     bool addr_faulted = false;
     if constexpr (FAULT) {
-      if (c.f.sid == SID && c.f.replica == r && c.f.elem >= (long long)idx &&
-          c.f.elem < (long long)idx + NW) {
+      const long long d = c.f.elem - (long long)idx;
+      if (c.f.sid == SID && c.f.replica == r && d >= 0 && d % (long long)stride == 0 &&
+          d / (long long)stride < NW) {
         if (c.f.site == SITE_STORE_VAL) {
-          int w = (int)(c.f.elem - (long long)idx);
+          int w = (int)(d / (long long)stride);
 #pragma unroll
           for (int k = 0; k < NW; ++k)
             if (k == w) v[k] ^= 1u << c.f.bit;
@@ -461,7 +470,7 @@ struct Rep {
       if (mask != 0u) {
         if constexpr (FAULT) {
           // a faulted address whose stored words fall outside the buffer: dropped
-          if (addr_faulted && idx + (31u - (unsigned)__clz(mask)) >= limit) return;
+          if (addr_faulted && idx + (31u - (unsigned)__clz(mask)) * stride >= limit) return;
         }
         store(idx, mask, v);
       }
@@ -561,13 +570,18 @@ struct Rep {
         } else {
           mism = true;
           if constexpr (LIVE) {  // highest stored word must be inside the buffer
-            if (mask != 0u && idx + (31u - (unsigned)__clz(mask)) < limit) store(idx, mask, v);
+            if (mask != 0u && idx + (31u - (unsigned)__clz(mask)) * stride < limit) store(idx, mask, v);
           }
         }
       }
-      // warp ballot over the compare results: completes every lane's loads
-      const unsigned mb = __ballot_sync(FULL, mism);
-      if (mb != 0u && lane == __ffs(mb) - 1) atomicAdd(c.err, (unsigned long long)__popc(mb));
+      if constexpr (INTRA) {
+        nerr += mism ? 1u : 0u;  // counted at finish(): no per-commit vote
+      } else {
+        // warp ballot over the compare results: completes every lane's loads
+        // (the inter queue frees the slots only after it)
+        const unsigned mb = __ballot_sync(FULL, mism);
+        if (mb != 0u && lane == __ffs(mb) - 1) atomicAdd(c.err, (unsigned long long)__popc(mb));
+      }
       if constexpr (INTER || CLUSTER) {
         ++j;
         ++pend;

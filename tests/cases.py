@@ -199,6 +199,23 @@ class FWT(Case):
     def out_elems(self):
         return 1, self.n
 
+    def commit_group(self, e):
+        # the final pass's 4-word commit holding word e (k_fwt.cu): the pass-1
+        # kernel (N = 4096) commits elements at stride 128, a 7-stage strided pass
+        # at stride 2^(s0+5), the generic pass 4 contiguous words
+        m = self.n.bit_length() - 1
+        if m < 12:
+            return super().commit_group(e)
+        b = (m - 12) % 7 or 7 if m > 12 else 0
+        if m == 12:
+            stride = 128
+        elif b == 7:
+            stride = 1 << (m - 7 + 5)
+        else:
+            return super().commit_group(e)
+        lo = e & ~(3 * stride)
+        return lo + stride * np.arange(4)
+
 
 class BinarySearch(Case):
     kernel = "binarysearch"
@@ -494,7 +511,7 @@ def small_cases():
         Reduction(0), Reduction(3), Reduction(1000003), Reduction(1 << 22),
         Transpose(4, 4), Transpose(68, 132), Transpose(256, 512, index_coded=True), Transpose(1000, 764),
         PrefixSum(1), PrefixSum(4095), PrefixSum(4096 * 37 + 11), PrefixSum(1 << 22), PrefixSum((1 << 25) + 12347),
-        FWT(1), FWT(2), FWT(64), FWT(4096), FWT(1 << 13), FWT(1 << 20), FWT(1 << 16, ternary=True),
+        FWT(1), FWT(2), FWT(64), FWT(4096), FWT(1 << 13), FWT(1 << 19), FWT(1 << 20), FWT(1 << 16, ternary=True),
         BinarySearch(0, 16), BinarySearch(1, 7), BinarySearch(1000, 1003), BinarySearch(1 << 16, 50000, odd=True),
         BinarySearch(1 << 22, 1 << 18), BinarySearch(15, 100, odd=True), BinarySearch(17, 999),
         BinarySearch((1 << 20) + 13, 70001), BinarySearch(4096 + 9, 5000, odd=True),
