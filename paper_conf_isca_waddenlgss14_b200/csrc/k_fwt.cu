@@ -295,17 +295,25 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
 // instruction covers 128 contiguous bytes).
 constexpr int BLS = 128;
 
-// Pass-1 layout: phys(e) = e + (e >> 5) (one pad word per 32) makes each of the
-// three access patterns (float4 staging: e = 4t + c + 512 it; round A:
-// e = (t & 3) + 4k + 128 (t >> 2); round B: e = t + 128 k) hit 32 distinct banks
-// over a warp, and it is additive over the disjoint bit fields of a thread's
-// base and the compile-time k, so every access is one LDS/STS with an
-// immediate offset.  +LDS replica planes sit P1_PLANE (== 16 mod 32) words
-// apart: disjoint banks in rounds A and B (a warp's 16 logical lanes cover 16
-// consecutive banks); the staging stores of a pair share banks (2-way).
+// Pass-1 layouts.  Three access patterns: staging (float4 chunk t + 128 it),
+// round A (e = (t & 3) + 4k + 128 (t >> 2)), round B (e = t + 128 k).
+//  * none: XOR swizzle p1x(e) = e ^ ((e >> 5) & 31), a bank permutation for
+//    each pattern over 32 lanes (measured 0.264 vs 0.283 ms at 2^26 against the
+//    pad layout below: the address arithmetic spaces out the shared-memory
+//    instructions of the unprotected kernel).
+//  * RMT variants: pad layout (measured faster for every one of them)
+//    p1_phys(e) = e + 4 (e >> 7) (one 16-B pad per 128 words): float4 chunks
+//    stay aligned (staging is one STS.128), every pattern is conflict-free, and
+//    it is additive over the disjoint bit fields of a thread's base and the
+//    compile-time k (immediate offsets: fewer issued instructions, which is
+//    what bounds the doubled intra kernels).  +LDS replica planes sit P1_PLANE
+//    (== 16 mod 32) words apart: a warp's 16 logical lanes cover 16
+//    consecutive banks in rounds A and B and 4 chunks per quarter-warp in
+//    staging, so the two replicas of a pair never share a bank.
 constexpr int P1_WORDS = TE_MAX + TE_MAX / 32;
 constexpr int P1_PLANE = P1_WORDS + 16;
-__device__ __forceinline__ constexpr int p1_phys(int e) { return e + (e >> 5); }
+__device__ __forceinline__ constexpr int p1_phys(int e) { return e + 4 * (e >> 7); }
+__device__ __forceinline__ int p1x(int e) { return e ^ ((e >> 5) & 31); }
 
 template <int NB>
 __device__ __forceinline__ void butterflies(float (&v)[1 << NB]) {
@@ -326,8 +334,9 @@ template <int V, int M>
 __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, Ctx c) {
   using R = Rep<V, M>;
   constexpr bool DUPL = R::SMDUP;
+  constexpr bool PAD = V != V_NONE;  // layout choice (see p1_phys / p1x): measured per variant
   __shared__ unsigned mb[mbox_words<V>(BLS * Geom<V>::DUP)];
-  __shared__ float tile[DUPL ? P1_PLANE + P1_WORDS : P1_WORDS];
+  __shared__ __align__(16) float tile[DUPL ? P1_PLANE + P1_WORDS : P1_WORDS];
   R rep(c);
   rep.init(mb);
   const unsigned tileid = (unsigned)rep.lblock;
@@ -355,18 +364,23 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, C
       w[k] = __float_as_uint(v[k]);
     }
     if (rep.template sts_ok<4>(w, (unsigned)e0)) {
+      if constexpr (PAD) {
+        *reinterpret_cast<float4*>(ps + p1_phys(512 * it)) = make_float4(v[0], v[1], v[2], v[3]);
+      } else {
 #pragma unroll
-      for (int k = 0; k < 4; ++k) ps[p1_phys(512 * it) + k] = v[k];
+        for (int k = 0; k < 4; ++k) tp[p1x(e0 + k)] = v[k];
+      }
     }
   }
   __syncthreads();
   {  // round A: stages 2..6 on elements ebase + 4k
     const int ebase = (t & 3) | ((t >> 2) << 7);
     float* const pb = tp + p1_phys(ebase);  // + p1_phys(4k): compile-time offsets
+    auto at = [&](int k) -> float& { return PAD ? pb[p1_phys(4 * k)] : tp[p1x(ebase + 4 * k)]; };
     float v[32];
 #pragma unroll
     for (int k = 0; k < 32; ++k) {
-      v[k] = pb[p1_phys(4 * k)];
+      v[k] = at(k);
       if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_SMEM, (long long)gbase + ebase + 4 * k, v[k]);
     }
     butterflies<5>(v);
@@ -376,7 +390,7 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, C
     // each thread reads and rewrites its own 32 elements: no barrier inside the round
     if (rep.template sts_ok<32>(w, (unsigned)ebase)) {
 #pragma unroll
-      for (int k = 0; k < 32; ++k) pb[p1_phys(4 * k)] = v[k];
+      for (int k = 0; k < 32; ++k) at(k) = v[k];
     }
   }
   __syncthreads();
@@ -384,7 +398,7 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, C
   float* const pt = tp + p1_phys(t);
   float v[32];
 #pragma unroll
-  for (int k = 0; k < 32; ++k) v[k] = pt[p1_phys(128 * k)];
+  for (int k = 0; k < 32; ++k) v[k] = PAD ? pt[p1_phys(128 * k)] : tp[p1x(t + 128 * k)];
   butterflies<5>(v);
 #pragma unroll
   for (int j = 0; j < 8; ++j) {
