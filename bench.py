@@ -101,6 +101,24 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
+def load_tensor_peak():
+    """Dense bf16 TFLOP/s: the SUSTAINED measured figure (a matmul launch sits
+    inside a long step of back-to-back launches), else the guide's fallback."""
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            pk = json.load(f)
+        return float(pk["bf16_tflops_sustained"]), "measured sustained bf16 (MEASURED_PEAKS.json)"
+    except Exception:
+        return 2250.0 * 0.75, "fallback (B200_PROFILING.md nominal x 0.75)"
+
+
+def job_flops(j):
+    if j.kernel == "matmul":
+        M, N, K = j.dims
+        return 2.0 * M * N * K
+    return None
+
+
 def load_traffic():
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
@@ -207,6 +225,25 @@ def oracle_sample_rate(jobs, min_seconds=1.0):
         elif j.kernel == "binomialoption":
             r = j.host_in[0][: 1 << 12]
             fn, units, what = (lambda: oracle.binomialoption(r)), r.size, "n=2^12"
+        elif j.kernel == "matmul":
+            # full-K dot products for a 128 x 128 block of C (units = C elements)
+            A, Bt = j.host_in[0], j.host_in[1]
+            M, N, K = j.dims
+            As = np.ascontiguousarray(A.reshape(M, K)[:128])
+            Bs = np.ascontiguousarray(Bt.reshape(N, K)[:128])
+            fn, units, what = (lambda: oracle.matmul_bf16(As, Bs)), 128 * 128, f"C[0:128,0:128] at K={K}"
+        elif j.kernel == "floydwarshall":
+            # the n'^3 relaxations of an n' = 512 sub-problem, converted to the
+            # full problem's units (n^3 relaxations per n nodes)
+            n = j.n
+            m = min(n, 512)
+            Wm = np.ascontiguousarray(j.host_in[0].reshape(n, n)[:m, :m])
+            fn, units, what = (lambda: oracle.floydwarshall(Wm)), m ** 3 / n ** 2, f"n'={m} sub-graph"
+        elif j.kernel == "dct":
+            H, W = j.dims
+            h = max(8, min(H, (1 << 22) // W) // 8 * 8)
+            X = np.ascontiguousarray(j.host_in[0].reshape(H, W)[:h])
+            fn, units, what = (lambda: oracle.dct8x8(X)), h * W, f"{h}x{W}"
         else:
             continue
         reps, t0 = 0, time.perf_counter()
@@ -356,6 +393,10 @@ def main():
             ms = per[(j.kernel, v)]
             gbs = j.alg_bytes / (ms * 1e-3) / 1e9
             d[v] = {"ms": round(ms, 4), "gbs": round(gbs, 1), "frac": round(gbs / peak, 4)}
+            if job_flops(j):
+                tf = job_flops(j) / (ms * 1e-3) / 1e12
+                d[v]["tflops"] = round(tf, 1)
+                d[v]["tensor_frac"] = round(tf / load_tensor_peak()[0], 4)
             if v != "none" and "none" in variants:
                 sd = ms / per[(j.kernel, "none")]
                 d[v]["slowdown"] = round(sd, 3)
@@ -379,6 +420,14 @@ def main():
                 "frac": round(ach / peak, 4), "traffic": traffic, "kernel": f"{dj.kernel}/{dv}",
                 "share_of_step": round(dms / (ms_total / args.steps), 3), "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": dj.alg_bytes}
+    if dj.bound == "tensor" and job_flops(dj):
+        tpk, tsrc = load_tensor_peak()
+        tach = job_flops(dj) / (dms * 1e-3) / 1e12
+        roofline.update({"bound": "tensor", "achieved": round(tach, 1), "peak": tpk, "unit": "TFLOP/s",
+                         "frac": round(tach / tpk, 4), "peak_source": tsrc,
+                         "algorithmic_flops_per_launch": job_flops(dj),
+                         "note": "both replicas run the full contraction on the tensor pipe; achieved counts "
+                                 "the algorithmic 2MNK once"})
     best_none = max((j for j in jobs if j.bound == "hbm"), key=lambda j: j.alg_bytes / per[(j.kernel, "none")],
                     default=None)
 

@@ -13,7 +13,7 @@ import os
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "librmt.so")
+LIB_PATH = os.environ.get("RMT_LIB") or os.path.join(_HERE, "librmt.so")  # RMT_LIB: experiment builds only
 
 KERNELS = {
     "blackscholes": 0, "binarysearch": 1, "fwt": 2, "prefixsum": 3, "reduction": 4,

@@ -160,6 +160,10 @@ def job_binomialoption(n, seed=12, rank=0):
 # ---------------------------------------------------------------- BASELINE.json configs
 
 def config_jobs(name: str, rank: int = 0):
+    if ":" in name:          # "<config>:<kernel>[,<kernel>]" -- a subset of a config (quick timing)
+        base, ks = name.split(":", 1)
+        keep = set(ks.split(","))
+        return [j for j in config_jobs(base, rank) if j.kernel in keep]
     if name == "suite":      # configs[1]: the APP SDK-style suite, "paper's sizes"
         return [job_binarysearch(1 << 26, 1 << 24, rank=rank), job_fwt(1 << 26, rank=rank),
                 job_prefixsum(1 << 26, rank=rank), job_reduction(1 << 26, rank=rank),
