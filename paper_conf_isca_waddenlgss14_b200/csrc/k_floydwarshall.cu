@@ -52,29 +52,57 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_init_kernel(FwArgs a, Ct
 }
 
 // One pass k.  Each logical thread handles VPT 16-B vectors strided by the CTA
-// width (coalesced); fat CTAs amortise the per-CTA RMT handshakes (inter-group
-// ticket / turn / queue latency) over 8192 elements.
-constexpr int VPT = 1;
+// width (coalesced), all loads in flight before the first use.  VPT per
+// variant, measured at n = 4096 (B200): none 4 (52 -> 40 ms), intra 2 (an
+// intra warp carries half the distinct bytes, so more vectors per thread),
+// inter 1 (larger inter CTAs were slower: 2 -> +5%, 8 -> 3.6x).
+#ifndef FW_VPT_INTER
+#define FW_VPT_INTER 1
+#endif
+#ifndef FW_VPT_INTRA
+#define FW_VPT_INTRA 2
+#endif
+#ifndef FW_VPT_NONE
+#define FW_VPT_NONE 4
+#endif
+template <int V>
+constexpr int fw_vpt() {
+  return (V == V_INTER || V == V_CLUSTER) ? FW_VPT_INTER : V == V_NONE ? FW_VPT_NONE : FW_VPT_INTRA;
+}
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ctx c) {
+  constexpr int VPT = fw_vpt<V>();
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned nn = a.n * a.n;
-#pragma unroll 1
+  // logical CTA = (row i, column chunk of BL*4*VPT words): the row and chunk
+  // are CTA-uniform (no per-thread division)
+  const unsigned cpr = (a.n + BL * 4 * VPT - 1) / (BL * 4 * VPT);
+  const unsigned i = (unsigned)rep.lblock / cpr;
+  const unsigned jc = ((unsigned)rep.lblock - i * cpr) * (BL * 4 * VPT);
+  const unsigned dik0 = a.D[(size_t)i * a.n + a.k];  // one broadcast word per CTA row
+  // all VPT vector pairs in flight before the first use (L2 latency-bound:
+  // an intra warp carries half the distinct bytes of an unprotected warp)
+  uint4 dkj[VPT], dij[VPT];
+#pragma unroll
   for (int it = 0; it < VPT; ++it) {
-    const unsigned e0 = ((unsigned)rep.lblock * (BL * VPT) + (unsigned)it * BL + (unsigned)rep.ltid) * 4;
-    const bool active = e0 < nn;
-    const unsigned i = active ? e0 / a.n : 0u, j = active ? e0 - i * a.n : 0u;
-    unsigned dik = 0;
-    uint4 dkj = make_uint4(0, 0, 0, 0), dij = make_uint4(0, 0, 0, 0);
-    if (active) {
-      dik = a.D[(size_t)i * a.n + a.k];
-      dkj = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
-      dij = *reinterpret_cast<const uint4*>(a.D + e0);
+    const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
+    dkj[it] = make_uint4(0, 0, 0, 0);
+    dij[it] = make_uint4(0, 0, 0, 0);
+    if (j < a.n) {
+      dkj[it] = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
+      dij[it] = *reinterpret_cast<const uint4*>(a.D + i * a.n + j);
     }
-    unsigned kj[4] = {dkj.x, dkj.y, dkj.z, dkj.w};
-    unsigned ij[4] = {dij.x, dij.y, dij.z, dij.w};
+  }
+#pragma unroll
+  for (int it = 0; it < VPT; ++it) {
+    const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
+    const bool active = j < a.n;
+    const unsigned e0 = i * a.n + j;
+    unsigned dik = dik0;
+    unsigned kj[4] = {dkj[it].x, dkj[it].y, dkj[it].z, dkj[it].w};
+    unsigned ij[4] = {dij[it].x, dij[it].y, dij[it].z, dij[it].w};
     if constexpr (M == M_FAULT) {
       dik = rep.fault(SITE_LOAD, (long long)i * a.n + a.k, dik);
 #pragma unroll
@@ -90,10 +118,10 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ct
       nd[q] = cand;
       np[q] = a.k;
     }
-    rep.template commit<4, 0>(mask, active ? e0 : 0u, nd, nn,
+    rep.template commit<4, 0, false, true>(mask, active ? e0 : 0u, nd, nn,
                               [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); },
                               /*defer=*/true);
-    rep.template commit<4, 1>(mask, active ? e0 : 0u, np, nn,
+    rep.template commit<4, 1, false, true>(mask, active ? e0 : 0u, np, nn,
                               [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
   }
   rep.finish();
@@ -118,14 +146,16 @@ namespace {
 int fw_issue(Launch& L) {
   const unsigned n = (unsigned)L.n;
   const unsigned nn = n * n;
-  const unsigned G = (nn / 4 + BL - 1) / BL;                // init: one vector per thread
-  const unsigned Gp = (nn / 4 + BL * VPT - 1) / (BL * VPT);  // passes: VPT vectors per thread
+  const unsigned G = (nn / 4 + BL - 1) / BL;  // init: one vector per thread
   FwArgs a{(unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, n, 0};
   // Fault element = k0 * n^2 + e: the pass k0 and the element e.
   const FaultDesc f = L.ctx.f;
   const unsigned k0 = (unsigned)(f.elem / nn);
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+    // passes: VPT vectors per thread (INFLATE runs the V_NONE kernel: its VPT)
+    const unsigned vpt = L.inflate ? (unsigned)fw_vpt<V_NONE>() : (unsigned)fw_vpt<V>();
+    const unsigned Gp = n * ((n + BL * 4 * vpt - 1) / (BL * 4 * vpt));  // rows x column chunks
     L.ctx.f.site = -1;  // the init pass carries no fault
     int rc = launch_std<V>(L, fw_init_kernel<V, M>, fw_init_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "fw/init");
     for (unsigned k = 0; k < n && rc == RMT_OK; ++k) {

@@ -446,7 +446,7 @@ struct Rep {
   //         DESIGN.md "Inter-Group queue").
   //   stride element distance between consecutive words (1: a contiguous vector;
   //         the store functor places word k at idx + k * stride)
-  template <int NW, int SID = 0, bool LIVE = false, class Store>
+  template <int NW, int SID = 0, bool LIVE = false, bool COND = false, class Store>
   __device__ __forceinline__ void commit(unsigned mask, unsigned idx, unsigned (&v)[NW], unsigned limit,
                                          Store&& store, bool defer = false, unsigned stride = 1) {
     static_assert(NW >= 1 && NW <= MAXW, "commit width");
@@ -496,20 +496,28 @@ struct Rep {
       bool have = true;  // consumer got the producer's record
       if constexpr (V == V_INTRA_REG || V == V_INTRA_NOLDS) {
         pk = __shfl_xor_sync(FULL, key, 1);
+        // COND (a conditional store site, e.g. FloydWarshall's improvements):
+        // values move only if some lane of the warp stores
+        if (!COND || __any_sync(FULL, mask != 0u)) {
 #pragma unroll
-        for (int k = 0; k < NW; ++k) pv[k] = __shfl_xor_sync(FULL, v[k], 1);
+          for (int k = 0; k < NW; ++k) pv[k] = __shfl_xor_sync(FULL, v[k], 1);
+        }
       } else if constexpr (V == V_INTRA_SMEM) {
         const int slot = lane >> 1;
+        // value words move only for the words a lane really stores;
+        // the key carries the predicate mask, so a word the consumer stores
+        // is compared only if the producer's key (same mask) matched
         if (!consumer) {
           mbox[slot] = key;
 #pragma unroll
-          for (int k = 0; k < NW; ++k) mbox[(1 + k) * 16 + slot] = v[k];
+          for (int k = 0; k < NW; ++k)
+            if ((mask >> k) & 1u) mbox[(1 + k) * 16 + slot] = v[k];
         }
         __syncwarp();
         if (consumer) {
           pk = mbox[slot];
 #pragma unroll
-          for (int k = 0; k < NW; ++k) pv[k] = mbox[(1 + k) * 16 + slot];
+          for (int k = 0; k < NW; ++k) pv[k] = ((mask >> k) & 1u) ? mbox[(1 + k) * 16 + slot] : 0u;
         }
         __syncwarp();
       } else if constexpr (V == V_CLUSTER) {  // DSMEM mailbox in the consumer CTA
@@ -523,12 +531,13 @@ struct Rep {
           }
           st_cl(pa, key);
 #pragma unroll
-          for (int k = 0; k < NW; ++k) st_cl(pa + (1 + k) * 32 * 4, v[k]);
+          for (int k = 0; k < NW; ++k)
+            if ((mask >> k) & 1u) st_cl(pa + (1 + k) * 32 * 4, v[k]);
         } else {
           have = spin_cl(fa, 1u, c, lane == 0);  // every lane acquires
           pk = ld_cl(pa);
 #pragma unroll
-          for (int k = 0; k < NW; ++k) pv[k] = ld_cl(pa + (1 + k) * 32 * 4);
+          for (int k = 0; k < NW; ++k) pv[k] = ((mask >> k) & 1u) ? ld_cl(pa + (1 + k) * 32 * 4) : 0u;
         }
       } else {  // V_INTER: per-(region, warp) queue of S records
         const size_t fi = slot_index(j);
@@ -544,7 +553,8 @@ struct Rep {
           }
           pl[lane] = key;
 #pragma unroll
-          for (int k = 0; k < NW; ++k) pl[(1 + k) * 32 + lane] = v[k];
+          for (int k = 0; k < NW; ++k)
+            if ((mask >> k) & 1u) pl[(1 + k) * 32 + lane] = v[k];  // only stored words move
           // The "ready" signal ("signals the work-item in the consumer") is
           // published by flush(): every lane fences its own payload stores (a
           // release by one lane does not order the other lanes' in-flight stores).
@@ -552,7 +562,7 @@ struct Rep {
           const bool ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
           pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
 #pragma unroll
-          for (int k = 0; k < NW; ++k) pv[k] = ld_relaxed(pl + (1 + k) * 32 + lane);
+          for (int k = 0; k < NW; ++k) pv[k] = ((mask >> k) & 1u) ? ld_relaxed(pl + (1 + k) * 32 + lane) : 0u;
           have = ok;
           // the buffer is freed only after every lane has consumed its words
           // (below, after the compare's warp ballot)
