@@ -102,12 +102,36 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c
 #pragma unroll
     for (int v = 0; v < 8; ++v) y[v] = xr == 0 ? __fmul_rn(cu, zz[v]) : __fmaf_rn(cu, zz[v], y[v]);
   }
-  const unsigned orow = by * 8 + u;
+  // Stores (measured per variant at 8192^2): none, intra_reg and intra_nolds
+  // first swap one 16-B half between output rows u and u^4 of a block through
+  // a shuffle, so that store h writes rows 4h..4h+3 of the warp's blocks as
+  // whole 128-B lines (lanes u < 4: half 0 of row 4h + u; lanes u >= 4: half 1
+  // of row 4h + u - 4) -- none 0.155 -> 0.145 ms, intra_reg 0.272 -> 0.253 ms;
+  // intra_smem and the inter variants were slower with it and store their own
+  // row u directly (8 rows of half-sectors per store).
+  constexpr bool XS = (V == V_NONE || V == V_INTRA_REG || V == V_INTRA_NOLDS);
+  const bool lowu = u < 4;
+  unsigned got[4];
+  if constexpr (XS) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) got[q] = rep.lshfl_xor(__float_as_uint(lowu ? y[4 + q] : y[q]), 4);
+  }
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
-    unsigned w[4] = {__float_as_uint(y[4 * h]), __float_as_uint(y[4 * h + 1]), __float_as_uint(y[4 * h + 2]),
-                     __float_as_uint(y[4 * h + 3])};
-    const unsigned idx = orow * a.W + col0 + 4 * h;
+    unsigned w[4];
+    unsigned orow, idx;
+    if constexpr (XS) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q)
+        w[q] = lowu ? (h == 0 ? __float_as_uint(y[q]) : got[q]) : (h == 0 ? got[q] : __float_as_uint(y[4 + q]));
+      orow = by * 8 + (lowu ? (unsigned)u + 4u * h : (unsigned)u - 4u + 4u * h);
+      idx = orow * a.W + col0 + (lowu ? 0u : 4u);
+    } else {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) w[q] = __float_as_uint(y[4 * h + q]);
+      orow = by * 8 + u;
+      idx = orow * a.W + col0 + 4 * h;
+    }
     rep.template commit<4, 0>(active ? 0xFu : 0u, active ? idx : 0u, w, a.H * a.W,
                               [&](unsigned i, unsigned m, const unsigned* v) {
                                 if (m == 0xFu)
