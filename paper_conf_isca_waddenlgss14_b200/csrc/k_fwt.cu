@@ -38,6 +38,55 @@ struct Swz {
   }
 };
 
+// Radix-2^NB butterfly network on registers, stages h = 1, 2, .., 2^(NB-1)
+// (the normative stage order, R-FWT2).  Two butterflies of a stage share one
+// packed FADD2 for the sums and one for the differences (add/sub.rn.f32x2:
+// lane-wise RN(a + b), RN(a - b), bit-identical to __fadd_rn / __fsub_rn),
+// halving the FP instructions of the issue-bound RMT variants.
+__device__ __forceinline__ unsigned long long f2pack(float lo, float hi) {
+  unsigned long long r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+  return r;
+}
+__device__ __forceinline__ void f2unpack(unsigned long long v, float& lo, float& hi) {
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(lo), "=f"(hi) : "l"(v));
+}
+template <int NB>
+__device__ __forceinline__ void butterflies(float (&v)[1 << NB]) {
+  constexpr int G = 1 << NB;
+  if constexpr (NB == 1) {
+    const float x0 = v[0], x1 = v[1];
+    v[0] = __fadd_rn(x0, x1);
+    v[1] = __fsub_rn(x0, x1);
+  } else {
+    // P[j] = {v[j], v[j + G/2]}: stages h < G/2 act on both halves alike, so
+    // they run on the packed pairs with the natural pairing (no register
+    // shuffling between stages); the last stage (h = G/2) is lo +- hi
+    constexpr int H = G / 2;
+    unsigned long long P[H];
+#pragma unroll
+    for (int j = 0; j < H; ++j) P[j] = f2pack(v[j], v[j + H]);
+#pragma unroll
+    for (int s = 0; s < NB - 1; ++s) {
+      const int h = 1 << s;
+#pragma unroll
+      for (int j = 0; j < H; ++j) {
+        if (j & h) continue;
+        const unsigned long long x0 = P[j], x1 = P[j + h];
+        asm("add.rn.f32x2 %0, %1, %2;" : "=l"(P[j]) : "l"(x0), "l"(x1));
+        asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(P[j + h]) : "l"(x0), "l"(x1));
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < H; ++j) {
+      float lo, hi;
+      f2unpack(P[j], lo, hi);
+      v[j] = __fadd_rn(lo, hi);
+      v[j + H] = __fsub_rn(lo, hi);
+    }
+  }
+}
+
 struct FwtArgs {
   const float* src;
   float* dst;
@@ -91,17 +140,7 @@ __device__ __forceinline__ void fwt_round(const R& rep, float* tp, int q, int te
           v[k] = rep.faultf(SITE_SMEM, (long long)gindex(a, tileid, ebase | (k << q)), v[k]);
       }
     }
-#pragma unroll
-    for (int s = 0; s < NB; ++s) {
-      const int h = 1 << s;
-#pragma unroll
-      for (int k = 0; k < G; ++k) {
-        if (k & h) continue;
-        const float x0 = v[k], x1 = v[k + h];
-        v[k] = __fadd_rn(x0, x1);
-        v[k + h] = __fsub_rn(x0, x1);
-      }
-    }
+    butterflies<NB>(v);
     unsigned vw[G];
 #pragma unroll
     for (int k = 0; k < G; ++k) {
@@ -141,17 +180,7 @@ __device__ __forceinline__ void fwt_round_ct(const R& rep, float* tp, const FwtA
           v[k] = rep.faultf(SITE_SMEM, (long long)gindex(a, tileid, ebase | (k << Q)), v[k]);
       }
     }
-#pragma unroll
-    for (int s = 0; s < NB; ++s) {
-      const int h = 1 << s;
-#pragma unroll
-      for (int k = 0; k < G; ++k) {
-        if (k & h) continue;
-        const float x0 = v[k], x1 = v[k + h];
-        v[k] = __fadd_rn(x0, x1);
-        v[k + h] = __fsub_rn(x0, x1);
-      }
-    }
+    butterflies<NB>(v);
     unsigned vw[G];
 #pragma unroll
     for (int k = 0; k < G; ++k) {
@@ -315,20 +344,6 @@ constexpr int P1_PLANE = P1_WORDS + 16;
 __device__ __forceinline__ constexpr int p1_phys(int e) { return e + 4 * (e >> 7); }
 __device__ __forceinline__ int p1x(int e) { return e ^ ((e >> 5) & 31); }
 
-template <int NB>
-__device__ __forceinline__ void butterflies(float (&v)[1 << NB]) {
-#pragma unroll
-  for (int s = 0; s < NB; ++s) {
-    const int h = 1 << s;
-#pragma unroll
-    for (int k = 0; k < (1 << NB); ++k) {
-      if (k & h) continue;
-      const float x0 = v[k], x1 = v[k + h];
-      v[k] = __fadd_rn(x0, x1);
-      v[k + h] = __fsub_rn(x0, x1);
-    }
-  }
-}
 
 template <int V, int M>
 __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, Ctx c) {
