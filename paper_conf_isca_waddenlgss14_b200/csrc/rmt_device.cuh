@@ -207,6 +207,13 @@ struct Rep {
   // Must be called by every thread of the CTA, first thing (may __syncthreads).
   // mbox_smem: MBOX_WORDS * (blockDim/32) words of shared memory (intra_smem only).
   __device__ __forceinline__ void init(unsigned* mbox_smem = nullptr) {
+    // Programmatic dependent launch (launch_std sets the attribute): this
+    // grid may be scheduled while the previous kernel on the stream drains;
+    // wait for it to complete (and its memory to be visible) before touching
+    // global memory or the inter ticket, then let the next kernel's CTAs be
+    // scheduled as this grid's CTAs retire.  No-ops without the attribute.
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     lane = threadIdx.x & 31;
     warp = threadIdx.x >> 5;
     if constexpr (INTRA) {

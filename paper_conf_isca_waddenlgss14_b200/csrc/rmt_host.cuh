@@ -11,6 +11,10 @@
 
 namespace rmt {
 
+#ifndef RMT_PDL
+#define RMT_PDL 1  // programmatic dependent launch between the library's kernels
+#endif
+
 // Inter-group queue geometry.
 constexpr int INTER_R = 1024;  // regions (> resident pairs, so a region is rarely waited for)
 constexpr int INTER_S = 8;     // slots (records in flight) per (region, warp)
@@ -165,18 +169,33 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
     cfg.blockDim = dim3(Geom<V>::block(BL));
     cfg.dynamicSmemBytes = dyn;
     cfg.stream = L.stream;
-    cudaLaunchAttribute at[1];
+    cudaLaunchAttribute at[2];
     at[0].id = cudaLaunchAttributeClusterDimension;
     at[0].val.clusterDim.x = 2;  // the replica pair
     at[0].val.clusterDim.y = 1;
     at[0].val.clusterDim.z = 1;
+    at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[1].val.programmaticStreamSerializationAllowed = RMT_PDL;
     cfg.attrs = at;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = 2;
     cudaError_t e = cudaLaunchKernelEx(&cfg, kr, a, c);
     if (e != cudaSuccess) return cuda_check(e, what);
   } else {
     if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    kr<<<Geom<V>::grid(G), Geom<V>::block(BL), smem, L.stream>>>(a, c);
+    // programmatic dependent launch: the grid is scheduled while the previous
+    // kernel drains; Rep::init waits (griddepcontrol.wait) before any access
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(Geom<V>::grid(G));
+    cfg.blockDim = dim3(Geom<V>::block(BL));
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = L.stream;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = RMT_PDL;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kr, a, c);
+    if (e != cudaSuccess) return cuda_check(e, what);
   }
   L.launches += 1;
   return cuda_check(cudaGetLastError(), what);
