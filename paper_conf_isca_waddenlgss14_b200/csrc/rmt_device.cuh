@@ -48,7 +48,10 @@ constexpr unsigned long long WATCHDOG_CYCLES = 1ull << 32;  // ~2 s at 2 GHz
 // (Ctx::S, a power of two chosen by the launcher): 8 lets the producer fill one
 // deferred batch (<= 4 records) while the consumer drains the previous one; 4
 // when a larger mailbox would cost occupancy (CTAs of more than 4 warps).
-constexpr int CL_S_SMALL = 4, CL_S_LARGE = 8;
+#ifndef RMT_CL_S_LARGE
+#define RMT_CL_S_LARGE 8
+#endif
+constexpr int CL_S_SMALL = 4, CL_S_LARGE = RMT_CL_S_LARGE;
 
 struct FaultDesc {
   int replica, site, bit, sid;

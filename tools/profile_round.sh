@@ -12,14 +12,25 @@ timeout 600 python bench.py > $out/bench.log 2>&1; grep '^{' $out/bench.log | ta
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $out/launches.csv \
   python bench.py --steps 2 --warmup 1 --no-cpu-baseline --e2e-steps 0 --energy-seconds 0 --extra-variants "" \
   > $out/launches_bench.log 2>&1
-for kv in "binarysearch bins_kernel" "fwt fwt_kernel" "prefixsum ps_scan_kernel" "reduction red_partial_kernel" \
-          "transpose tr_kernel" "sobel sobel_kernel"; do
+# cfg kernel capture-name kernel-regex skip
+for kv in "suite binarysearch binarysearch bins_kernel 1" "suite fwt fwt_p1 fwt_p1_kernel 1" "suite fwt fwt_ps fwt_ps_kernel 1" \
+          "suite prefixsum prefixsum ps_scan_kernel 1" "suite reduction reduction red_partial_kernel 1" \
+          "suite transpose transpose tr_kernel 1" "suite sobel sobel sobel_kernel 1" \
+          "fwdct dct dct dct_kernel 1" "fwdct floydwarshall fw_pass fw_pass_kernel 300"; do
   set -- $kv
   for vv in "none 0" "intra_smem 1" "intra_reg 2" "inter_group 3"; do
     set -- $kv $vv
-    timeout 200 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
-      -k "regex:$2<.int.$4, .int.0" -s 1 -c 1 -o $out/full/$1_$3 \
-      python tools/prof_run.py suite $1 $3 2 > $out/full/$1_$3.log 2>&1
+    reps=2; [ "$2" = floydwarshall ] && reps=1
+    timeout 300 ncu --set full --clock-control none --import-source on --kernel-name-base demangled \
+      -k "regex:$4<.int.$7, .int.0" -s $5 -c 1 -o $out/full/$3_$6 \
+      python tools/prof_run.py $1 $2 $6 $reps > $out/full/$3_$6.log 2>&1
   done
 done
 ls -la $out $out/full
+# summarise on the box (the .ncu-rep files together exceed gpurun's 64 MiB
+# copy-back limit); keep the dominant kernel's report only
+python tools/ncu_summary.py $out/full/*.ncu-rep --json $out/ncu_full_summary.json > $out/ncu_full_summary.txt 2>&1
+mkdir -p $out/keep
+mv $out/full/binarysearch_inter_group.ncu-rep $out/keep/ 2>/dev/null
+rm -f $out/full/*.ncu-rep
+du -sh $out
