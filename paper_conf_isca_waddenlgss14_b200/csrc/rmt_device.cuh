@@ -141,6 +141,12 @@ __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+#ifndef RMT_SPIN_NS0
+#define RMT_SPIN_NS0 32     // first back-off sleep of a queue wait (0: pure spin)
+#endif
+#ifndef RMT_SPIN_NSMAX
+#define RMT_SPIN_NSMAX 512  // back-off cap
+#endif
 // Spin until *p == want (acquire), with back-off and a watchdog that converts a
 // hang (a fault that desynchronised a pair) into err+1 and a sticky flag.
 // Every thread that will touch the guarded data must do its own acquire: a lane
@@ -148,11 +154,11 @@ __device__ __forceinline__ void cluster_sync_all() {
 __device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, const Ctx& c, bool count = true) {
   if (ld_acquire(p) == want) return true;
   unsigned long long t0 = clock64();
-  unsigned ns = 32;
+  unsigned ns = RMT_SPIN_NS0;
   while (true) {
-    __nanosleep(ns);
+    if (ns) __nanosleep(ns);
     if (ld_acquire(p) == want) return true;
-    if (ns < 512) ns <<= 1;
+    if (ns && ns < RMT_SPIN_NSMAX) ns <<= 1;
     if (clock64() - t0 > WATCHDOG_CYCLES) {
       if (count) {
         atomicAdd(c.err, 1ull);
