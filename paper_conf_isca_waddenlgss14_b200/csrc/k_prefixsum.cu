@@ -61,7 +61,12 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_reduce_kernel(PsArgs a, 
   const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
   unsigned s = 0;
   // 16-B coalesced loads, 4 in flight per thread (chunk starts are 16-B aligned)
-  for (unsigned e = lo + 4 * rep.ltid; e < hi; e += 4 * BL * 4) {
+  // blocks of 16 BL elements visited from the END of the chunk: the scan pass
+  // reads each chunk from its start, which is then what L2 still holds
+  const unsigned nblk = hi > lo ? (hi - lo + 16 * BL - 1) / (16 * BL) : 0u;
+#pragma unroll 1
+  for (unsigned b = nblk; b-- > 0;) {
+    const unsigned e = lo + b * 16 * BL + 4 * rep.ltid;
     uint4 v[4];
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
@@ -98,12 +103,23 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_reduce_kernel(PsArgs a, 
 }
 
 template <int V, int M>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ctx c) {
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   constexpr int LW = 32 / DUP;
   constexpr int NLW = BL / LW;
+  // none / inter (32-lane logical warps): NQ = 4 sub-tiles of 4 BL elements, a
+  // thread owning 4 consecutive elements of each (coalesced 16-B accesses, one
+  // 512-B line per warp instruction; with 16 consecutive elements per thread
+  // every access touched twice the sectors and L1 ran at 80%: 0.168 -> 0.135 ms
+  // at 2^26).  Intra (16-lane logical warps): one run of 16 per thread -- its
+  // accesses are 256 B per instruction either way, and 4 scan chains cost more
+  // shuffles than they save (measured: intra_reg 0.18 -> 0.195 ms).
+  constexpr int NQ = DUP == 1 ? ITEMS / 4 : 1;  // sub-tiles per tile
+  constexpr int RUN = ITEMS / NQ;                // consecutive elements per thread and sub-tile
+  constexpr unsigned SUB = RUN * BL;             // elements per sub-tile
+  constexpr bool FLAT = NQ * NLW == LW;          // every (sub-tile, warp) total on its own lane
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
-  __shared__ unsigned sw[NLW * Geom<V>::SMDUP];
+  __shared__ unsigned sw[NQ * NLW * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
   const unsigned ch = a.nch - 1u - (unsigned)rep.lblock;  // reverse order: L2-hot chunks first
@@ -113,65 +129,107 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ct
   unsigned carry = a.carry_in + block_sum_u32(rep, cs, sw);
   const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
   const int lw = rep.ltid / LW;
-  // register double buffer: the next tile's loads are in flight while this
-  // tile is scanned and stored
+  // Register double buffer: the next tile's loads are in flight while this
+  // tile is scanned and stored.  v[q * RUN + k] = x[t0 + q SUB + ltid RUN + k].
   auto load_tile = [&](unsigned t0, unsigned (&v)[ITEMS]) {
-    const unsigned base = t0 + (unsigned)rep.ltid * ITEMS;
-    if (base + ITEMS <= hi) {
 #pragma unroll
-      for (int q = 0; q < ITEMS / 4; ++q) {
-        uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.x + base) + q);
-        v[4 * q] = w.x; v[4 * q + 1] = w.y; v[4 * q + 2] = w.z; v[4 * q + 3] = w.w;
+    for (int q = 0; q < NQ; ++q) {
+      const unsigned e = t0 + q * SUB + RUN * (unsigned)rep.ltid;
+      if (e + RUN <= hi) {
+#pragma unroll
+        for (int j = 0; j < RUN / 4; ++j) {
+          uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.x + e) + j);
+          v[q * RUN + 4 * j] = w.x; v[q * RUN + 4 * j + 1] = w.y;
+          v[q * RUN + 4 * j + 2] = w.z; v[q * RUN + 4 * j + 3] = w.w;
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < RUN; ++k) v[q * RUN + k] = e + k < hi ? a.x[e + k] : 0u;
       }
-    } else {
-#pragma unroll
-      for (int i = 0; i < ITEMS; ++i) v[i] = base + i < hi ? a.x[base + i] : 0u;
     }
   };
   unsigned nxt[ITEMS];
   if (lo < hi) load_tile(lo, nxt);
 #pragma unroll 1
   for (unsigned t0 = lo; t0 < hi; t0 += TILE) {  // uniform trip count per CTA
-    const unsigned base = t0 + (unsigned)rep.ltid * ITEMS;
     unsigned v[ITEMS];
 #pragma unroll
     for (int i = 0; i < ITEMS; ++i) v[i] = nxt[i];
     if (t0 + TILE < hi) load_tile(t0 + TILE, nxt);
     if constexpr (M == M_FAULT) {
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i) v[i] = rep.fault(SITE_LOAD, (long long)base + i, v[i]);
+      for (int i = 0; i < ITEMS; ++i)
+        v[i] = rep.fault(SITE_LOAD, (long long)t0 + (i / RUN) * SUB + RUN * rep.ltid + (i % RUN), v[i]);
+    }
+    unsigned tsum[NQ], ws[NQ];
+#pragma unroll
+    for (int q = 0; q < NQ; ++q) {  // thread-local inclusive scans
+#pragma unroll
+      for (int k = 1; k < RUN; ++k) v[q * RUN + k] += v[q * RUN + k - 1];
+      tsum[q] = ws[q] = v[q * RUN + RUN - 1];
     }
 #pragma unroll
-    for (int i = 1; i < ITEMS; ++i) v[i] += v[i - 1];  // thread-local inclusive scan
-    const unsigned tsum = v[ITEMS - 1];
-    unsigned ws = tsum;  // logical-warp inclusive scan of thread totals
+    for (int d = 1; d < LW; d <<= 1) {  // logical-warp scans, NQ independent chains
 #pragma unroll
-    for (int d = 1; d < LW; d <<= 1) {
-      const unsigned u = rep.lshfl_up(ws, d);
-      if (rep.llane >= d) ws += u;
+      for (int q = 0; q < NQ; ++q) {
+        const unsigned u = rep.lshfl_up(ws[q], d);
+        if (rep.llane >= d) ws[q] += u;
+      }
     }
-    if (rep.llane == LW - 1 && rep.sts_ok1(ws, lw)) rep.sm(sw, lw) = ws;
+#pragma unroll
+    for (int q = 0; q < NQ; ++q)  // warp totals, sub-tile-major
+      if (rep.llane == LW - 1 && rep.sts_ok1(ws[q], q * NLW + lw)) rep.sm(sw, q * NLW + lw) = ws[q];
     __syncthreads();
-    unsigned wt = rep.llane < NLW ? rep.sm(sw, rep.llane) : 0u;  // every warp scans the warp totals
-    if constexpr (M == M_FAULT) wt = rep.fault(SITE_SMEM, (long long)ch * BL + rep.llane * LW, wt);
-    unsigned winc = wt;
+    unsigned pre[NQ];  // exclusive prefix of this thread's sub-tile-q run within the tile
+    unsigned total;
+    if constexpr (FLAT) {
+      // lane l holds total l = (sub-tile l / NLW, warp l % NLW): one scan over the lanes
+      unsigned wt = rep.sm(sw, rep.llane);
+      if constexpr (M == M_FAULT) wt = rep.fault(SITE_SMEM, (long long)ch * BL + rep.llane, wt);
+      unsigned winc = wt;
 #pragma unroll
-    for (int d = 1; d < NLW; d <<= 1) {
-      const unsigned u = rep.lshfl_up(winc, d);
-      if (rep.llane >= d) winc += u;
+      for (int d = 1; d < LW; d <<= 1) {
+        const unsigned u = rep.lshfl_up(winc, d);
+        if (rep.llane >= d) winc += u;
+      }
+      const unsigned wex = winc - wt;
+#pragma unroll
+      for (int q = 0; q < NQ; ++q) pre[q] = rep.lshfl_idx(wex, q * NLW + lw);
+      total = rep.lshfl_idx(winc, LW - 1);
+    } else {
+      unsigned wt[NQ], winc[NQ];
+#pragma unroll
+      for (int q = 0; q < NQ; ++q) {
+        wt[q] = rep.llane < NLW ? rep.sm(sw, q * NLW + rep.llane) : 0u;
+        if constexpr (M == M_FAULT) wt[q] = rep.fault(SITE_SMEM, (long long)ch * BL + q * NLW + rep.llane, wt[q]);
+        winc[q] = wt[q];
+      }
+#pragma unroll
+      for (int d = 1; d < NLW; d <<= 1) {
+#pragma unroll
+        for (int q = 0; q < NQ; ++q) {
+          const unsigned u = rep.lshfl_up(winc[q], d);
+          if (rep.llane >= d) winc[q] += u;
+        }
+      }
+      total = 0;
+#pragma unroll
+      for (int q = 0; q < NQ; ++q) {
+        pre[q] = total + rep.lshfl_idx(winc[q] - wt[q], lw);
+        total += rep.lshfl_idx(winc[q], NLW - 1);
+      }
     }
-    const unsigned wexcl = rep.lshfl_idx(winc - wt, lw);
-    const unsigned total = rep.lshfl_idx(winc, NLW - 1);
     __syncthreads();  // sw is reused by the next tile
-    const unsigned prefix = carry + wexcl + (ws - tsum);
 #pragma unroll
-    for (int q = 0; q < ITEMS / 4; ++q) {
-      const unsigned e0 = base + 4 * q;
+    for (int i = 0; i < ITEMS / 4; ++i) {
+      const int q = (4 * i) / RUN;
+      const unsigned e0 = t0 + q * SUB + RUN * (unsigned)rep.ltid + (4 * i) % RUN;
+      const unsigned prefix = carry + pre[q] + (ws[q] - tsum[q]);
       unsigned w[4];
       unsigned mask = 0;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
-        w[k] = prefix + v[4 * q + k];
+        w[k] = prefix + v[4 * i + k];
         mask |= (e0 + k < hi ? 1u : 0u) << k;
       }
       rep.template commit<4, 0>(mask, mask ? e0 : 0u, w, a.n, [&](unsigned idx, unsigned m, const unsigned* x) {
@@ -179,7 +237,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ct
         else
           for (int k = 0; k < 4; ++k)
             if ((m >> k) & 1u) a.y[idx + k] = x[k];
-      }, /*defer=*/q < ITEMS / 4 - 1);
+      }, /*defer=*/i < ITEMS / 4 - 1);
     }
     carry += total;
   }
