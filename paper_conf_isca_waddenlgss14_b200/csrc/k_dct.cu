@@ -28,6 +28,7 @@ struct DctArgs {
   float* Y;
   unsigned H, W;
   unsigned nbx;  // logical CTAs across a row strip
+  unsigned v8;   // X is 32-B aligned: 256-bit row loads
   float C[8][8];
 };
 
@@ -49,9 +50,16 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c
   const unsigned row = by * 8 + r;
   float x[8];
   if (active) {
-    const float4* src = reinterpret_cast<const float4*>(a.X + (size_t)row * a.W + col0);
-    float4 p = __ldcs(src), q = __ldcs(src + 1);
-    x[0] = p.x; x[1] = p.y; x[2] = p.z; x[3] = p.w; x[4] = q.x; x[5] = q.y; x[6] = q.z; x[7] = q.w;
+    if (a.v8) {  // one 256-bit load: the warp's 1 KiB row segment in whole lines
+      unsigned w[8];
+      ldcs8(a.X + (size_t)row * a.W + col0, w);
+#pragma unroll
+      for (int y = 0; y < 8; ++y) x[y] = __uint_as_float(w[y]);
+    } else {  // X only 16-B aligned (the ABI minimum)
+      const float4* src = reinterpret_cast<const float4*>(a.X + (size_t)row * a.W + col0);
+      float4 p = __ldcs(src), q = __ldcs(src + 1);
+      x[0] = p.x; x[1] = p.y; x[2] = p.z; x[3] = p.w; x[4] = q.x; x[5] = q.y; x[6] = q.z; x[7] = q.w;
+    }
   } else {
 #pragma unroll
     for (int y = 0; y < 8; ++y) x[y] = 0.0f;
@@ -170,6 +178,7 @@ int dct_run(Launch& L) {
   a.H = H;
   a.W = W;
   a.nbx = nbx;
+  a.v8 = ((uintptr_t)a.X % 32) == 0 ? 1u : 0u;
   for (int u = 0; u < 8; ++u)  // C[u][x] = alpha(u) cos((2x+1) u pi / 16), in fp64 then rounded
     for (int x = 0; x < 8; ++x)
       a.C[u][x] = (float)((u == 0 ? sqrt(0.125) : 0.5) * cos((2.0 * x + 1.0) * u * 3.14159265358979323846 / 16.0));

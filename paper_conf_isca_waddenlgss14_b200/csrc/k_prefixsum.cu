@@ -32,6 +32,7 @@ struct PsArgs {
   unsigned chunk;      // elements per chunk (multiple of TILE)
   unsigned nch;        // chunks actually used
   unsigned carry_in;   // added to every output (multi-GPU shard offset)
+  unsigned v8;         // x is 32-B aligned: 256-bit loads where a thread's run allows
 };
 
 // u32 sum over the logical CTA (logical warps + duplicated smem)
@@ -136,11 +137,21 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_k
     for (int q = 0; q < NQ; ++q) {
       const unsigned e = t0 + q * SUB + RUN * (unsigned)rep.ltid;
       if (e + RUN <= hi) {
+        if (RUN % 8 == 0 && a.v8) {  // 256-bit loads: 32 B per lane, whole lines per instruction
 #pragma unroll
-        for (int j = 0; j < RUN / 4; ++j) {
-          uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.x + e) + j);
-          v[q * RUN + 4 * j] = w.x; v[q * RUN + 4 * j + 1] = w.y;
-          v[q * RUN + 4 * j + 2] = w.z; v[q * RUN + 4 * j + 3] = w.w;
+          for (int j = 0; j < RUN / 8; ++j) {
+            unsigned w[8];
+            ldcs8(a.x + e + 8 * j, w);
+#pragma unroll
+            for (int k = 0; k < 8; ++k) v[q * RUN + 8 * j + k] = w[k];
+          }
+        } else {
+#pragma unroll
+          for (int j = 0; j < RUN / 4; ++j) {
+            uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.x + e) + j);
+            v[q * RUN + 4 * j] = w.x; v[q * RUN + 4 * j + 1] = w.y;
+            v[q * RUN + 4 * j + 2] = w.z; v[q * RUN + 4 * j + 3] = w.w;
+          }
         }
       } else {
 #pragma unroll
@@ -264,7 +275,7 @@ int prefixsum_run(Launch& L) {
   const unsigned chunk = tiles_per_chunk * TILE;
   const unsigned nch = (n + chunk - 1) / chunk;
   PsArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, (unsigned*)L.scratch, n, chunk, nch,
-           (unsigned)(L.bufs->dims[0] & 0xFFFFFFFFu)};
+           (unsigned)(L.bufs->dims[0] & 0xFFFFFFFFu), ((uintptr_t)L.bufs->buf[0].ptr % 32) == 0 ? 1u : 0u};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     int rc = launch_std<V>(L, ps_reduce_kernel<V, M>, ps_reduce_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a,

@@ -101,6 +101,14 @@ __device__ __forceinline__ uint4 ldg4(const void* p) { return __ldg(reinterpret_
 __device__ __forceinline__ void stg4(void* p, uint4 v) { *reinterpret_cast<uint4*>(p) = v; }
 __device__ __forceinline__ uint4 ldcs4(const void* p) { return __ldcs(reinterpret_cast<const uint4*>(p)); }
 __device__ __forceinline__ void stcs4(void* p, uint4 v) { __stcs(reinterpret_cast<uint4*>(p), v); }
+// 256-bit streaming load (sm_100 LDG.256, evict-first): lanes 32 B apart cover
+// whole 128-B lines with one instruction, where two 16-B loads each touch
+// every line of the span half-used (twice the L1 wavefronts)
+__device__ __forceinline__ void ldcs8(const void* p, unsigned (&w)[8]) {
+  asm volatile("ld.global.cs.v8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+               : "l"(p));
+}
 
 // ---- thread-block-cluster / distributed shared memory (inter_cluster)
 __device__ __forceinline__ unsigned cluster_ctarank() {

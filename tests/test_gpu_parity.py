@@ -6,7 +6,7 @@ import pytest
 import torch
 
 from paper_conf_isca_waddenlgss14_b200 import rmt
-from cases import Case, small_cases
+from cases import DCT, Case, PrefixSum, small_cases
 from helpers import VARIANTS, run
 
 pytestmark = pytest.mark.gpu
@@ -96,7 +96,7 @@ def test_fault_is_live_in_none(case):
     assert any(not np.array_equal(a, b) for a, b in zip(outs, ref))
 
 
-@pytest.mark.parametrize("variant", ["none"] + list(rmt.RMT_VARIANTS))
+@pytest.mark.parametrize("variant", sorted(set(["none", *rmt.RMT_VARIANTS])))
 def test_prefixsum_carry_in(variant):
     """The multi-GPU shard offset (dims[0] = carry-in) is added to every output."""
     import oracle
@@ -117,3 +117,25 @@ def test_cluster_placement_probe():
     same = rmt.probe_cluster_placement(pairs)
     assert 0 <= same <= pairs
     print(f"cluster pairs sharing an SM: {same}/{pairs}")
+
+
+@pytest.mark.parametrize("variant", sorted(set(["none", *rmt.RMT_VARIANTS])))
+@pytest.mark.parametrize("make", [lambda: PrefixSum(4096 * 9 + 5), lambda: DCT(32, 264)], ids=["prefixsum", "dct"])
+def test_input_only_16byte_aligned(make, variant):
+    """DCT and PrefixSum take 256-bit loads when the input is 32-B aligned and
+    16-B loads otherwise (the ABI minimum is 16 B): an input placed 16 B past a
+    32-B boundary must give the same bits, against the oracle."""
+    from helpers import dev
+
+    case = make()
+    b = case.buffers()
+    src = b[0].reshape(-1)
+    pad = torch.empty(src.numel() + 8, dtype=src.dtype, device="cuda")
+    assert pad.data_ptr() % 32 == 0
+    shifted = pad[4: 4 + src.numel()]
+    assert shifted.data_ptr() % 32 == 16
+    shifted.copy_(src)
+    b[0] = shifted.view(b[0].shape)
+    err = run(case.kernel, variant, b, case.n, case.dims)
+    assert err == 0
+    case.check(case.outputs(b))
