@@ -113,7 +113,9 @@ typedef struct {
 } rmt_buf_t;
 
 /* Buffer schema per kernel (n = logical units; dims as listed, others 0):
- *   BLACKSCHOLES  buf {r:F32[n], call:F32[n], put:F32[n]}           n = options
+ *   BLACKSCHOLES  buf {r:F32[n], call:F32[n], put:F32[n]}           n = options, dims {mode}
+ *                 mode 0: one draw r per option, (S,K,T,R,sigma) from r with S == K (DESIGN.md R-BS1)
+ *                 mode 1: buf[0] = params:F32[5n], planes S | K | T | R | sigma, n%4 = 0 (R-BS4)
  *   BINARYSEARCH  buf {A:U32[N] sorted, q:U32[Q], idx:U32[Q]}       n = Q, dims {N, Q}
  *   FWT           buf {x:F32[N], y:F32[N]}                          n = N = 2^m
  *   PREFIXSUM     buf {x:U32[n], y:U32[n]}  inclusive, mod 2^32     n, dims {carry_in} (u32 added
@@ -133,7 +135,11 @@ typedef struct {
  *   BINOMIALOPTION buf {r:F32[n], call:F32[n]}                      n = options <= 2^28
  *                 CRR European call, 254 steps, R = 0.02, sigma = 0.30, (S, K, T) from r
  *                 (DESIGN.md R-BO1/2)
- * Vector-committed buffers must have < 2^30 elements.
+ * Commit key: every storing commit compares the FULL
+ * 32-bit element index and the store predicate of both replicas, key = idx ^
+ * (mask << 28) for vector commits (idx for scalar ones); vector-committed
+ * buffers must have < 2^30 elements (so that no storing key equals the
+ * non-storing key 0xFFFFFFFF under a one-bit predicate fault).
  */
 typedef struct {
     rmt_buf_t buf[6];
@@ -149,6 +155,7 @@ typedef struct {
 #define RMT_EWORKSPACE (-3)   /* workspace NULL or smaller than rmt_workspace_size() */
 #define RMT_ECUDA (-4)        /* CUDA launch/copy error; detail in rmt_last_error() */
 #define RMT_ENODEV (-5)       /* no sm_100 device */
+#define RMT_EWATCHDOG (-6)    /* rmt_workspace_status: an inter-group launch hit the watchdog */
 
 /*
  * rmt_launch -- run kernel `kernel` under RMT variant `variant`, asynchronously
@@ -211,6 +218,42 @@ int rmt_clear_faults(void);
 #define RMT_ABL_NOCOMM 1
 #define RMT_ABL_INFLATE 2
 int rmt_set_ablation(int mode);
+
+/*
+ * rmt_workspace_status -- report (and clear) the inter-group queue's sticky
+ * watchdog flag.  The queue waits are bounded: a replica that waits longer than
+ * the watchdog bound for its partner (a fault that desynchronised the pair, or a
+ * lost producer) gives up, adds 1 to *err_count, suppresses the affected stores
+ * and sets a sticky flag in the workspace ("a watchdog-aborted
+ * inter-group pair adds to err_count and sets a sticky flag that rmt_last_error
+ * reports"); the launch's last CTA then clears every queue slot so the
+ * workspace stays reusable.  This call reads the flag (synchronising `stream`):
+ * RMT_OK if clear (or for any variant other than RMT_INTER_GROUP, whose queue
+ * lives in the workspace); RMT_EWATCHDOG if it was set -- the flag is then
+ * cleared and rmt_last_error() describes the event.
+ */
+int rmt_workspace_status(int variant, void* workspace, void* stream);
+
+/*
+ * rmt_set_stress -- queue-protocol stress configuration for the inter variants
+ * (test use; SURVEY 8(c) "C-Q inter-group ring" pins).  While depth > 0 or
+ * flags != 0, RMT_INTER_GROUP / RMT_INTER_CLUSTER launches run the STRESS
+ * instantiation:
+ *   depth           queue slots per (pair, warp) in use: 1, 2, 4 or 8 (0 = default 8;
+ *                   inter_cluster: capped at its default mailbox depth)
+ *   flags           1 TAGS: a (pair, warp, sequence) tag is folded into every record's
+ *                   compared key, so a record consumed out of order, twice or from
+ *                   another ring is counted in *err_count;
+ *                   2 SKEW: random __nanosleep (0..skew_ns) at every CTA start and
+ *                   before one commit in eight, per role;
+ *                   4 DROP: the producer of pair 0 never publishes (a lost replica):
+ *                   its consumer must time out through the watchdog
+ *   skew_ns         maximum sleep for SKEW
+ *   watchdog_cycles watchdog bound in SM clock cycles (0 = default 2^32) -- applies to
+ *                   every launch, stress or not
+ * All zero restores the timed configuration.  Process-global, like the fault state.
+ */
+int rmt_set_stress(int depth, int flags, int skew_ns, long long watchdog_cycles);
 
 /* Kernel launches the last rmt_launch issued (for the bench's launch count). */
 int rmt_last_launch_count(void);

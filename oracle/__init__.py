@@ -48,6 +48,7 @@ def lib():
         L.orc_cnd.restype = D
         L.orc_bs_price.argtypes = [D, D, D, D, D, P, P]
         L.orc_blackscholes.argtypes = [P, I, P, P]
+        L.orc_blackscholes_indep.argtypes = [P, I, P, P, P, P]
         L.orc_binarysearch.argtypes = [P, I, P, I, P]
         L.orc_fwt_f64.argtypes = [P, I, P]
         L.orc_fwt_f32dag.argtypes = [P, I, P]
@@ -99,6 +100,16 @@ def blackscholes(r: np.ndarray):
     put = np.empty(r.size, np.float64)
     lib().orc_blackscholes(_p(r), r.size, _p(call), _p(put))
     return call, put
+
+
+def blackscholes_indep(prm: np.ndarray):
+    """prm: float32 (5, n) planes S, K, T, R, sigma -> (call, put, call_scale, put_scale)."""
+    prm = np.ascontiguousarray(prm, dtype=np.float32)
+    assert prm.ndim == 2 and prm.shape[0] == 5
+    n = prm.shape[1]
+    out = [np.empty(n, np.float64) for _ in range(4)]
+    lib().orc_blackscholes_indep(_p(prm), n, *[_p(o) for o in out])
+    return tuple(out)
 
 
 def binarysearch(A: np.ndarray, q: np.ndarray) -> np.ndarray:

@@ -90,6 +90,27 @@ void orc_blackscholes(const float* r, int64_t n, double* call, double* put) {
     }
 }
 
+/* Independent parameters (reading R-BS4, SURVEY 8(c) "bs_indep"): option i has
+ * S = prm[i], K = prm[n+i], T = prm[2n+i], R = prm[3n+i], sigma = prm[4n+i].
+ * Besides the prices, returns the conditioning scale of each price, the sum of
+ * the magnitudes of its two terms: |S N(d1)| + |K e^{-RT} N(d2)| for the call,
+ * |K e^{-RT} N(-d2)| + |S N(-d1)| for the put (the fp32 error of a difference
+ * scales with the terms, not with the difference). */
+void orc_blackscholes_indep(const float* prm, int64_t n, double* call, double* put, double* call_scale,
+                            double* put_scale) {
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; ++i) {
+        double S = prm[i], K = prm[n + i], T = prm[2 * n + i], R = prm[3 * n + i], V = prm[4 * n + i];
+        double sT = V * sqrt(T);
+        double d1 = (log(S / K) + (R + 0.5 * V * V) * T) / sT;
+        double d2 = d1 - sT;
+        double disc = K * exp(-R * T);
+        orc_bs_price(S, K, T, R, V, &call[i], &put[i]);
+        call_scale[i] = fabs(S * orc_cnd(d1)) + fabs(disc * orc_cnd(d2));
+        put_scale[i] = fabs(disc * orc_cnd(-d2)) + fabs(S * orc_cnd(-d1));
+    }
+}
+
 /* ------------------------------------------------------------------------ */
 /* BinarySearch (Fig.2 "BinS"; reading R-BIN1: batched lower_bound)   */
 /* ------------------------------------------------------------------------ */

@@ -10,8 +10,10 @@
 // improving relaxations write) and are committed with a per-word
 // predicate mask: (mask, address, D words) and (mask, address, P words).
 // D (n^2 u32 = 64 MiB at n = 4096) stays L2-resident across passes.
-#include <map>
-#include <tuple>
+#include <list>
+#include <mutex>
+#include <string>
+#include <utility>
 
 #include "rmt_host.cuh"
 
@@ -171,13 +173,44 @@ int fw_issue(Launch& L) {
 }
 
 // Host launch overhead (~n launches per call) would starve the GPU: the pass
-// sequence is captured once into a CUDA graph (keyed by every launch parameter)
-// and replayed on the caller's stream.  Inside a caller's capture the launches
-// are simply recorded into the caller's graph.
-typedef std::tuple<int, int, int, void*, void*, unsigned, void*, void*, void*, void*, int, int, int, int, long long>
-    FwKey;
-std::map<FwKey, cudaGraphExec_t> g_fw_graphs;
+// sequence is captured once into a CUDA graph (keyed by every launch parameter:
+// variant, mode, buffers, n and the whole Ctx -- error counter, queue pointers
+// and geometry, watchdog/stress settings, fault descriptor) and replayed on the
+// caller's stream.  The cache is a bounded LRU (evicted graphs are destroyed)
+// guarded by a mutex.  Inside a caller's capture the launches are simply
+// recorded into the caller's graph.
+constexpr size_t FW_GRAPH_CACHE = 16;
+std::mutex g_fw_mu;
+std::list<std::pair<std::string, cudaGraphExec_t>> g_fw_graphs;  // front = most recently used
 cudaStream_t g_fw_capture_stream = nullptr;
+
+std::string fw_key(const Launch& L) {
+  std::string k;
+  auto put = [&k](const void* p, size_t n) { k.append((const char*)p, n); };
+  put(&L.variant, sizeof L.variant);
+  put(&L.mode, sizeof L.mode);
+  put(&L.inflate, sizeof L.inflate);
+  put(&L.bufs->buf[0].ptr, sizeof(void*));
+  put(&L.bufs->buf[1].ptr, sizeof(void*));
+  put(&L.n, sizeof L.n);
+  const Ctx& c = L.ctx;
+  put(&c.err, sizeof c.err);
+  put(&c.ctrl, sizeof c.ctrl);
+  put(&c.flags, sizeof c.flags);
+  put(&c.payload, sizeof c.payload);
+  put(&c.R, sizeof c.R);
+  put(&c.W, sizeof c.W);
+  put(&c.S, sizeof c.S);
+  put(&c.wd, sizeof c.wd);
+  put(&c.stress, sizeof c.stress);
+  put(&c.skew_ns, sizeof c.skew_ns);
+  put(&c.f.replica, sizeof c.f.replica);
+  put(&c.f.site, sizeof c.f.site);
+  put(&c.f.bit, sizeof c.f.bit);
+  put(&c.f.sid, sizeof c.f.sid);
+  put(&c.f.elem, sizeof c.f.elem);
+  return k;
+}
 
 }  // namespace
 
@@ -190,11 +223,13 @@ int floydwarshall_run(Launch& L) {
     cs = cudaStreamCaptureStatusNone;
   }
   if (cs != cudaStreamCaptureStatusNone || n < 64) return fw_issue(L);
-  const FaultDesc& f = L.ctx.f;
-  FwKey key{L.variant, L.mode, (int)L.inflate, L.bufs->buf[0].ptr, L.bufs->buf[1].ptr, n, (void*)L.ctx.err,
-            (void*)L.ctx.ctrl, (void*)L.ctx.flags, (void*)L.ctx.payload, f.replica, f.site, f.bit, f.sid, f.elem};
-  auto it = g_fw_graphs.find(key);
-  if (it == g_fw_graphs.end()) {
+  const std::string key = fw_key(L);
+  std::lock_guard<std::mutex> lock(g_fw_mu);
+  auto it = g_fw_graphs.begin();
+  while (it != g_fw_graphs.end() && it->first != key) ++it;
+  if (it != g_fw_graphs.end()) {
+    g_fw_graphs.splice(g_fw_graphs.begin(), g_fw_graphs, it);  // most recently used
+  } else {
     int rc;
     if (!g_fw_capture_stream &&
         (rc = cuda_check(cudaStreamCreateWithFlags(&g_fw_capture_stream, cudaStreamNonBlocking), "fw: stream")))
@@ -213,10 +248,14 @@ int floydwarshall_run(Launch& L) {
     rc = cuda_check(cudaGraphInstantiate(&ge, g, 0), "fw: instantiate");
     cudaGraphDestroy(g);
     if (rc) return rc;
-    it = g_fw_graphs.emplace(key, ge).first;
+    g_fw_graphs.emplace_front(key, ge);
+    while (g_fw_graphs.size() > FW_GRAPH_CACHE) {  // evict the least recently used graph
+      cudaGraphExecDestroy(g_fw_graphs.back().second);
+      g_fw_graphs.pop_back();
+    }
   }
   L.launches += (int)n + 1;
-  return cuda_check(cudaGraphLaunch(it->second, L.stream), "fw: graph launch");
+  return cuda_check(cudaGraphLaunch(g_fw_graphs.front().second, L.stream), "fw: graph launch");
 }
 
 }  // namespace rmt

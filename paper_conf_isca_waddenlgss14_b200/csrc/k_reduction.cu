@@ -79,7 +79,9 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) red_partial_kernel(RedArgs 
       s += (unsigned long long)v[u].x + v[u].y + (unsigned long long)v[u].z + v[u].w;
     }
   }
-  for (unsigned e = nvec * 4 + gt; e < a.n; e += T) s += rep.fault(SITE_LOAD, (long long)e, a.x[e]);  // ragged tail
+  // ragged tail (< 4 elements), indexed in 64 bits: n may be within T of 2^32
+  for (unsigned long long e = (unsigned long long)nvec * 4 + gt; e < a.n; e += T)
+    s += rep.fault(SITE_LOAD, (long long)e, a.x[e]);
   s = (s & 0xffffffff00000000ull) | rep.fault(SITE_COMPUTE, (long long)gt, (unsigned)s);
   unsigned long long t = block_sum(rep, s, sm_warp);
   if (rep.warp == 0) {  // warp-uniform: only warp 0 holds the CTA's store (P:809 ghost warps)

@@ -15,6 +15,12 @@ thread_local std::string g_err;
 FaultDesc g_fault = {0, 0, 0, 0, 0};
 bool g_armed = false;
 int g_ablation = RMT_ABL_FULL;
+struct StressCfg {
+  int depth;                 // queue slots in use (0: default)
+  int flags;                 // STRESS_* bits
+  unsigned skew_ns;
+  unsigned long long wd;     // watchdog cycles (0: WATCHDOG_CYCLES)
+} g_stress = {0, 0, 0, 0};
 thread_local int g_last_launches = 0;
 
 struct KEntry {
@@ -193,6 +199,7 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
     L.n = n;
     L.stream = (cudaStream_t)stream;
     L.ctx.err = err_count;
+    L.ctx.wd = WATCHDOG_CYCLES;
     rc = run_dup(L, e, (char*)workspace, g_armed, g_fault);
     g_last_launches = L.launches;
     if (rc == RMT_OK) rc = cuda_check(cudaGetLastError(), "kernel launch");
@@ -205,13 +212,22 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
   Launch L{};
   L.kernel = kernel;
   L.variant = variant;
-  L.mode = g_armed ? M_FAULT : (g_ablation == RMT_ABL_NOCOMM && variant != RMT_NONE ? M_NOCOMM : M_NORMAL);
+  const bool queue_variant = variant == RMT_INTER_GROUP || variant == RMT_INTER_CLUSTER;
+  const bool stress = queue_variant && (g_stress.depth > 0 || g_stress.flags != 0);
+  L.mode = g_armed ? M_FAULT
+         : (g_ablation == RMT_ABL_NOCOMM && variant != RMT_NONE) ? M_NOCOMM
+         : stress ? M_STRESS
+                  : M_NORMAL;
   L.inflate = !g_armed && g_ablation == RMT_ABL_INFLATE && variant != RMT_NONE;
   L.bufs = bufs;
   L.n = n;
   L.stream = (cudaStream_t)stream;
   L.ctx.err = err_count;
   L.ctx.f = g_fault;
+  L.ctx.wd = g_stress.wd ? g_stress.wd : WATCHDOG_CYCLES;
+  L.ctx.stress = g_stress.flags;
+  L.ctx.skew_ns = g_stress.skew_ns;
+  L.cl_depth = (variant == RMT_INTER_CLUSTER) ? g_stress.depth : 0;
   char* ws = (char*)workspace;
   if (variant == RMT_INTER_GROUP) {
     int W = e.inter_warps(n, bufs->dims);
@@ -221,7 +237,7 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
     L.ctx.payload = (unsigned*)(ws + CTRL_BYTES + slots * 4);
     L.ctx.R = INTER_R;
     L.ctx.W = W;
-    L.ctx.S = INTER_S;
+    L.ctx.S = g_stress.depth > 0 ? g_stress.depth : INTER_S;
   }
   L.scratch = ws ? ws + inter_part : nullptr;
   L.scratch_bytes = need - inter_part;
@@ -304,6 +320,38 @@ int rmt_set_ablation(int mode) {
 
 int rmt_last_launch_count(void) { return g_last_launches; }
 
+int rmt_set_stress(int depth, int flags, int skew_ns, long long watchdog_cycles) {
+  if (depth < 0 || depth > INTER_S || (depth & (depth - 1)) != 0 || flags < 0 ||
+      flags > (STRESS_TAGS | STRESS_SKEW | STRESS_DROP) || skew_ns < 0 || watchdog_cycles < 0) {
+    set_error("rmt_set_stress: depth in {0,1,2,4,8}, flags in 0..7, skew_ns >= 0, watchdog_cycles >= 0");
+    return RMT_EINVAL;
+  }
+  g_stress.depth = depth;
+  g_stress.flags = flags;
+  g_stress.skew_ns = (unsigned)skew_ns;
+  g_stress.wd = (unsigned long long)watchdog_cycles;
+  return RMT_OK;
+}
+
+int rmt_workspace_status(int variant, void* workspace, void* stream) {
+  if (variant != RMT_INTER_GROUP || workspace == nullptr) return RMT_OK;  // only the L2 queue has sticky state
+  cudaStream_t s = (cudaStream_t)stream;
+  unsigned flag = 0;
+  unsigned* ctrl = (unsigned*)workspace;
+  int rc = cuda_check(cudaMemcpyAsync(&flag, ctrl + CTRL_WATCHDOG, 4, cudaMemcpyDeviceToHost, s), "status: read");
+  if (!rc) rc = cuda_check(cudaStreamSynchronize(s), "status: sync");
+  if (rc) return rc;
+  if (flag == 0u) return RMT_OK;
+  // the last CTA of the aborted launch already cleared the slot flags; clear the
+  // sticky flag so the workspace is reusable
+  rc = cuda_check(cudaMemsetAsync(ctrl + CTRL_WATCHDOG, 0, 4, s), "status: clear");
+  if (!rc) rc = cuda_check(cudaStreamSynchronize(s), "status: sync");
+  if (rc) return rc;
+  set_error("inter_group watchdog fired: a replica waited longer than the watchdog bound for its partner "
+            "(each timeout was counted in *err_count, the affected stores were not committed); the queue was reset");
+  return RMT_EWATCHDOG;
+}
+
 const char* rmt_strerror(int code) {
   switch (code) {
     case RMT_OK: return "ok";
@@ -312,6 +360,7 @@ const char* rmt_strerror(int code) {
     case RMT_EWORKSPACE: return "workspace too small";
     case RMT_ECUDA: return "CUDA error";
     case RMT_ENODEV: return "no sm_100 device";
+    case RMT_EWATCHDOG: return "inter-group watchdog fired (a replica pair timed out)";
   }
   return "unknown error";
 }

@@ -4,6 +4,10 @@
 //   V    = V_NONE | V_INTRA_SMEM | V_INTRA_REG | V_INTER | V_CLUSTER | V_INTRA_NOLDS  (include/rmt.h)
 //   MODE = M_NORMAL | M_FAULT (single-bit fault hooks compiled in) | M_NOCOMM
 //          (ablation: replicas run, no exchange/compare)
+//          | M_STRESS (inter variants only: queue-protocol stress test build --
+//          per-CTA / per-commit random __nanosleep skew, (pair, warp, seq) tags
+//          folded into every record key, an optional dropped producer; SURVEY
+//          8(c) C-Q pins)
 //
 // What this header implements, with the paper passage each piece follows
 // ("P:NNN" = line of /root/reference/PAPER.md):
@@ -36,14 +40,19 @@
 namespace rmt {
 
 constexpr int V_NONE = 0, V_INTRA_SMEM = 1, V_INTRA_REG = 2, V_INTER = 3, V_CLUSTER = 4, V_INTRA_NOLDS = 5;
-constexpr int M_NORMAL = 0, M_FAULT = 1, M_NOCOMM = 2;
+constexpr int M_NORMAL = 0, M_FAULT = 1, M_NOCOMM = 2, M_STRESS = 3;
 constexpr int SITE_LOAD = 0, SITE_COMPUTE = 1, SITE_SMEM = 2, SITE_STORE_VAL = 3, SITE_STORE_ADDR = 4;
 constexpr int MAXW = 4;               // max value words per commit
 constexpr int RING_WORDS = 1 + MAXW;  // key + values per lane per record
 constexpr int MBOX_WORDS = RING_WORDS * 16;  // intra_smem mailbox words per warp
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int CTRL_TURN = 64;         // ctrl[64 ..) = per-region turn counters
-constexpr unsigned long long WATCHDOG_CYCLES = 1ull << 32;  // ~2 s at 2 GHz
+constexpr unsigned long long WATCHDOG_CYCLES = 1ull << 32;  // default Ctx::wd: ~2 s at 2 GHz
+// Ctx::stress bits (M_STRESS builds)
+constexpr int STRESS_TAGS = 1, STRESS_SKEW = 2, STRESS_DROP = 4;
+// ctrl[] words of the inter queue control block
+constexpr int CTRL_TICKET = 0, CTRL_DONE = 1, CTRL_WATCHDOG = 2;
+constexpr int INTER_SLOTS_MAX = 8;  // slots allocated per (region, warp); Ctx::S <= this
 // inter_cluster: record slots per warp in the consumer CTA's shared memory
 // (Ctx::S, a power of two chosen by the launcher): 8 lets the producer fill one
 // deferred batch (<= 4 records) while the consumer drains the previous one; 4
@@ -64,8 +73,11 @@ struct Ctx {
   unsigned* ctrl;           // inter: [0] ticket [1] done [2] watchdog flag, [64..64+R) turn
   unsigned* flags;          // inter: R*W*S slot flags (0 free, 1 full)
   unsigned* payload;        // inter: R*W*S records of RING_WORDS*32 words
-  int R, W, S;              // inter queue geometry (regions, warps per CTA, slots)
+  int R, W, S;              // inter queue geometry (regions, warps per CTA, slots in use: 1..INTER_S)
   int nblocks;              // logical CTAs in this launch
+  unsigned long long wd;    // watchdog bound in clock64 cycles (WATCHDOG_CYCLES unless a stress test lowers it)
+  int stress;               // M_STRESS: STRESS_* bits
+  unsigned skew_ns;         // M_STRESS: maximum random sleep (ns) per CTA start / per commit
   FaultDesc f;
 };
 
@@ -167,10 +179,10 @@ __device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, con
     if (ns) __nanosleep(ns);
     if (ld_acquire(p) == want) return true;
     if (ns && ns < RMT_SPIN_NSMAX) ns <<= 1;
-    if (clock64() - t0 > WATCHDOG_CYCLES) {
+    if (clock64() - t0 > c.wd) {
       if (count) {
         atomicAdd(c.err, 1ull);
-        atomicExch(c.ctrl + 2, 1u);
+        atomicExch(c.ctrl + CTRL_WATCHDOG, 1u);
       }
       return false;
     }
@@ -184,11 +196,21 @@ __device__ __forceinline__ bool spin_cl(unsigned addr, unsigned want, const Ctx&
   while (true) {
     __nanosleep(20);
     if (ld_acquire_cl(addr) == want) return true;
-    if (clock64() - t0 > WATCHDOG_CYCLES) {
+    if (clock64() - t0 > c.wd) {
       if (count) atomicAdd(c.err, 1ull);
       return false;
     }
   }
+}
+
+// 32-bit mixer (stress skew and record tags): lowbias32
+__device__ __forceinline__ unsigned mix32(unsigned x) {
+  x ^= x >> 16;
+  x *= 0x7feb352du;
+  x ^= x >> 15;
+  x *= 0x846ca68bu;
+  x ^= x >> 16;
+  return x;
 }
 
 // ---------------------------------------------------------------- replica state
@@ -205,6 +227,7 @@ struct Rep {
   static constexpr int LW = 32 / DUP;        // logical warp width
   static constexpr bool FAULT = (MODE == M_FAULT);
   static constexpr bool NOCOMM = (MODE == M_NOCOMM);
+  static constexpr bool STRESS = (MODE == M_STRESS) && (V == V_INTER || V == V_CLUSTER);
 
   const Ctx& c;
   int r;          // replica id 0/1 (fault targeting)
@@ -252,6 +275,9 @@ struct Rep {
       llane = lane;
       region = (unsigned)lblock % (unsigned)c.R;
       epoch = (unsigned)lblock / (unsigned)c.R;
+      if constexpr (STRESS) {  // random per-CTA start skew: perturbs which role runs ahead
+        if (c.stress & STRESS_SKEW) __nanosleep(mix32(t * 0x9E3779B9u + 1u) % (c.skew_ns + 1u));
+      }
       if constexpr (!NOCOMM) {
         // Exclusive ownership of the queue region: wait until the pair that used
         // it before (lblock - R) has fully drained it (both roles wait).
@@ -272,6 +298,9 @@ struct Rep {
       lblock = (int)cluster_id_x();
       ltid = threadIdx.x;
       llane = lane;
+      if constexpr (STRESS) {
+        if (c.stress & STRESS_SKEW) __nanosleep(mix32((unsigned)(2 * lblock + r) * 0x9E3779B9u + 1u) % (c.skew_ns + 1u));
+      }
       if constexpr (!NOCOMM) {
         const unsigned nw = blockDim.x >> 5;
         const unsigned base = (unsigned)__cvta_generic_to_shared(rmt_dyn_smem) + (unsigned)c.R;
@@ -353,9 +382,17 @@ struct Rep {
       if (s_last) {  // self-reset: the next launch starts from zero
         __threadfence();
         for (int i = threadIdx.x; i < c.R; i += blockDim.x) c.ctrl[CTRL_TURN + i] = 0;
+        // After a watchdog abort a producer may have published records its
+        // consumer never freed: clear every slot flag (all other CTAs have
+        // finished, so no flag store is in flight).  The sticky watchdog flag
+        // itself stays set for rmt_workspace_status() to report.
+        if (ld_relaxed(c.ctrl + CTRL_WATCHDOG) != 0u) {
+          const size_t nslots = (size_t)c.R * (size_t)c.W * (size_t)INTER_SLOTS_MAX;
+          for (size_t i = threadIdx.x; i < nslots; i += blockDim.x) c.flags[i] = 0u;
+        }
         if (threadIdx.x == 0) {
-          c.ctrl[0] = 0;
-          c.ctrl[1] = 0;
+          c.ctrl[CTRL_TICKET] = 0;
+          c.ctrl[CTRL_DONE] = 0;
         }
       }
     }
@@ -456,7 +493,7 @@ struct Rep {
   // ---- the commit.  Warp-collective: every lane of the warp must
   // call it at the same program point (uniform control flow around commits).
   //   mask  bit k set = word k is stored (a store instruction's predicate)
-  //   idx   element index of word 0 in the destination (multiple of NW if NW>1)
+  //   idx   element index of word 0 in the destination (any value; the key keeps all 32 bits)
   //   v     the NW 32-bit value words
   //   limit destination element count (bounds for address faults in V_NONE)
   //   store functor store(idx, mask, v) performing the actual global store(s)
@@ -485,7 +522,7 @@ struct Rep {
           for (int k = 0; k < NW; ++k)
             if (k == w) v[k] ^= 1u << c.f.bit;
         } else if (c.f.site == SITE_STORE_ADDR) {
-          idx ^= (NW == 1 ? 1u : (unsigned)NW) << c.f.bit;  // bit of the (vector) index
+          idx ^= 1u << c.f.bit;  // any bit of the element index (0..31)
           addr_faulted = true;
         }
       }
@@ -493,8 +530,13 @@ struct Rep {
     if constexpr (V == V_NONE) {
       if (mask != 0u) {
         if constexpr (FAULT) {
-          // a faulted address whose stored words fall outside the buffer: dropped
-          if (addr_faulted && idx + (31u - (unsigned)__clz(mask)) * stride >= limit) return;
+          // a faulted address whose stored words fall outside the buffer, or that
+          // is misaligned for a contiguous vector store, is dropped (the hardware
+          // would raise an exception instead; either way the word is not written)
+          if (addr_faulted && ((unsigned long long)idx + (31u - (unsigned)__clz(mask)) * (unsigned long long)stride >=
+                                   limit ||
+                               (NW > 1 && stride == 1u && idx % (unsigned)NW != 0u)))
+            return;
         }
         store(idx, mask, v);
       }
@@ -512,10 +554,33 @@ struct Rep {
         return;
       }
       (void)defer;
-      // Record key: address + predicate in one word.
+      // Record key: address + predicate in one word.  For a storing lane,
+      // key = idx ^ (mask << 28) keeps every bit of the element index (vector
+      // sites need not be aligned, e.g. FWT's strided commits) and is injective
+      // in each argument separately: a fault in either the address or the
+      // predicate of one replica (any single bit, or any corruption of only one
+      // of the two) changes the key.  A lane that stores nothing has no address
+      // to compare (key 0xFFFFFFFF); since vector-committed buffers hold < 2^30
+      // elements, no storing lane whose mask differs from 0 in one bit can have
+      // that key.
       unsigned key;
       if constexpr (NW == 1) key = mask ? idx : 0xffffffffu;
-      else key = mask ? (((idx / NW) << NW) | mask) : 0u;
+      else key = mask ? (idx ^ (mask << 28)) : 0xffffffffu;
+      if constexpr (STRESS) {
+        // (pair, warp, sequence) tag folded into the key on both sides: a record
+        // consumed out of order, twice, or from another pair's/warp's ring fails
+        // the compare (counted in err)
+        const unsigned tag = mix32(((unsigned)lblock * 64u + (unsigned)warp) * 0x01000193u) ^ mix32(j + 0x51ED270Bu);
+        if (c.stress & STRESS_TAGS) key ^= tag;
+        if (c.stress & STRESS_SKEW) {  // one commit in 8 (per warp and role) sleeps a random while
+          const unsigned h = mix32(tag ^ (unsigned)r * 0x2545F491u);
+          if ((h & 7u) == 0u) __nanosleep((h >> 3) % (c.skew_ns + 1u));
+        }
+        if ((c.stress & STRESS_DROP) && lblock == 0 && !consumer) {  // a lost producer: pair 0 never publishes
+          ++j;
+          return;
+        }
+      }
       unsigned pk = 0, pv[NW];
       bool have = true;  // consumer got the producer's record
       if constexpr (V == V_INTRA_REG || V == V_INTRA_NOLDS) {
@@ -561,6 +626,9 @@ struct Rep {
           for (int k = 0; k < NW; ++k)
             if (!COND || ((mask >> k) & 1u)) st_cl(pa + (1 + k) * 32 * 4, v[k]);
         } else {
+          // a consumer holding S unfreed records frees them before it waits on
+          // a slot (any depth S >= 1, however long the deferred run)
+          if (pend >= (unsigned)c.S) flush();
           have = spin_cl(fa, 1u, c, lane == 0);  // every lane acquires
           pk = ld_cl(pa);
 #pragma unroll
@@ -586,6 +654,7 @@ struct Rep {
           // published by flush(): every lane fences its own payload stores (a
           // release by one lane does not order the other lanes' in-flight stores).
         } else {
+          if (pend >= (unsigned)c.S) flush();  // as above: never wait on a slot we still hold
           const bool ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
           pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
 #pragma unroll
@@ -606,8 +675,11 @@ struct Rep {
           if (mask != 0u) store(idx, mask, v);
         } else {
           mism = true;
-          if constexpr (LIVE) {  // highest stored word must be inside the buffer
-            if (mask != 0u && idx + (31u - (unsigned)__clz(mask)) * stride < limit) store(idx, mask, v);
+          if constexpr (LIVE) {  // highest stored word inside the buffer, vector aligned
+            if (mask != 0u &&
+                (unsigned long long)idx + (31u - (unsigned)__clz(mask)) * (unsigned long long)stride < limit &&
+                !(NW > 1 && stride == 1u && idx % (unsigned)NW != 0u))
+              store(idx, mask, v);
           }
         }
       }

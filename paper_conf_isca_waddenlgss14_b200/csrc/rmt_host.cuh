@@ -17,12 +17,13 @@ namespace rmt {
 
 // Inter-group queue geometry.
 constexpr int INTER_R = 1024;  // regions (> resident pairs, so a region is rarely waited for)
-constexpr int INTER_S = 8;     // slots (records in flight) per (region, warp)
+constexpr int INTER_S = INTER_SLOTS_MAX;  // slots allocated per (region, warp); Ctx::S <= INTER_S in use
 constexpr size_t CTRL_BYTES = (size_t)(CTRL_TURN + INTER_R) * 4;
 
 struct Launch {
   int kernel, variant, mode;
   bool inflate;               // RMT_ABL_INFLATE: run V_NONE with the RMT variant's residency
+  int cl_depth;               // inter_cluster mailbox slots requested by a stress test (0: default)
   const rmt_bufs_t* bufs;
   int64_t n;
   Ctx ctx;                    // err + fault + inter queue pointers
@@ -49,7 +50,8 @@ struct VM {
 };
 
 // Call f(VM<V, M>{}) for the runtime (variant, mode).  M_NOCOMM only exists for
-// the RMT variants; the none variant ignores it.
+// the RMT variants; the none variant ignores it.  M_STRESS only exists for the
+// queue variants (inter_group, inter_cluster); the others run M_NORMAL.
 template <class F>
 int dispatch(int v, int m, F&& f) {
   switch (v) {
@@ -66,6 +68,7 @@ int dispatch(int v, int m, F&& f) {
     case V_INTER:
       return m == M_FAULT ? f(VM<V_INTER, M_FAULT>{})
            : m == M_NOCOMM ? f(VM<V_INTER, M_NOCOMM>{})
+           : m == M_STRESS ? f(VM<V_INTER, M_STRESS>{})
                            : f(VM<V_INTER, M_NORMAL>{});
     case V_INTRA_NOLDS:
       return m == M_FAULT ? f(VM<V_INTRA_NOLDS, M_FAULT>{})
@@ -74,6 +77,7 @@ int dispatch(int v, int m, F&& f) {
     case V_CLUSTER:
       return m == M_FAULT ? f(VM<V_CLUSTER, M_FAULT>{})
            : m == M_NOCOMM ? f(VM<V_CLUSTER, M_NOCOMM>{})
+           : m == M_STRESS ? f(VM<V_CLUSTER, M_STRESS>{})
                            : f(VM<V_CLUSTER, M_NORMAL>{});
   }
   return RMT_EINVAL;
@@ -161,6 +165,7 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
     if (L.mode != M_NOCOMM) {
       c.R = (int)align_up(smem, 16);
       c.S = BL <= 128 ? CL_S_LARGE : CL_S_SMALL;
+      if (L.cl_depth > 0 && L.cl_depth < c.S) c.S = L.cl_depth;  // stress test: a shallower mailbox (power of 2)
       dyn = (size_t)c.R + (size_t)(BL / 32) * c.S * (RING_WORDS * 32 + 1) * 4;
     }
     cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);

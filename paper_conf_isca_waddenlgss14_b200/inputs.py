@@ -59,6 +59,64 @@ def blackscholes_r(seed: int, n: int, offset: int = 0) -> np.ndarray:
     return uniform_f32(seed, n, offset)
 
 
+def blackscholes_indep(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """Independent parameters (SURVEY 8(c) "bs_indep"): uniform S in [5,30],
+    K in [1,100], T in [0.25,10], R in [0.01,0.05], sigma in [0.1,0.5]; returned
+    as float32 planes (5, n): S | K | T | R | sigma (the ABI's mode-1 layout)."""
+    lo = (5.0, 1.0, 0.25, 0.01, 0.10)
+    hi = (30.0, 100.0, 10.0, 0.05, 0.50)
+    out = np.empty((5, n), np.float32)
+    for k in range(5):
+        u = uniform_f32(seed, n, offset, stream=30 + k).astype(np.float64)
+        out[k] = (lo[k] + (hi[k] - lo[k]) * u).astype(np.float32)
+    return out
+
+
+# Hand-picked option rows (S, K, T, R, sigma) for the independent-parameter
+# mode: textbook points, at/in/out of the money, negative d1 and d2, extremes
+# of the bs_indep ranges.
+BS_EDGE_ROWS = [
+    (100.0, 100.0, 1.0, 0.05, 0.20),   # textbook ATM point (C = 10.45058, P = 5.57353)
+    (42.0, 40.0, 0.5, 0.10, 0.20),     # Hull, Options Futures & Other Derivatives, Ex. 15.6 (C ~ 4.76, P ~ 0.81)
+    (30.0, 1.0, 10.0, 0.05, 0.50),     # deep in the money call
+    (5.0, 100.0, 0.25, 0.01, 0.10),    # deep out of the money call (d1 ~ -60)
+    (20.0, 40.0, 2.0, 0.03, 0.30),     # d1 < 0, d2 < 0
+    (25.0, 30.0, 5.0, 0.02, 0.15),     # slightly out of the money: d1, d2 just below 0
+    (10.0, 10.5, 0.25, 0.01, 0.50),    # near the money, short expiry, high vol
+    (5.0, 1.0, 0.25, 0.05, 0.10),      # deep ITM, short expiry
+    (30.0, 100.0, 10.0, 0.01, 0.50),   # OTM, long expiry, high vol
+    (12.0, 11.0, 0.25, 0.05, 0.10),    # d1 > 0, d2 > 0
+    (7.5, 8.0, 3.0, 0.04, 0.40),       # d1 > 0 > d2
+    (1.0, 100.0, 10.0, 0.05, 0.10),    # extreme OTM: prices underflow to 0
+]
+
+
+def blackscholes_edges() -> np.ndarray:
+    """BS_EDGE_ROWS as float32 planes (5, n), n padded to a multiple of 4 by
+    repeating the first row."""
+    rows = list(BS_EDGE_ROWS)
+    while len(rows) % 4:
+        rows.append(rows[0])
+    return np.ascontiguousarray(np.array(rows, dtype=np.float32).T)
+
+
+def with_specials(x: np.ndarray, seed: int, frac: float = 0.01, kinds=("nan", "+0", "-0")) -> np.ndarray:
+    """A copy of float32 x with a seeded fraction of entries replaced by IEEE
+    special values (quiet NaN, +0, -0, optionally +/-inf): the bitwise-compare
+    reading R-RMT4 must give no false alarm on any of them."""
+    x = np.array(x, dtype=np.float32, copy=True)
+    flat = x.reshape(-1)
+    n = flat.size
+    m = max(1, int(n * frac))
+    pos = (u64(seed, m, 0, stream=40) % np.uint64(max(n, 1))).astype(np.int64)
+    sel = (u32(seed, m, 0, stream=41) % np.uint32(len(kinds))).astype(np.int64)
+    vals = {"nan": np.float32(np.nan), "+0": np.float32(0.0), "-0": np.float32(-0.0),
+            "+inf": np.float32(np.inf), "-inf": np.float32(-np.inf)}
+    for i, k in enumerate(kinds):
+        flat[pos[sel == i]] = vals[k]
+    return x
+
+
 def binarysearch_inputs(seed: int, N: int, Q: int, q_offset: int = 0):
     """Sorted, strictly increasing u32 A[N] spread over the full u32 range, and
     uniform u32 queries q[Q].  A[i] = i*stride + (h(i) mod stride) (no prefix sum
@@ -70,6 +128,21 @@ def binarysearch_inputs(seed: int, N: int, Q: int, q_offset: int = 0):
     A = (np.arange(N, dtype=np.uint64) * np.uint64(stride) + h % np.uint64(stride)).astype(np.uint32)
     q = u32(seed, Q, q_offset, stream=2)
     return A, q
+
+
+def binarysearch_dups(seed: int, N: int, Q: int, distinct: int = 1000):
+    """Sorted A[N] with heavy duplication: values from a pool of `distinct`
+    random keys plus 0 and 0xFFFFFFFF (both extremes present, in runs);
+    queries drawn from the pool, its neighbours (key - 1, key + 1) and the two
+    extremes, so every lower_bound lands on the first element of a run."""
+    pool = np.unique(np.concatenate([u32(seed, distinct, 0, stream=42),
+                                     np.array([0, 1, 0xFFFFFFFE, 0xFFFFFFFF], np.uint32)]))
+    A = np.sort(pool[(u32(seed, N, 0, stream=43) % np.uint32(pool.size)).astype(np.int64)])
+    pick = pool[(u32(seed, Q, 0, stream=44) % np.uint32(pool.size)).astype(np.int64)].astype(np.int64)
+    delta = (u32(seed, Q, 0, stream=45) % np.uint32(3)).astype(np.int64) - 1
+    q = np.clip(pick + delta, 0, 0xFFFFFFFF).astype(np.uint32)
+    q[: min(Q, 4)] = np.array([0, 0xFFFFFFFF, 1, 0xFFFFFFFE], np.uint32)[: min(Q, 4)]
+    return A.astype(np.uint32), q
 
 
 def fwt_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
@@ -114,6 +187,21 @@ def floydwarshall_w(seed: int, n: int) -> np.ndarray:
     w = (u32(seed, n * n, 0, stream=8) % np.uint32(200) + np.uint32(1)).reshape(n, n)
     np.fill_diagonal(w, 0)
     return w.astype(np.uint32)
+
+
+FW_INF = 0x3FFFFFFF  # "no edge" weight of the sparse FloydWarshall graphs
+
+
+def floydwarshall_sparse(seed: int, n: int, p_edge: float = 0.05) -> np.ndarray:
+    """Sparse digraph: each off-diagonal edge present with probability p_edge
+    (weight U{1..200}), absent edges FW_INF = 0x3FFFFFFF (2 * FW_INF < 2^32: the
+    u32 relaxation sum cannot wrap), zero diagonal.  Small p_edge leaves some
+    pairs unreachable (their distance stays >= FW_INF)."""
+    w = (u32(seed, n * n, 0, stream=8) % np.uint32(200) + np.uint32(1)).reshape(n, n)
+    present = (u32(seed, n * n, 0, stream=46).astype(np.float64) * 2.0 ** -32).reshape(n, n) < p_edge
+    w = np.where(present, w, np.uint32(FW_INF)).astype(np.uint32)
+    np.fill_diagonal(w, 0)
+    return w
 
 
 def dct_x(seed: int, H: int, W: int, row_offset: int = 0) -> np.ndarray:

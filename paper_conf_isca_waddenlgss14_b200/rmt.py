@@ -91,6 +91,10 @@ def lib() -> ctypes.CDLL:
         L.rmt_variant_name.restype = ctypes.c_char_p
         L.rmt_probe_cluster_placement.argtypes = [I64, ctypes.POINTER(ctypes.c_int64)]
         L.rmt_probe_cluster_placement.restype = I32
+        L.rmt_workspace_status.argtypes = [I32, P, P]
+        L.rmt_workspace_status.restype = I32
+        L.rmt_set_stress.argtypes = [I32, I32, I32, ctypes.c_longlong]
+        L.rmt_set_stress.restype = I32
         _lib = L
     return _lib
 
@@ -187,6 +191,30 @@ def clear_faults():
 def set_ablation(mode):
     m = ABLATIONS[mode] if isinstance(mode, str) else int(mode)
     _check(lib().rmt_set_ablation(m), "rmt_set_ablation")
+
+
+STRESS_TAGS, STRESS_SKEW, STRESS_DROP = 1, 2, 4
+EWATCHDOG = -6
+
+
+def set_stress(depth: int = 0, flags: int = 0, skew_ns: int = 0, watchdog_cycles: int = 0):
+    """rmt_set_stress (include/rmt.h): queue depth / tags / skew / dropped producer
+    for the inter variants, and the watchdog bound.  All zero = timed configuration."""
+    _check(lib().rmt_set_stress(int(depth), int(flags), int(skew_ns), int(watchdog_cycles)), "rmt_set_stress")
+
+
+def workspace_status(variant: str, workspace, stream=None) -> str | None:
+    """rmt_workspace_status: None if the inter-group watchdog flag is clear,
+    else its rmt_last_error message (the flag is cleared)."""
+    if stream is None:
+        stream = torch.cuda.current_stream().cuda_stream
+    L = lib()
+    rc = L.rmt_workspace_status(VARIANTS[variant], workspace.data_ptr() if workspace is not None else None, stream)
+    if rc == 0:
+        return None
+    if rc != EWATCHDOG:
+        _check(rc, "rmt_workspace_status")
+    return L.rmt_last_error().decode()
 
 
 def last_launch_count() -> int:

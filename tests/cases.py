@@ -21,6 +21,11 @@ class Case:
     kernel: str
     n: int
     dims: tuple = ()
+    tag: str = ""  # input-set qualifier for test ids (specials, dups, sparse, ...)
+
+    @property
+    def id(self):
+        return f"{self.kernel}-{self.n}{self.tag}"
 
     def buffers(self):
         """Fresh device buffers in schema order (outputs sentinel-filled)."""
@@ -56,12 +61,25 @@ class Case:
         return np.arange(lo, min(lo + 4, ne))
 
 
+def _nan_aware_equal(got_bits, ref_bits):
+    """Bitwise equality, except that any NaN matches any NaN (the CPU and the
+    GPU quiet NaNs with different payloads; the RMT variants are still compared
+    with `none` bit for bit)."""
+    g = got_bits.view(np.float32)
+    r = ref_bits.view(np.float32)
+    gn, rn = np.isnan(g), np.isnan(r)
+    return np.array_equal(gn, rn) and np.array_equal(got_bits[~gn], ref_bits[~rn])
+
+
 class BlackScholes(Case):
     kernel = "blackscholes"
 
-    def __init__(self, n, seed=1):
+    def __init__(self, n, seed=1, specials=False):
         self.n = n
         self.r = inputs.blackscholes_r(seed, n)
+        if specials:  # NaN and +-0 draws (R-RMT4: bitwise compare, no false alarm)
+            self.r = inputs.with_specials(self.r, seed, 0.02)
+            self.tag = "-specials"
 
     @functools.cached_property
     def r_d(self):
@@ -78,12 +96,51 @@ class BlackScholes(Case):
         call_ref, put_ref = oracle.blackscholes(r)
         rr = r.astype(np.float64)
         S = 10 * rr + 100 * (1 - rr)
+        nan_in = np.isnan(rr)
         for got_bits, ref in zip(outs, (call_ref, put_ref)):
             got = got_bits.view(np.float32).astype(np.float64)
+            assert np.array_equal(np.isnan(got), nan_in), "NaN inputs (only) must give NaN prices"
             # reading R-BS3: relative 1e-4 (BJ tolerance for BlackScholes), floored at 1e-2*S
             tol = 1e-4 * np.maximum(np.abs(ref), 1e-2 * S)
-            bad = ~(np.abs(got - ref) <= tol)
+            bad = ~(np.abs(got - ref) <= tol) & ~nan_in
             assert not bad.any(), f"{bad.sum()} mismatches, first at {np.argmax(bad)}"
+
+    def out_elems(self):
+        return 1, self.n
+
+
+class BlackScholesIndep(Case):
+    """Independent-parameter mode (dims[0] = 1; reading R-BS4): S != K, so the
+    moneyness term ln(S/K) and the x < 0 branch of the CND are exercised."""
+    kernel = "blackscholes"
+
+    def __init__(self, n=None, seed=13, edges=False):
+        self.prm = inputs.blackscholes_edges() if edges else inputs.blackscholes_indep(seed, n)
+        self.n = self.prm.shape[1]
+        self.dims = (1,)
+        self.tag = "-edges" if edges else "-indep"
+
+    @functools.cached_property
+    def p_d(self):
+        return dev(self.prm.reshape(-1))
+
+    def buffers(self):
+        return [self.p_d, out_like(4 * self.n), out_like(4 * self.n)]
+
+    def outputs(self, b):
+        return [host(b[1], np.uint32), host(b[2], np.uint32)]
+
+    def check(self, outs, prm=None):
+        prm = self.prm if prm is None else prm
+        call, put, cs, ps = oracle.blackscholes_indep(prm)
+        scale_floor = 1e-7 * np.maximum(prm[0], prm[1]).astype(np.float64)
+        for got_bits, ref, scale in zip(outs, (call, put), (cs, ps)):
+            got = got_bits.view(np.float32).astype(np.float64)
+            # reading R-BS4: 1e-4 (BJ) relative to the price's two terms |t1| + |t2|
+            # (a difference of near-equal terms is ill-conditioned), floored at
+            # 1e-7 max(S, K) (~1 fp32 ulp of the price scale)
+            bad = ~(np.abs(got - ref) <= 1e-4 * scale + scale_floor)
+            assert not bad.any(), f"{bad.sum()} mismatches, first at {np.argmax(bad)}: got {got[bad][:4]} want {ref[bad][:4]}"
 
     def out_elems(self):
         return 1, self.n
@@ -172,10 +229,15 @@ class PrefixSum(Case):
 class FWT(Case):
     kernel = "fwt"
 
-    def __init__(self, n, seed=5, ternary=False):
+    def __init__(self, n, seed=5, ternary=False, specials=False):
         self.n = n
         self.multipass = n > 4096
         self.x = inputs.fwt_ternary(seed, n) if ternary else inputs.fwt_x(seed, n)
+        self.specials = specials
+        if specials:  # a few +-0 everywhere and one NaN (which spreads to every output)
+            self.x = inputs.with_specials(self.x, seed, 0.01, kinds=("+0", "-0"))
+            self.x[n // 3] = np.float32(np.nan)
+            self.tag = "-specials"
 
     @functools.cached_property
     def x_d(self):
@@ -189,6 +251,11 @@ class FWT(Case):
 
     def check(self, outs, x=None):
         x = self.x if x is None else x
+        if np.isnan(x).any():
+            # a NaN reaches every output through the butterflies (payloads differ
+            # between CPU and GPU): every output NaN, on both sides
+            assert _nan_aware_equal(outs[0], oracle.fwt_f32dag(x).view(np.uint32))
+            return
         # R-FWT2: bit-exact vs the fp32 butterfly DAG in the normative stage order
         assert np.array_equal(outs[0], oracle.fwt_f32dag(x).view(np.uint32))
         # and within fp32 rounding of the fp64 definition (BJ 1e-5 relative, scaled by ||x||_1)
@@ -220,11 +287,14 @@ class FWT(Case):
 class BinarySearch(Case):
     kernel = "binarysearch"
 
-    def __init__(self, N, Q, seed=6, odd=False):
+    def __init__(self, N, Q, seed=6, odd=False, dups=False):
         self.N, self.Q = N, Q
         self.n = Q
         self.dims = (N, Q)
-        if odd:
+        if dups:  # runs of equal keys, 0 and 0xFFFFFFFF in A and in the queries
+            self.A, self.q = inputs.binarysearch_dups(seed, N, Q)
+            self.tag = "-dups"
+        elif odd:
             self.A = (2 * np.arange(N, dtype=np.uint64) + 1).astype(np.uint32)
             self.q = inputs.u32(seed, Q) % np.uint32(2 * N + 8)
         else:
@@ -288,11 +358,15 @@ class Sobel(Case):
 class DCT(Case):
     kernel = "dct"
 
-    def __init__(self, H, W, seed=9):
+    def __init__(self, H, W, seed=9, specials=False):
         self.H, self.W = H, W
         self.n = H * W
         self.dims = (H, W)
         self.X = inputs.dct_x(seed, H, W)
+        if specials:  # NaN and +-0 samples, and one all-(-0) block
+            self.X = inputs.with_specials(self.X, seed, 0.002)
+            self.X[:8, 8:16] = np.float32(-0.0)
+            self.tag = "-specials"
 
     @functools.cached_property
     def X_d(self):
@@ -310,6 +384,14 @@ class DCT(Case):
         got = outs[0].view(np.float32).reshape(H, W).astype(np.float64)
         ref = oracle.dct8x8(X)
         bound = oracle.dct8x8_absbound(X)
+        # NaN inputs: every output of that 8x8 block is NaN on both sides (every
+        # DCT-II coefficient C[u][x] is nonzero); the other blocks as usual
+        nan = np.isnan(ref)
+        assert np.array_equal(np.isnan(got), nan)
+        got = np.where(nan, 0.0, got)
+        ref = np.where(nan, 0.0, ref)
+        bound = np.where(nan, 0.0, bound)
+        X = np.where(np.isnan(X), np.float32(0), X)
         # reading R-DCT3: componentwise condition-scaled 1e-5, and per-block normwise 1e-5
         assert np.all(np.abs(got - ref) <= 1e-5 * bound + 1e-30)
         d = (got - ref).reshape(H // 8, 8, W // 8, 8)
@@ -325,9 +407,11 @@ class DCT(Case):
 class FloydWarshall(Case):
     kernel = "floydwarshall"
 
-    def __init__(self, n, seed=8):
+    def __init__(self, n, seed=8, sparse=None):
         self.n = n
-        self.Wm = inputs.floydwarshall_w(seed, n)
+        # sparse: edge probability; absent edges = FW_INF (reading R-FW1's secondary graph)
+        self.Wm = inputs.floydwarshall_w(seed, n) if sparse is None else inputs.floydwarshall_sparse(seed, n, sparse)
+        self.tag = "" if sparse is None else f"-sparse{sparse}"
 
     @functools.cached_property
     def W_d(self):
@@ -508,16 +592,23 @@ def small_cases():
     """Sizes the oracle finishes in seconds that still span several tiles and a ragged tail."""
     return [
         BlackScholes(1), BlackScholes(7), BlackScholes(1024 * 3 + 5), BlackScholes(1 << 16),
+        BlackScholes(5003, specials=True),
+        BlackScholesIndep(edges=True), BlackScholesIndep(4), BlackScholesIndep(1024 * 3 + 4),
+        BlackScholesIndep(1 << 18),
         Reduction(0), Reduction(3), Reduction(1000003), Reduction(1 << 22),
         Transpose(4, 4), Transpose(68, 132), Transpose(256, 512, index_coded=True), Transpose(1000, 764),
         PrefixSum(1), PrefixSum(4095), PrefixSum(4096 * 37 + 11), PrefixSum(1 << 22), PrefixSum((1 << 25) + 12347),
         FWT(1), FWT(2), FWT(64), FWT(4096), FWT(1 << 13), FWT(1 << 19), FWT(1 << 20), FWT(1 << 16, ternary=True),
+        FWT(1 << 15, specials=True), FWT(64, specials=True),
         BinarySearch(0, 16), BinarySearch(1, 7), BinarySearch(1000, 1003), BinarySearch(1 << 16, 50000, odd=True),
         BinarySearch(1 << 22, 1 << 18), BinarySearch(15, 100, odd=True), BinarySearch(17, 999),
         BinarySearch((1 << 20) + 13, 70001), BinarySearch(4096 + 9, 5000, odd=True),
+        BinarySearch(5, 64, dups=True), BinarySearch(4096 * 3 + 7, 20001, dups=True),
+        BinarySearch((1 << 21) + 5, 1 << 16, dups=True),
         Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
-        DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8),
+        DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8), DCT(64, 512, specials=True),
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
+        FloydWarshall(64, sparse=0.03), FloydWarshall(128, sparse=0.1),
         MatMul(128, 256, 64), MatMul(256, 512, 192, integer=True), MatMul(384, 256, 1024),
         DWT(1), DWT(2), DWT(4), DWT(8), DWT(64), DWT(4096), DWT(8192), DWT(1 << 20), DWT(1 << 23),
         BitonicSort(1), BitonicSort(2), BitonicSort(8), BitonicSort(16), BitonicSort(64, bits=3),

@@ -12,7 +12,7 @@ from helpers import VARIANTS, run
 pytestmark = pytest.mark.gpu
 
 CASES = small_cases()
-IDS = [f"{c.kernel}-{c.n}" for c in CASES]
+IDS = [c.id for c in CASES]
 
 
 def _run_case(case, variant):
@@ -44,7 +44,7 @@ FAULT_CASES = [c for c in CASES if c.n >= 1000]
 
 @pytest.mark.parametrize("variant", rmt.RMT_VARIANTS)
 @pytest.mark.parametrize("replica", [0, 1])
-@pytest.mark.parametrize("case", FAULT_CASES, ids=[f"{c.kernel}-{c.n}" for c in FAULT_CASES])
+@pytest.mark.parametrize("case", FAULT_CASES, ids=[c.id for c in FAULT_CASES])
 def test_store_value_fault_detected(case, replica, variant):
     """A flipped store value in one replica: exactly one mismatching commit, the
     faulted word is not committed (sentinel kept), everything else is clean."""
@@ -82,7 +82,7 @@ def test_store_value_fault_detected(case, replica, variant):
         assert np.array_equal(a, b)
 
 
-@pytest.mark.parametrize("case", FAULT_CASES, ids=[f"{c.kernel}-{c.n}" for c in FAULT_CASES])
+@pytest.mark.parametrize("case", FAULT_CASES, ids=[c.id for c in FAULT_CASES])
 def test_fault_is_live_in_none(case):
     """Liveness control: the same flip in the unprotected kernel corrupts the output."""
     _, ref = _run_case(case, "none")

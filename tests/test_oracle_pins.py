@@ -65,6 +65,43 @@ def test_bs_workload_mapping_and_exact_price():
         assert abs(put[i] - pe) <= 3e-7 * S
 
 
+def test_bs_indep_printed_values():
+    # printed textbook values through the independent-parameter path (R-BS4):
+    # Hull's ATM point and Hull Example 15.6 (S=42, K=40, T=0.5, r=10%, sigma=20%:
+    # c = 4.76, p = 0.81 to the printed 2 decimals)
+    prm = inputs.blackscholes_edges()
+    call, put, _, _ = oracle.blackscholes_indep(prm)
+    assert abs(call[0] - 10.45058) < 1e-4 and abs(put[0] - 5.57353) < 1e-4
+    assert round(call[1], 2) == 4.76 and round(put[1], 2) == 0.81
+
+
+def test_bs_indep_exact_parity_bounds_scale():
+    # independent draws: S != K, d1/d2 of both signs, deep ITM/OTM
+    prm = np.concatenate([inputs.blackscholes_indep(21, 5000), inputs.blackscholes_edges()], axis=1)
+    call, put, cs, ps = oracle.blackscholes_indep(prm)
+    S, K, T, R, V = (prm[k].astype(np.float64) for k in range(5))
+    disc = K * np.exp(-R * T)
+    d1 = (np.log(S / K) + (R + V * V / 2) * T) / (V * np.sqrt(T))
+    assert (d1 < -1).any() and (d1 > 1).any() and (d1 - V * np.sqrt(T) < 0).any()  # both CND branches
+    # put-call parity (exact for any N with N(-x) = 1 - N(x)), and the no-arbitrage bounds
+    assert np.max(np.abs(call - put - (S - disc)) / np.maximum(S, K)) < 1e-12
+    assert np.all(call >= np.maximum(0, S - disc) - 1e-9) and np.all(call <= S + 1e-9)
+    assert np.all(put >= np.maximum(0, disc - S) - 1e-9) and np.all(put <= disc + 1e-9)
+    # against the exact-erfc price (a different CND): the A&S bound 7.5e-8 per N
+    for i in range(0, prm.shape[1], 7):
+        ce, pe = _bs_exact(S[i], K[i], T[i], R[i], V[i])
+        assert abs(call[i] - ce) <= 7.5e-8 * (S[i] + disc[i]) + 1e-12
+        assert abs(put[i] - pe) <= 7.5e-8 * (S[i] + disc[i]) + 1e-12
+    # the conditioning scales bound the prices and the terms
+    assert np.all(cs >= np.abs(call) - 1e-12) and np.all(ps >= np.abs(put) - 1e-12)
+    assert np.all(cs <= S + disc + 1e-9) and np.all(ps <= S + disc + 1e-9)
+    # deep OTM call underflows, deep ITM call = S - K e^{-RT} to within the tail
+    i_otm, i_itm = 3, 7  # BS_EDGE_ROWS: (5, 100, .25, .01, .1) and (5, 1, .25, .05, .1)
+    assert call[prm.shape[1] - inputs.blackscholes_edges().shape[1] + i_otm] < 1e-30
+    j = prm.shape[1] - inputs.blackscholes_edges().shape[1] + i_itm
+    assert abs(call[j] - (S[j] - disc[j])) < 1e-9
+
+
 def test_bs_put_call_parity_and_bounds():
     r = inputs.blackscholes_r(3, 1 << 16)
     call, put = oracle.blackscholes(r)
@@ -104,6 +141,27 @@ def test_binarysearch_vs_searchsorted():
     A, q = inputs.binarysearch_inputs(5, 1 << 18, 1 << 16)
     assert np.all(A[1:] > A[:-1])
     assert np.array_equal(oracle.binarysearch(A, q), np.searchsorted(A, q, side="left").astype(np.uint32))
+
+
+def test_binarysearch_duplicates_and_extremes():
+    # runs of equal keys, 0 and 0xFFFFFFFF in A and in q: lower_bound is the
+    # first index of the run (brute-force count and numpy's side="left")
+    for N, Q in [(1, 50), (5, 64), (300, 2000), (1 << 16, 1 << 14)]:
+        A, q = inputs.binarysearch_dups(N, N, Q)
+        assert np.all(A[1:] >= A[:-1]) and (N < 8 or (A[1:] == A[:-1]).any())
+        idx = oracle.binarysearch(A, q)
+        assert np.array_equal(idx, np.searchsorted(A, q, side="left").astype(np.uint32))
+        if N <= 300:
+            assert np.array_equal(idx, np.array([(A < k).sum() for k in q], np.uint32))
+        # found <=> A[idx] == key, and then idx is the first of its run
+        f = idx < N
+        hit = f.copy()
+        hit[f] = A[idx[f]] == q[f]
+        assert np.all((idx[hit] == 0) | (A[np.maximum(idx[hit].astype(np.int64) - 1, 0)] < q[hit]))
+    A = np.full(10, 0xFFFFFFFF, np.uint32)
+    assert list(oracle.binarysearch(A, np.array([0, 0xFFFFFFFE, 0xFFFFFFFF], np.uint32))) == [0, 0, 0]
+    A = np.zeros(10, np.uint32)
+    assert list(oracle.binarysearch(A, np.array([0, 1, 0xFFFFFFFF], np.uint32))) == [0, 10, 10]
 
 
 # ---------------------------------------------------------------- FastWalshTransform
@@ -273,6 +331,33 @@ def test_floydwarshall_vs_dijkstra_and_invariants():
 def test_floydwarshall_brute_force_paths_tiny():
     n = 6
     Wm = inputs.floydwarshall_w(12, n)
+    D, _ = oracle.floydwarshall(Wm)
+    for i in range(n):
+        for j in range(n):
+            best = int(Wm[i, j]) if i != j else 0
+            others = [v for v in range(n) if v not in (i, j)]
+            for L in range(1, len(others) + 1):
+                for mid in itertools.permutations(others, L):
+                    path = (i,) + mid + (j,)
+                    best = min(best, sum(int(Wm[a, b]) for a, b in zip(path, path[1:])))
+            assert D[i, j] == best
+
+
+def test_floydwarshall_sparse_inf_edges():
+    # absent edges = FW_INF (R-FW1 secondary graph): D rows against Dijkstra,
+    # unreachable pairs keep exactly FW_INF with P = i, brute force on n = 6
+    n = 80
+    Wm = inputs.floydwarshall_sparse(3, n, 0.03)
+    D, P = oracle.floydwarshall(Wm)
+    for s in [0, 1, 40, 79]:
+        assert np.array_equal(D[s], oracle.dijkstra_row(Wm, s))
+    unreach = D >= inputs.FW_INF
+    assert unreach.any() and (~unreach).sum() > n
+    assert np.all(D[unreach] == inputs.FW_INF)
+    rows = np.repeat(np.arange(n, dtype=np.uint32)[:, None], n, axis=1)
+    assert np.array_equal(P[unreach], rows[unreach])
+    n = 6
+    Wm = inputs.floydwarshall_sparse(5, n, 0.4)
     D, _ = oracle.floydwarshall(Wm)
     for i in range(n):
         for j in range(n):
