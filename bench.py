@@ -8,11 +8,18 @@ every kernel of the config launched once under each variant
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config suite] [--impl rmt|reference]
 
-value   = whole-job algorithmic HBM bytes of all launches / max-over-ranks device time
-          (GB/s; inputs resident in HBM; every input > L2, so no flush is needed).
-e2e     = the same metric through rmt_run_host (host pinned buffers; H2D of each
-          launch's inputs and D2H of its outputs inside the timed region).
-slowdown= per kernel t(variant)/t(none) and the geomean per variant.
+value      = the unprotected baseline's aggregate HBM GB/s over the config's kernels:
+             sum of their algorithmic bytes / sum of their `none` launch times
+             (CUDA events inside the timed region, max over ranks; the metric's
+             "baseline HBM GB/s"); inputs resident in HBM, every input > L2.
+slowdown   = per kernel t(variant) / t(none) (median launch time), and the geomean
+             per variant over the config, over all ten BASELINE.json kernels
+             (the configs[1] suite timed in the step + BlackScholes 2^30,
+             FloydWarshall 4096, DCT 8192^2, MatrixMultiplication 16384^3 timed
+             after it) and over SURVEY's memory-bound subset.
+e2e        = the same baseline metric through rmt_run_host_variants (pinned host
+             buffers; per kernel one H2D of its inputs, the four variants, one D2H
+             of the committed outputs and error counts, inside the timed region).
 The reference arm (--impl reference) is the CPU oracle (oracle/), timed as it
 stands on this host's cores on a bounded sample of the same workload.
 """
@@ -22,6 +29,7 @@ import argparse
 import json
 import math
 import os
+import platform
 import statistics
 import sys
 import threading
@@ -34,6 +42,7 @@ METRIC = "RMT slowdown vs unprotected kernel per variant; baseline HBM GB/s vs p
 VARIANTS = ("none", "intra_smem", "intra_reg", "inter_group")
 # B200 extensions: measured after the timed step, not part of it
 EXTRA_VARIANTS = ("inter_cluster", "intra_nolds", "dup_kernel")
+SPEC_HBM_GBS = 8000.0  # BASELINE.json north_star "~8 TB/s" (the >= 70 % target is vs 8 TB/s)
 
 
 # ---------------------------------------------------------------- energy (NVML; Fig. 5)
@@ -79,10 +88,12 @@ def parse():
     p.add_argument("--impl", default="rmt", choices=["rmt", "reference"])
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-rest10", action="store_true",
+                   help="skip the four other BASELINE.json kernels (all-10 slowdown geomean)")
     p.add_argument("--variants", default=",".join(VARIANTS))
     p.add_argument("--extra-variants", default=",".join(EXTRA_VARIANTS),
                    help="variants timed per launch after the timed region (reported, not in the step)")
-    p.add_argument("--energy-seconds", type=float, default=0.5,
+    p.add_argument("--energy-seconds", type=float, default=0.25,
                    help="per (kernel, variant) NVML energy window; 0 disables the energy table")
     p.add_argument("--ablations", action="store_true",
                    help="also time the INFLATE and NOCOMM ablations per kernel x RMT variant (cost attribution)")
@@ -96,7 +107,7 @@ def load_peaks():
     try:
         with open(path) as f:
             pk = json.load(f)
-        return float(pk["hbm_gbs"]), "measured (MEASURED_PEAKS.json)"
+        return float(pk["hbm_gbs"]), "measured copy (MEASURED_PEAKS.json hbm_gbs)"
     except Exception:
         return 6650.0, "fallback (B200_PROFILING.md)"
 
@@ -126,6 +137,11 @@ def load_traffic():
             return json.load(f)
     except Exception:
         return {}
+
+
+def geomean(xs):
+    xs = [x for x in xs if x and x > 0]
+    return round(math.exp(sum(math.log(x) for x in xs) / len(xs)), 3) if xs else None
 
 
 # ---------------------------------------------------------------- clocks (NVML, sampled during the timed region)
@@ -176,87 +192,113 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------- CPU oracle (reference arm / cpu_baseline)
-def oracle_sample_rate(jobs, min_seconds=1.0):
-    """Time the oracle as it stands on a bounded sample of every job; return
-    (equivalent GB/s, seconds, cores, description).  Rates are converted to the
-    GPU metric with each job's full-size algorithmic bytes per unit."""
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return platform.processor() or platform.machine()
+
+
+def oracle_call(j, frac=1.0):
+    """(callable, units, description) timing the oracle on job j, on the first
+    `frac` of its units (frac = 1: the full config size; rows/elements taken from
+    the job's own host inputs)."""
     import numpy as np
 
     import oracle
-    from paper_conf_isca_waddenlgss14_b200 import inputs
+    if j.kernel == "binarysearch":
+        A, q = j.host_in[0], j.host_in[1]
+        q = q[: max(1, int(q.size * frac))]
+        return (lambda: oracle.binarysearch(A, q)), q.size, f"binarysearch Q={q.size} on N={A.size}"
+    if j.kernel == "fwt":
+        m = max(1, int(j.n * frac))
+        m = 1 << (m.bit_length() - 1)
+        x = j.host_in[0][:m]
+        return (lambda: oracle.fwt_f64(x)), x.size, f"fwt N={m}"
+    if j.kernel in ("prefixsum", "reduction"):
+        x = j.host_in[0][: max(1, int(j.n * frac))]
+        fn = oracle.prefixsum_u32 if j.kernel == "prefixsum" else oracle.reduction_u32
+        return (lambda: fn(x)), x.size, f"{j.kernel} n={x.size}"
+    if j.kernel == "transpose":
+        H, W = j.dims
+        h = max(4, int(H * frac))
+        A = np.ascontiguousarray(j.host_in[0].reshape(H, W)[:h])
+        return (lambda: oracle.transpose_u32(A)), A.size, f"transpose {h}x{W}"
+    if j.kernel == "sobel":
+        H, W = j.dims
+        h = max(3, int(H * frac))
+        I = np.ascontiguousarray(j.host_in[0].reshape(H, W)[:h]).view(np.uint8).reshape(h, W, 4)
+        return (lambda: oracle.sobel(I)), h * W, f"sobel {h}x{W}"
+    if j.kernel == "blackscholes":
+        r = j.host_in[0][: max(1, int(j.n * frac))]
+        return (lambda: oracle.blackscholes(r)), r.size, f"blackscholes n={r.size}"
+    if j.kernel == "dct":
+        H, W = j.dims
+        h = max(8, int(H * frac) // 8 * 8)
+        X = np.ascontiguousarray(j.host_in[0].reshape(H, W)[:h])
+        return (lambda: oracle.dct8x8(X)), h * W, f"dct {h}x{W}"
+    return None
 
-    total_bytes_equiv = 0.0
-    total_s = 0.0
-    desc = []
-    for j in jobs:
-        bpu = j.alg_bytes / j.n
-        if j.kernel == "binarysearch":
-            A = j.host_in[0]
-            q = inputs.u32(6, 1 << 20, 0, stream=2)
-            fn, units, what = (lambda: oracle.binarysearch(A, q)), q.size, f"Q=2^20 on N={A.size}"
-        elif j.kernel == "fwt":
-            x = j.host_in[0][: 1 << 22]
-            fn, units, what = (lambda: oracle.fwt_f64(x)), x.size, "N=2^22"
-        elif j.kernel == "prefixsum":
-            x = j.host_in[0][: 1 << 24]
-            fn, units, what = (lambda: oracle.prefixsum_u32(x)), x.size, "n=2^24"
-        elif j.kernel == "reduction":
-            x = j.host_in[0][: 1 << 24]
-            fn, units, what = (lambda: oracle.reduction_u32(x)), x.size, "n=2^24"
-        elif j.kernel == "transpose":
-            H, W = j.dims
-            h = max(4, min(H, (1 << 24) // W))
-            A = np.ascontiguousarray(j.host_in[0].reshape(H, W)[:h])
-            fn, units, what = (lambda: oracle.transpose_u32(A)), A.size, f"{h}x{W}"
-        elif j.kernel == "sobel":
-            H, W = j.dims
-            h = max(3, min(H, (1 << 23) // W))
-            I = np.ascontiguousarray(j.host_in[0].reshape(H, W)[:h]).view(np.uint8).reshape(h, W, 4)
-            fn, units, what = (lambda: oracle.sobel(I)), h * W, f"{h}x{W}"
-        elif j.kernel == "blackscholes":
-            r = j.host_in[0][: 1 << 22]
-            fn, units, what = (lambda: oracle.blackscholes(r)), r.size, f"n={r.size}"
-        elif j.kernel == "dwthaar1d":
-            x = j.host_in[0][: 1 << 22]
-            fn, units, what = (lambda: oracle.dwthaar1d_f64(x)), x.size, "N=2^22"
-        elif j.kernel == "bitonicsort":
-            k = j.host_in[0][: 1 << 22]
-            fn, units, what = (lambda: oracle.sort_u32(k)), k.size, "N=2^22"
-        elif j.kernel == "binomialoption":
-            r = j.host_in[0][: 1 << 12]
-            fn, units, what = (lambda: oracle.binomialoption(r)), r.size, "n=2^12"
-        elif j.kernel == "matmul":
-            # full-K dot products for a 128 x 128 block of C (units = C elements)
-            A, Bt = j.host_in[0], j.host_in[1]
-            M, N, K = j.dims
-            As = np.ascontiguousarray(A.reshape(M, K)[:128])
-            Bs = np.ascontiguousarray(Bt.reshape(N, K)[:128])
-            fn, units, what = (lambda: oracle.matmul_bf16(As, Bs)), 128 * 128, f"C[0:128,0:128] at K={K}"
-        elif j.kernel == "floydwarshall":
-            # the n'^3 relaxations of an n' = 512 sub-problem, converted to the
-            # full problem's units (n^3 relaxations per n nodes)
-            n = j.n
-            m = min(n, 512)
-            Wm = np.ascontiguousarray(j.host_in[0].reshape(n, n)[:m, :m])
-            fn, units, what = (lambda: oracle.floydwarshall(Wm)), m ** 3 / n ** 2, f"n'={m} sub-graph"
-        elif j.kernel == "dct":
-            H, W = j.dims
-            h = max(8, min(H, (1 << 22) // W) // 8 * 8)
-            X = np.ascontiguousarray(j.host_in[0].reshape(H, W)[:h])
-            fn, units, what = (lambda: oracle.dct8x8(X)), h * W, f"{h}x{W}"
-        else:
-            continue
-        reps, t0 = 0, time.perf_counter()
-        while True:
+
+def oracle_rate(jobs, frac=1.0, threads=None):
+    """Time the oracle as it stands on every job (one run each at `frac` of the
+    config size): returns (baseline-equivalent GB/s, seconds, cores, description).
+    Units are converted with each job's algorithmic bytes per unit, so the rate
+    is the GPU line's `value` measure."""
+    import oracle
+    if threads:
+        oracle.set_threads(threads)
+    try:
+        tot_b = tot_s = 0.0
+        desc = []
+        for j in jobs:
+            c = oracle_call(j, frac)
+            if c is None:
+                continue
+            fn, units, what = c
+            t0 = time.perf_counter()
             fn()
-            reps += 1
             dt = time.perf_counter() - t0
-            if dt >= min_seconds:
-                break
-        total_bytes_equiv += reps * units * bpu
-        total_s += dt
-        desc.append(f"{j.kernel} {what} x{reps}")
-    return total_bytes_equiv / total_s / 1e9, total_s, oracle.num_threads(), "; ".join(desc)
+            tot_b += units * (j.alg_bytes / j.n)
+            tot_s += dt
+            desc.append(f"{what} {dt:.2f}s")
+        return tot_b / tot_s / 1e9, tot_s, oracle.num_threads(), "; ".join(desc)
+    finally:
+        if threads:
+            oracle.set_threads(os.cpu_count() or 1)
+
+
+# ---------------------------------------------------------------- reference arm
+def reference_arm(args, rank):
+    if rank != 0:
+        return  # rank 0 alone runs the CPU reference arm
+    from paper_conf_isca_waddenlgss14_b200 import workloads
+    jobs = workloads.config_jobs(args.config, 0)
+    frac = 1.0 / 16  # each step: a bounded 1/16 sample of every kernel of the config
+    for _ in range(args.warmup):
+        oracle_rate(jobs, frac / 4)
+    rates, times = [], []
+    desc, cores = "", 0
+    for _ in range(args.steps):
+        rate, secs, cores, desc = oracle_rate(jobs, frac)
+        rates.append(rate)
+        times.append(secs)
+    rate = statistics.median(rates)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(rate, 3), "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(1e3 * statistics.mean(times), 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32/u8x4", "data": "synthetic",
+        "config": {"workload": workloads.CONFIG_TITLES[args.config], "preset": args.config},
+        "cpu_baseline": {"value": round(rate, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
+                         "sample": f"1/16 of every kernel per step: {desc}", "cpu": cpu_model()},
+        "e2e": {"value": round(rate, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
 
 
 # ---------------------------------------------------------------- main
@@ -265,37 +307,13 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-
-    from paper_conf_isca_waddenlgss14_b200 import workloads
-
     if args.impl == "reference":
-        if rank != 0:
-            return  # rank 0 alone runs the CPU reference arm
-        jobs = workloads.config_jobs(args.config, 0)
-        for _ in range(args.warmup):
-            pass
-        times = []
-        rate = None
-        for _ in range(args.steps):
-            rate, secs, cores, desc = oracle_sample_rate(jobs, min_seconds=0.5)
-            times.append(secs)
-        line = {
-            "impl": "reference", "metric": METRIC, "value": round(rate, 3), "unit": "GB/s",
-            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(1e3 * statistics.mean(times), 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32", "data": "synthetic",
-            "config": {"workload": workloads.CONFIG_TITLES[args.config], "preset": args.config},
-            "cpu_baseline": {"value": round(rate, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
-                             "sample": desc},
-            "e2e": {"value": round(rate, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-        }
-        print(json.dumps(line), flush=True)
-        return
+        return reference_arm(args, rank)
 
     import torch
     import torch.distributed as dist
 
-    from paper_conf_isca_waddenlgss14_b200 import rmt
+    from paper_conf_isca_waddenlgss14_b200 import parallel, rmt, workloads
 
     dev_index = local_rank % max(1, torch.cuda.device_count())
     torch.cuda.set_device(dev_index)
@@ -321,8 +339,6 @@ def main():
     launches = [(j, v) for j in jobs for v in variants]
     ev = {(j.kernel, v): [] for j, v in launches}
     counts = {"gpu_launches": 0}
-
-    from paper_conf_isca_waddenlgss14_b200 import parallel
     s_tmp = torch.zeros(2, dtype=torch.int32, device="cuda")
 
     def one(j, v):
@@ -350,8 +366,6 @@ def main():
                 b.record(stream)
                 ev[(j.kernel, v)].append((a, b))
                 counts["gpu_launches"] += nk
-        if world > 1:
-            parallel.allreduce_sum_(err)  # error counters of every rank
 
     for _ in range(args.warmup):
         step(False)
@@ -371,24 +385,25 @@ def main():
     if world > 1:
         dist.barrier()
     ms_total = t0.elapsed_time(t1)
+    # device time of every `none` launch in the timed region (the baseline metric)
+    none_ms = sum(a.elapsed_time(b) for (k, v), lst in ev.items() if v == "none" for a, b in lst)
     if world > 1:
-        tt = torch.tensor([ms_total], dtype=torch.float64, device="cuda")
+        tt = torch.tensor([ms_total, none_ms], dtype=torch.float64, device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms_total = float(tt.item())
+        ms_total, none_ms = float(tt[0].item()), float(tt[1].item())
+        parallel.allreduce_sum_(err)  # error counters of every rank, once for the whole timed region
     errs = int(err.item())
 
     # per-launch device times
-    per = {}
-    for (k, v), lst in ev.items():
-        per[(k, v)] = statistics.median(a.elapsed_time(b) for a, b in lst)
+    per = {(k, v): statistics.median(a.elapsed_time(b) for a, b in lst) for (k, v), lst in ev.items()}
     peak, peak_src = load_peaks()
+    none_bytes = sum(j.alg_bytes for j in jobs) if "none" in variants else 0
+    value = none_bytes * args.steps * world / (none_ms * 1e-3) / 1e9 if none_ms else None
     step_bytes = sum(j.alg_bytes for j, _ in launches)
-    value = step_bytes * args.steps * world / (ms_total * 1e-3) / 1e9
 
     kernels = {}
-    slow = {v: [] for v in variants if v != "none"}
     for j in jobs:
-        d = {}
+        d = {"bound": j.bound}
         for v in variants:
             ms = per[(j.kernel, v)]
             gbs = j.alg_bytes / (ms * 1e-3) / 1e9
@@ -398,58 +413,122 @@ def main():
                 d[v]["tflops"] = round(tf, 1)
                 d[v]["tensor_frac"] = round(tf / load_tensor_peak()[0], 4)
             if v != "none" and "none" in variants:
-                sd = ms / per[(j.kernel, "none")]
-                d[v]["slowdown"] = round(sd, 3)
-                slow[v].append(sd)
-        d["bound"] = j.bound
+                d[v]["slowdown"] = round(ms / per[(j.kernel, "none")], 3)
         kernels[j.kernel] = d
-    geo = {v: round(math.exp(sum(math.log(x) for x in s) / len(s)), 3) for v, s in slow.items() if s}
-    geo_mem = {}
-    for v, s in slow.items():
-        mem = [per[(j.kernel, v)] / per[(j.kernel, "none")] for j in jobs if j.bound == "hbm"]
-        if mem:
-            geo_mem[v] = round(math.exp(sum(math.log(x) for x in mem) / len(mem)), 3)
+
+    # ---- the four other BASELINE.json kernels (per-launch medians after the step)
+    rest = {}
+    if not args.no_rest10 and args.config == "suite" and "none" in variants:
+        err_r = torch.zeros(1, dtype=torch.int64, device="cuda")
+        for j in workloads.config_jobs("rest10", rank):
+            j.device_buffers()
+            d = {"bound": j.bound}
+            for v in variants:
+                w = rmt.make_workspace(j.kernel, v, j.n, j.dims)
+                reps = 2 if j.kernel == "floydwarshall" and v == "inter_group" else 3
+                ts = []
+                for r in range(reps + 1):
+                    if j.kernel == "floydwarshall":  # D is in/out: every launch restarts from W
+                        j.dev[0].copy_(torch.from_numpy(j.host_in[0].view("int32").reshape(-1)).cuda())
+                    a = torch.cuda.Event(enable_timing=True)
+                    b = torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
+                    rmt.launch(j.kernel, v, j.dev, j.n, err_r, dims=j.dims, workspace=w, stream=stream.cuda_stream)
+                    b.record(stream)
+                    torch.cuda.synchronize()
+                    if r:
+                        ts.append(a.elapsed_time(b))
+                ms = statistics.median(ts)
+                gbs = j.alg_bytes / (ms * 1e-3) / 1e9
+                d[v] = {"ms": round(ms, 4), "gbs": round(gbs, 1), "frac": round(gbs / peak, 4)}
+                if job_flops(j):
+                    tf = job_flops(j) / (ms * 1e-3) / 1e12
+                    d[v]["tflops"] = round(tf, 1)
+                    d[v]["tensor_frac"] = round(tf / load_tensor_peak()[0], 4)
+                del w
+            for v in variants:
+                if v != "none":
+                    d[v]["slowdown"] = round(d[v]["ms"] / d["none"]["ms"], 3)
+            d["mem_subset"] = j.mem_subset
+            rest[j.kernel] = d
+            j.dev = None
+            torch.cuda.empty_cache()
+        rest["err_count"] = int(err_r.item())
+
+    all_k = dict(kernels)
+    all_k.update({k: d for k, d in rest.items() if isinstance(d, dict)})
+    mem_kernels = {"reduction", "transpose", "sobel", "prefixsum", "fwt", "dct"}
+    slowdown_geomean = {}
+    for v in variants:
+        if v == "none":
+            continue
+        slowdown_geomean[v] = {
+            "config": geomean([kernels[k][v]["slowdown"] for k in kernels]),
+            "all10": geomean([all_k[k][v]["slowdown"] for k in all_k]) if rest else None,
+            "mem_subset": geomean([all_k[k][v]["slowdown"] for k in all_k if k in mem_kernels]),
+            "kernels": sorted(all_k),
+        }
+    baseline_frac = {}
+    for k, d in all_k.items():
+        if "none" not in d:
+            continue
+        g = d["none"]["gbs"]
+        e = {"gbs": g, "vs_8tbps": round(g / SPEC_HBM_GBS, 4), "vs_copy_peak": round(g / peak, 4),
+             "bound": d["bound"], "target_applies": k in mem_kernels}
+        if "tflops" in d["none"]:
+            e["tflops"] = d["none"]["tflops"]
+            e["tensor_frac"] = d["none"]["tensor_frac"]
+        baseline_frac[k] = e
 
     # dominant kernel (largest share of the step) -> roofline
-    dom = max(launches, key=lambda jv: per[(jv[0].kernel, jv[1])])
-    dj, dv = dom
+    dj, dv = max(launches, key=lambda jv: per[(jv[0].kernel, jv[1])])
     dms = per[(dj.kernel, dv)]
     ach = dj.alg_bytes / (dms * 1e-3) / 1e9
     traffic = load_traffic().get(f"{dj.kernel}/{dv}")
     roofline = {"bound": "hbm", "achieved": round(ach, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(ach / peak, 4), "traffic": traffic, "kernel": f"{dj.kernel}/{dv}",
-                "share_of_step": round(dms / (ms_total / args.steps), 3), "peak_source": peak_src,
-                "algorithmic_bytes_per_launch": dj.alg_bytes}
+                "kernel_bound_class": dj.bound,
+                "share_of_step": round(dms * args.steps / ms_total, 3), "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": dj.alg_bytes, "bytes_per_unit": round(dj.alg_bytes / dj.n, 3),
+                "units_per_launch": dj.n}
     if dj.bound == "tensor" and job_flops(dj):
         tpk, tsrc = load_tensor_peak()
         tach = job_flops(dj) / (dms * 1e-3) / 1e12
         roofline.update({"bound": "tensor", "achieved": round(tach, 1), "peak": tpk, "unit": "TFLOP/s",
                          "frac": round(tach / tpk, 4), "peak_source": tsrc,
-                         "algorithmic_flops_per_launch": job_flops(dj),
-                         "note": "both replicas run the full contraction on the tensor pipe; achieved counts "
-                                 "the algorithmic 2MNK once"})
-    best_none = max((j for j in jobs if j.bound == "hbm"), key=lambda j: j.alg_bytes / per[(j.kernel, "none")],
-                    default=None)
+                         "algorithmic_flops_per_launch": job_flops(dj)})
 
-    # end-to-end through the public C ABI with host buffers
+    # ---- end to end through the public C ABI with host buffers
     e2e = None
-    if args.e2e_steps > 0:
+    if args.e2e_steps > 0 and all(j.host_inputs for j in jobs):
         hosts = {j.kernel: j.pinned_host() for j in jobs}
-        h2d = d2h = 0
-        for j, v in launches:  # warm
-            rmt.run_host(j.kernel, v, hosts[j.kernel], j.dev, j.n, err, dims=j.dims, workspace=ws[(j.kernel, v)])
+        err_v = torch.zeros(len(variants), dtype=torch.int64, device="cuda")
+        wsl = {j.kernel: [ws[(j.kernel, v)] for v in variants] for j in jobs}
+
+        def e2e_step():
+            hb = db = 0
+            e_all = 0
+            for j in jobs:
+                errs_v, h, d_ = rmt.run_host_variants(j.kernel, variants, hosts[j.kernel], j.dev, j.n, err_v,
+                                                      wsl[j.kernel], dims=j.dims)
+                hb += h
+                db += d_
+                e_all += sum(errs_v)
+            return hb, db, e_all
+
+        e2e_step()  # warm
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
+        h2d = d2h = e2e_err = 0
         e0.record(stream)
         for _ in range(args.e2e_steps):
-            for j, v in launches:
-                _, hb, db = rmt.run_host(j.kernel, v, hosts[j.kernel], j.dev, j.n, err, dims=j.dims,
-                                         workspace=ws[(j.kernel, v)])
-                h2d += hb
-                d2h += db
+            hb, db, ee = e2e_step()
+            h2d += hb
+            d2h += db
+            e2e_err += ee
         e1.record(stream)
         torch.cuda.synchronize()
         ems = e0.elapsed_time(e1)
@@ -457,13 +536,15 @@ def main():
             tt = torch.tensor([ems], dtype=torch.float64, device="cuda")
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ems = float(tt.item())
-        e2e = {"value": round(step_bytes * args.e2e_steps * world / (ems * 1e-3) / 1e9, 3), "unit": "GB/s",
+        # the baseline metric end to end: the unprotected bytes over the wall of the
+        # whole host-buffer step (copies + every variant)
+        e2e = {"value": round(none_bytes * args.e2e_steps * world / (ems * 1e-3) / 1e9, 3), "unit": "GB/s",
                "h2d_bytes_per_step": h2d // args.e2e_steps, "d2h_bytes_per_step": d2h // args.e2e_steps,
-               "ms_per_step": round(ems / args.e2e_steps, 3)}
+               "ms_per_step": round(ems / args.e2e_steps, 3), "err_count": e2e_err,
+               "note": "per kernel: one H2D of its inputs, the variants, one D2H of the committed outputs and "
+                       "error counts (rmt_run_host_variants)"}
 
-    # Cost attribution "as the paper does": t(none) ->
-    # inflate (none with the RMT variant's per-SM residency: redundant scheduling)
-    # -> nocomm (both replicas, no exchange: redundant compute) -> full (+ comm).
+    # ---- cost attribution "as the paper does"
     attribution = None
     if args.ablations:
         attribution = {}
@@ -495,13 +576,13 @@ def main():
             attribution[j.kernel] = d
         err.zero_()
 
-    # B200-native extension variants: per-launch medians outside the timed step
+    # ---- B200-native extension variants: per-launch medians outside the timed step
     extra = None
     xvars = [v for v in args.extra_variants.split(",") if v and v not in variants]
     if xvars and "none" in variants:
         extra = {"kernels": {}, "slowdown_geomean": {}}
         xs = {v: [] for v in xvars}
-        err.zero_()
+        err_x = torch.zeros(1, dtype=torch.int64, device="cuda")
         for j in jobs:
             d = {}
             for v in xvars:
@@ -511,7 +592,7 @@ def main():
                     a = torch.cuda.Event(enable_timing=True)
                     b = torch.cuda.Event(enable_timing=True)
                     a.record(stream)
-                    rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=wsx, stream=stream.cuda_stream)
+                    rmt.launch(j.kernel, v, j.dev, j.n, err_x, dims=j.dims, workspace=wsx, stream=stream.cuda_stream)
                     b.record(stream)
                     torch.cuda.synchronize()
                     if r:
@@ -522,22 +603,22 @@ def main():
                 xs[v].append(sd)
                 del wsx
             extra["kernels"][j.kernel] = d
-        extra["slowdown_geomean"] = {v: round(math.exp(sum(math.log(x) for x in s_) / len(s_)), 3)
-                                     for v, s_ in xs.items()}
-        extra["err_count"] = int(err.item())
+        extra["slowdown_geomean"] = {v: geomean(s_) for v, s_ in xs.items()}
+        extra["err_count"] = int(err_x.item())
 
-    # average power and energy per launch for every kernel x variant
+    # ---- average power and energy per launch for every kernel x variant
     energy = None
     if args.energy_seconds > 0 and world == 1:
         energy = {}
         allv = variants + [v for v in args.extra_variants.split(",") if v and v not in variants]
+        err_e = torch.zeros(1, dtype=torch.int64, device="cuda")
         for j in jobs:
             d = {}
             for v in allv:
                 wsx = ws.get((j.kernel, v))
                 if wsx is None:
                     wsx = rmt.make_workspace(j.kernel, v, j.n, j.dims)
-                r = measure_energy(dev_index, lambda: rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims,
+                r = measure_energy(dev_index, lambda: rmt.launch(j.kernel, v, j.dev, j.n, err_e, dims=j.dims,
                                                                  workspace=wsx, stream=stream.cuda_stream),
                                    args.energy_seconds)
                 if r is None:
@@ -548,27 +629,32 @@ def main():
                 energy = None
                 break
             energy[j.kernel] = d
-        err.zero_()
 
+    # ---- the oracle on this host: the full config, all cores; and one thread at <= 2^24 units
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        rate, secs, cores, desc = oracle_sample_rate(jobs)
-        cpu = {"value": round(rate, 3), "unit": "GB/s", "cores": cores, "kind": "oracle", "sample": desc,
-               "seconds": round(secs, 2)}
+        rate, secs, cores, desc = oracle_rate(jobs, 1.0)
+        frac1 = min(1.0, min((1 << 24) / j.n for j in jobs))
+        rate1, secs1, _, desc1 = oracle_rate(jobs, frac1, threads=1)
+        cpu = {"value": round(rate, 3), "unit": "GB/s", "cores": cores, "kind": "oracle",
+               "sample": f"the full config, one run per kernel: {desc}", "seconds": round(secs, 2),
+               "cpu": cpu_model(), "affinity_cores": len(os.sched_getaffinity(0)),
+               "one_thread": {"value": round(rate1, 3), "unit": "GB/s", "cores": 1,
+                              "sample": f"{frac1:.4g} of every kernel: {desc1}", "seconds": round(secs1, 2)}}
 
     if rank == 0:
         line = {
-            "metric": METRIC, "value": round(value, 1), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms_total / args.steps, 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32/u8x4", "data": "synthetic",
+            "metric": METRIC, "value": round(value, 1) if value else None, "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_total / args.steps, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32/u8x4",
+            "data": "synthetic",
             "config": {"workload": workloads.CONFIG_TITLES[args.config], "preset": args.config,
                        "variants": variants, "l2": "every input > 126 MB L2 (no flush needed)",
-                       "parallelism": f"dp{world} (data-sharded, weak)"},
-            "slowdown_geomean": geo, "slowdown_geomean_hbm_kernels": geo_mem,
-            "baseline_best": ({"kernel": best_none.kernel,
-                               "gbs": kernels[best_none.kernel]["none"]["gbs"],
-                               "frac": kernels[best_none.kernel]["none"]["frac"]} if best_none else None),
-            "kernels": kernels, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                       "parallelism": f"dp{world} (data-sharded, weak)",
+                       "value": "baseline (none) HBM GB/s: sum of algorithmic bytes / sum of none launch times"},
+            "step_gbs_all_variants": round(step_bytes * args.steps * world / (ms_total * 1e-3) / 1e9, 1),
+            "slowdown_geomean": slowdown_geomean, "baseline_frac": baseline_frac,
+            "kernels": kernels, "rest10": rest or None, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "attribution": attribution, "extra_variants": extra, "energy": energy,
             "gpu_launches": counts["gpu_launches"], "err_count": errs,
             "clocks": clk.summary(),

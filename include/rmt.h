@@ -192,6 +192,22 @@ int rmt_run_host(int kernel, int variant, const rmt_bufs_t* host, const rmt_bufs
                  unsigned long long* err_host, unsigned long long* err_dev, void* workspace,
                  size_t ws_bytes, void* stream, int64_t* h2d_bytes, int64_t* d2h_bytes);
 
+/*
+ * rmt_run_host_variants -- the end-to-end call for one kernel under several
+ * variants (e.g. the unprotected baseline and each RMT variant, as bench.py's
+ * e2e leg runs them): copy the INPUT buffers host->device once (an in/out
+ * buffer, FloydWarshall's D, again before every variant), launch variant
+ * variants[v] with its own error counter err_dev[v] (device u64[nvar], zeroed
+ * here) and workspace workspaces[v] (ws_bytes[v] bytes), copy the OUTPUT buffers
+ * back once after the last launch (every variant commits the same bits) and the
+ * nvar error counts into err_host[nvar], then synchronise `stream`.  Returns as
+ * rmt_launch; *h2d_bytes / *d2h_bytes (nullable) receive the bytes copied.
+ */
+int rmt_run_host_variants(int kernel, int nvar, const int* variants, const rmt_bufs_t* host, const rmt_bufs_t* dev,
+                          int64_t n, unsigned long long* err_host, unsigned long long* err_dev,
+                          void* const* workspaces, const size_t* ws_bytes, void* stream, int64_t* h2d_bytes,
+                          int64_t* d2h_bytes);
+
 /* Fault injection (BASELINE.json north_star item (4)): arm ONE single-bit flip
  * for subsequent launches until rmt_clear_faults().
  *   replica  0|1 (intra: 0 = even lane = consumer, 1 = odd lane = producer;

@@ -44,6 +44,7 @@ def lib():
         I = ctypes.c_int64
         D = ctypes.c_double
         L.orc_num_threads.restype = ctypes.c_int
+        L.orc_set_threads.argtypes = [ctypes.c_int]
         L.orc_cnd.argtypes = [D]
         L.orc_cnd.restype = D
         L.orc_bs_price.argtypes = [D, D, D, D, D, P, P]
@@ -81,6 +82,10 @@ def _p(a: np.ndarray):
 
 def num_threads() -> int:
     return lib().orc_num_threads()
+
+
+def set_threads(n: int) -> None:
+    lib().orc_set_threads(int(n))
 
 
 def cnd(x: float) -> float:

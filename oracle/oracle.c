@@ -40,6 +40,15 @@ int orc_num_threads(void) {
 #endif
 }
 
+/* Thread count for the timing legs (bench.py's 1-thread cpu_baseline run). */
+void orc_set_threads(int n) {
+#ifdef _OPENMP
+    omp_set_num_threads(n > 0 ? n : 1);
+#else
+    (void)n;
+#endif
+}
+
 /* ------------------------------------------------------------------------ */
 /* BlackScholes  (P:157 / Fig.2 "BlkSch"; R-BS1 input mapping, R-BS2 CND)    */
 /* ------------------------------------------------------------------------ */

@@ -291,6 +291,58 @@ int rmt_run_host(int kernel, int variant, const rmt_bufs_t* host, const rmt_bufs
   return RMT_OK;
 }
 
+int rmt_run_host_variants(int kernel, int nvar, const int* variants, const rmt_bufs_t* host, const rmt_bufs_t* dev,
+                          int64_t n, unsigned long long* err_host, unsigned long long* err_dev,
+                          void* const* workspaces, const size_t* ws_bytes, void* stream, int64_t* h2d_bytes,
+                          int64_t* d2h_bytes) {
+  if (kernel < 0 || kernel >= RMT_K_COUNT || nvar < 1 || !variants || !host || !dev || !err_host || !err_dev ||
+      !workspaces || !ws_bytes) {
+    set_error("rmt_run_host_variants: bad arguments");
+    return RMT_EINVAL;
+  }
+  const KEntry& e = kTable[kernel];
+  cudaStream_t s = (cudaStream_t)stream;
+  int64_t hb = 0, db = 0;
+  int rc;
+  auto is_out = [&](int bi) {
+    for (int k = 0; k < e.nout; ++k)
+      if (e.out[k] == bi) return true;
+    return false;
+  };
+  for (int v = 0; v < nvar; ++v) {
+    // inputs: once; an in/out buffer (FloydWarshall's D) again before every variant
+    for (int i = 0; i < e.nin; ++i) {
+      const int bi = e.in[i];
+      if (v > 0 && !is_out(bi)) continue;
+      const rmt_buf_t& h = host->buf[bi];
+      const rmt_buf_t& d = dev->buf[bi];
+      if (!h.ptr || h.numel != d.numel || h.dtype != d.dtype) { set_error("host/dev schema mismatch"); return RMT_EINVAL; }
+      size_t bytes = (size_t)h.numel * dtype_bytes(h.dtype);
+      if ((rc = cuda_check(cudaMemcpyAsync(d.ptr, h.ptr, bytes, cudaMemcpyHostToDevice, s), "H2D"))) return rc;
+      hb += (int64_t)bytes;
+    }
+    if ((rc = cuda_check(cudaMemsetAsync(err_dev + v, 0, sizeof(unsigned long long), s), "memset err"))) return rc;
+    rc = rmt_launch(kernel, variants[v], dev, n, err_dev + v, workspaces[v], ws_bytes[v], stream);
+    if (rc) return rc;
+  }
+  // the committed outputs (every variant writes the same bits) and every error count
+  for (int i = 0; i < e.nout; ++i) {
+    const rmt_buf_t& h = host->buf[e.out[i]];
+    const rmt_buf_t& d = dev->buf[e.out[i]];
+    if (!h.ptr || h.numel != d.numel) { set_error("host/dev schema mismatch"); return RMT_EINVAL; }
+    size_t bytes = (size_t)h.numel * dtype_bytes(h.dtype);
+    if ((rc = cuda_check(cudaMemcpyAsync(h.ptr, d.ptr, bytes, cudaMemcpyDeviceToHost, s), "D2H"))) return rc;
+    db += (int64_t)bytes;
+  }
+  if ((rc = cuda_check(cudaMemcpyAsync(err_host, err_dev, 8 * (size_t)nvar, cudaMemcpyDeviceToHost, s), "D2H err")))
+    return rc;
+  db += 8 * nvar;
+  if ((rc = cuda_check(cudaStreamSynchronize(s), "stream sync"))) return rc;
+  if (h2d_bytes) *h2d_bytes = hb;
+  if (d2h_bytes) *d2h_bytes = db;
+  return RMT_OK;
+}
+
 int rmt_inject_fault(int replica, int site, int bit, int64_t elem) {
   if (replica < 0 || replica > 1 || site < RMT_SITE_LOAD || site > RMT_SITE_STORE_ADDR || bit < 0 || bit > 31 ||
       elem < 0) {

@@ -260,3 +260,70 @@ def dwt_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
 def binomial_r(seed: int, n: int, offset: int = 0) -> np.ndarray:
     """One U[0,1) draw per option (APP-SDK style; the kernel maps r -> S, K, T)."""
     return uniform_f32(seed, n, offset, stream=12)
+
+
+# --------------------------------------------------------------------------
+# Device-side twins of the generators above (torch tensor ops, no method
+# arithmetic): the same splitmix64 counter stream, bit for bit, produced in HBM
+# for the bench's largest inputs (BlackScholes 2^30 options, MatrixMultiplication
+# 16384^2 operands) where host generation would take minutes.
+# tests/test_inputs_cpu.py pins u64_t / uniform_f32_t against the numpy versions.
+# --------------------------------------------------------------------------
+
+def _srl(z, k: int):
+    """Logical right shift of int64 tensors holding uint64 bit patterns."""
+    import torch
+    return (z >> k) & ((1 << (64 - k)) - 1)
+
+
+def _mix_t(z):
+    M1 = 0xBF58476D1CE4E5B9 - (1 << 64)  # the same constants as int64 bit patterns
+    M2 = 0x94D049BB133111EB - (1 << 64)
+    z = (z ^ _srl(z, 30)) * M1
+    z = (z ^ _srl(z, 27)) * M2
+    return z ^ _srl(z, 31)
+
+
+def u64_t(seed: int, n: int, offset: int = 0, stream: int = 0, device="cuda"):
+    """int64 tensor with the bit patterns of u64(seed, n, offset, stream)."""
+    import torch
+    key = int(_mix(np.array([(seed * 0x100000001B3 + stream * 0x1000193 + 1) & (2**64 - 1)], dtype=np.uint64))[0])
+    key = key - (1 << 64) if key >= (1 << 63) else key
+    gold = 0x9E3779B97F4A7C15 - (1 << 64)
+    out = torch.empty(n, dtype=torch.int64, device=device)
+    for s in range(0, n, _CHUNK):
+        e = min(n, s + _CHUNK)
+        idx = torch.arange(offset + s, offset + e, dtype=torch.int64, device=device)
+        out[s:e] = _mix_t(idx * gold + key)
+    return out
+
+
+def uniform_f32_t(seed: int, n: int, offset: int = 0, stream: int = 0, device="cuda"):
+    import torch
+    out = torch.empty(n, dtype=torch.float32, device=device)
+    for s in range(0, n, _CHUNK):
+        e = min(n, s + _CHUNK)
+        k = _srl(u64_t(seed, e - s, offset + s, stream, device), 40).to(torch.float64)
+        out[s:e] = (k * (2.0 ** -24)).to(torch.float32)
+    return out
+
+
+def blackscholes_r_t(seed: int, n: int, offset: int = 0, device="cuda"):
+    return uniform_f32_t(seed, n, offset, 0, device)
+
+
+def matmul_bf16_normal_t(seed: int, rows: int, cols: int, stream: int, row_offset: int = 0, device="cuda"):
+    """bf16 N(0,1) on the device (Box-Muller on the same two counter streams as
+    matmul_bf16_normal; the device log/cos may round a rare value differently
+    from numpy's), returned as an int16 tensor of bf16 bit patterns."""
+    import torch
+    n = rows * cols
+    off = row_offset * cols
+    out = torch.empty(n, dtype=torch.bfloat16, device=device)
+    for s in range(0, n, _CHUNK):
+        e = min(n, s + _CHUNK)
+        u1 = _srl(u64_t(seed, e - s, off + s, stream, device), 11).to(torch.float64) * 2.0 ** -53
+        u2 = _srl(u64_t(seed, e - s, off + s, stream + 1, device), 11).to(torch.float64) * 2.0 ** -53
+        g = torch.sqrt(-2.0 * torch.log1p(-u1)) * torch.cos(2.0 * np.pi * u2)
+        out[s:e] = g.to(torch.float32).to(torch.bfloat16)
+    return out.view(torch.int16)

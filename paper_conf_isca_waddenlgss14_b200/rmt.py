@@ -76,6 +76,11 @@ def lib() -> ctypes.CDLL:
         L.rmt_run_host.argtypes = [I32, I32, ctypes.POINTER(_Bufs), ctypes.POINTER(_Bufs), I64, P, P, P, SZ, P,
                                    ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]
         L.rmt_run_host.restype = I32
+        L.rmt_run_host_variants.argtypes = [I32, I32, ctypes.POINTER(I32), ctypes.POINTER(_Bufs),
+                                            ctypes.POINTER(_Bufs), I64, P, P, ctypes.POINTER(P),
+                                            ctypes.POINTER(SZ), P, ctypes.POINTER(ctypes.c_int64),
+                                            ctypes.POINTER(ctypes.c_int64)]
+        L.rmt_run_host_variants.restype = I32
         L.rmt_inject_fault.argtypes = [I32, I32, I32, I64]
         L.rmt_inject_fault.restype = I32
         L.rmt_clear_faults.restype = I32
@@ -177,6 +182,28 @@ def run_host(kernel: str, variant: str, host, dev, n: int, err_dev, dims=(), wor
                               ctypes.byref(e), err_dev.data_ptr(), ws_ptr, ws_bytes, stream,
                               ctypes.byref(h2d), ctypes.byref(d2h)), f"rmt_run_host({kernel},{variant})")
     return e.value, h2d.value, d2h.value
+
+
+def run_host_variants(kernel: str, variants, host, dev, n: int, err_dev, workspaces, dims=(), stream=None):
+    """rmt_run_host_variants: H2D of the inputs once, one launch per variant
+    (each with its own device error counter err_dev[v] and workspace), D2H of
+    the outputs once and of every error count, sync.  err_dev: int64 device
+    tensor [len(variants)].  Returns (error counts, h2d_bytes, d2h_bytes)."""
+    if stream is None:
+        stream = torch.cuda.current_stream().cuda_stream
+    nv = len(variants)
+    hb = make_bufs(kernel, host, dims)
+    db = make_bufs(kernel, dev, dims)
+    vids = (ctypes.c_int * nv)(*[VARIANTS[v] for v in variants])
+    errs = (ctypes.c_ulonglong * nv)()
+    wsp = (ctypes.c_void_p * nv)(*[w.data_ptr() if w is not None else None for w in workspaces])
+    wsb = (ctypes.c_size_t * nv)(*[w.numel() if w is not None else 0 for w in workspaces])
+    h2d = ctypes.c_int64(0)
+    d2h = ctypes.c_int64(0)
+    _check(lib().rmt_run_host_variants(KERNELS[kernel], nv, vids, ctypes.byref(hb), ctypes.byref(db), int(n),
+                                       errs, err_dev.data_ptr(), wsp, wsb, stream, ctypes.byref(h2d),
+                                       ctypes.byref(d2h)), f"rmt_run_host_variants({kernel})")
+    return list(errs), h2d.value, d2h.value
 
 
 def inject_fault(replica: int, site, bit: int, elem: int):

@@ -1,10 +1,16 @@
 """Benchmark workloads: BASELINE.json configs as named presets.
 
 A Job is one kernel at one size: host inputs (numpy, from the seeded
-generators in inputs.py), device buffers in schema order, and the kernel's
-algorithmic HBM bytes per launch (SURVEY 8(d) / DESIGN.md "Roofline").  No
-method arithmetic lives here.  Shards: rank r of G takes rows/elements
-[r*n, (r+1)*n) of the global index space (weak scaling: fixed per-GPU size).
+generators in inputs.py) or a device-side generator for the largest inputs,
+device buffers in schema order, and the kernel's algorithmic HBM bytes per
+launch (SURVEY 8(d) / DESIGN.md section 7).  No method arithmetic lives here.
+Shards: rank r of G takes rows/elements [r*n, (r+1)*n) of the global index
+space (weak scaling: fixed per-GPU size).
+
+`bound` is the roofline class SURVEY 8(d) assigns (SURVEY.md:548-552): "hbm"
+(streaming; the >= 70 % target applies), "latency" (BinarySearch: random
+sectors), "mufu" (BlackScholes: MUFU ~ HBM), "l2" (FloydWarshall: the matrix
+stays L2-resident), "tensor" (MatrixMultiplication), "alu" (BinomialOption).
 """
 from __future__ import annotations
 
@@ -30,19 +36,31 @@ class Job:
     bound: str = "hbm"
     note: str = ""
     dev: list | None = None
+    dev_gen: object = None  # callable(i) -> device tensor of input i (instead of host_in[i])
+
+    @property
+    def mem_subset(self) -> bool:
+        """The survey's memory-bound subset (SURVEY.md:548): R, T, Sobel, PS, FWT, DCT."""
+        return self.kernel in ("reduction", "transpose", "sobel", "prefixsum", "fwt", "dct")
 
     def device_buffers(self):
-        """Allocate device buffers once (inputs copied, outputs zeroed)."""
+        """Allocate device buffers once (inputs copied or generated in HBM, outputs zeroed)."""
         if self.dev is None:
             bufs = []
             for i, h in enumerate(self.host_in):
                 if h is not None:
                     bufs.append(_to_dev(h))
+                elif i not in dict(self.out_shapes):
+                    bufs.append(self.dev_gen(i))
                 else:
                     nbytes = dict(self.out_shapes)[i]
                     bufs.append(torch.zeros(max(nbytes // 4, 4), dtype=torch.int32, device="cuda")[: nbytes // 4])
             self.dev = bufs
         return self.dev
+
+    @property
+    def host_inputs(self) -> bool:
+        return all(h is not None for i, h in enumerate(self.host_in) if i not in dict(self.out_shapes))
 
     def pinned_host(self):
         """Pinned host buffers (inputs filled, outputs empty) for the end-to-end call."""
@@ -72,13 +90,17 @@ def _to_dev(a: np.ndarray) -> torch.Tensor:
 
 # ---------------------------------------------------------------- per-kernel jobs
 
+BINS_BYTES_PER_QUERY = 88  # 8 B (q, idx) + ~80 B of A no cache holds
+
+
 def job_binarysearch(N, Q, seed=6, rank=0):
     A, _ = inputs.binarysearch_inputs(seed, N, 1)
     q = inputs.u32(seed, Q, rank * Q, stream=2)
-    return Job("binarysearch", Q, (N, Q), [A, q, None], [(2, 4 * Q)], alg_bytes=136 * Q, unit="queries",
-               note="136 B/query compulsory: q + idx + the 128-B DRAM line of A holding the answer (any comparison "
-                    "search must touch it; a random access of 4..128 B moves one ~128-B line on B200, measured by "
-                    "tools/gather_probe.cu); upper levels are L2-resident")
+    return Job("binarysearch", Q, (N, Q), [A, q, None], [(2, 4 * Q)], alg_bytes=BINS_BYTES_PER_QUERY * Q,
+               unit="queries", bound="latency",
+               note="88 B/query (SURVEY 8(d)): 8 B of q and idx + ~80 B of A per query -- the search levels that "
+                    "are neither L2-resident (the top ~20 at N=2^26) nor inside the final shared sector (the last "
+                    "3), i.e. 2-3 random 32-B sectors; below ncu's measured DRAM bytes per query")
 
 
 def job_fwt(N, seed=5, rank=0):
@@ -110,17 +132,27 @@ def job_sobel(H, W, seed=7, rank=0):
     return Job("sobel", H * W, (H, W), [I, None], [(1, 4 * H * W)], alg_bytes=8 * H * W, unit="pixels")
 
 
-def job_blackscholes(n, seed=1, rank=0):
-    return Job("blackscholes", n, (), [inputs.blackscholes_r(seed, n, rank * n), None, None],
-               [(1, 4 * n), (2, 4 * n)], alg_bytes=12 * n, unit="options")
+def job_blackscholes(n, seed=1, rank=0, device_gen=False):
+    if device_gen:  # 2^30 options: generated in HBM (inputs.blackscholes_r_t, the same bits)
+        return Job("blackscholes", n, (0,), [None, None, None], [(1, 4 * n), (2, 4 * n)], alg_bytes=12 * n,
+                   unit="options", bound="mufu",
+                   dev_gen=lambda i: inputs.blackscholes_r_t(seed, n, rank * n))
+    return Job("blackscholes", n, (0,), [inputs.blackscholes_r(seed, n, rank * n), None, None],
+               [(1, 4 * n), (2, 4 * n)], alg_bytes=12 * n, unit="options", bound="mufu")
 
 
-def job_matmul(M, N, K, seed=10, rank=0):
+def job_matmul(M, N, K, seed=10, rank=0, device_gen=False):
+    note = f"{2 * M * N * K:.3e} flop"
+    if device_gen:
+        gen = {0: lambda: inputs.matmul_bf16_normal_t(seed, M, K, stream=22, row_offset=rank * M),
+               1: lambda: inputs.matmul_bf16_normal_t(seed, N, K, stream=24)}
+        return Job("matmul", M * N, (M, N, K), [None, None, None], [(2, 4 * M * N)],
+                   alg_bytes=2 * (M * K + N * K) + 4 * M * N, unit="C elements", bound="tensor", note=note,
+                   dev_gen=lambda i: gen[i]())
     A = inputs.matmul_bf16_normal(seed, M, K, stream=22, row_offset=rank * M)
     Bt = inputs.matmul_bf16_normal(seed, N, K, stream=24)
     return Job("matmul", M * N, (M, N, K), [A, Bt, None], [(2, 4 * M * N)],
-               alg_bytes=2 * (M * K + N * K) + 4 * M * N, unit="C elements", bound="tensor",
-               note=f"{2 * M * N * K:.3e} flop")
+               alg_bytes=2 * (M * K + N * K) + 4 * M * N, unit="C elements", bound="tensor", note=note)
 
 
 def job_dct(H, W, seed=9, rank=0):
@@ -175,9 +207,12 @@ def config_jobs(name: str, rank: int = 0):
     if name == "bs16":       # configs[0]
         return [job_blackscholes(1 << 16, rank=rank)]
     if name == "bs30":       # configs[4] (BlackScholes part)
-        return [job_blackscholes(1 << 30, rank=rank)]
+        return [job_blackscholes(1 << 30, rank=rank, device_gen=True)]
     if name == "mm16k":      # configs[4] (MatrixMultiplication part)
-        return [job_matmul(16384, 16384, 16384, rank=rank)]
+        return [job_matmul(16384, 16384, 16384, rank=rank, device_gen=True)]
+    if name == "rest10":     # the four BASELINE.json kernels outside configs[1] (bench.py's all-10 geomean)
+        return [job_blackscholes(1 << 30, rank=rank, device_gen=True), job_floydwarshall(4096),
+                job_dct(8192, 8192, rank=rank), job_matmul(16384, 16384, 16384, rank=rank, device_gen=True)]
     if name == "mm8k":
         return [job_matmul(8192, 8192, 8192, rank=rank)]
     if name == "fwdct":      # configs[3]
@@ -198,6 +233,7 @@ CONFIG_TITLES = {
     "suite28": "suite at 2^28 elements (BinarySearch N=2^28 Q=2^26, Transpose/Sobel 16384^2)",
     "bs16": "BlackScholes 2^16 options",
     "bs30": "BlackScholes 2^30 options",
+    "rest10": "BlackScholes 2^30, FloydWarshall 4096, DCT 8192^2, MatrixMultiplication 16384^3",
     "small": "suite at smoke sizes",
     "mm16k": "MatrixMultiplication 16384^3 bf16 -> fp32 (tcgen05)",
     "mm8k": "MatrixMultiplication 8192^3 bf16 -> fp32 (tcgen05)",
