@@ -104,33 +104,35 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned v = (unsigned)rep.lblock * BL + (unsigned)rep.ltid;
-  const unsigned total = a.L.vecs_before[a.L.T + 1];
-  int k = 1;
+  for (; rep.active(); rep.advance()) {
+    const unsigned v = (unsigned)rep.lblock * BL + (unsigned)rep.ltid;
+    const unsigned total = a.L.vecs_before[a.L.T + 1];
+    int k = 1;
 #pragma unroll 1
-  while (k < a.L.T && v >= a.L.vecs_before[k + 1]) ++k;
-  const bool tail = v >= total && v < total + 4u;
-  const bool active = v < total || tail;
-  const unsigned j0 = tail ? (v - total) * 4 : active ? (v - a.L.vecs_before[k]) * 4 : 0u;
-  unsigned stride = 1;
+    while (k < a.L.T && v >= a.L.vecs_before[k + 1]) ++k;
+    const bool tail = v >= total && v < total + 4u;
+    const bool active = v < total || tail;
+    const unsigned j0 = tail ? (v - total) * 4 : active ? (v - a.L.vecs_before[k]) * 4 : 0u;
+    unsigned stride = 1;
 #pragma unroll 1
-  for (int i = 0; i < k; ++i) stride *= FAN;
-  unsigned w[4];
+    for (int i = 0; i < k; ++i) stride *= FAN;
+    unsigned w[4];
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const unsigned j = j0 + q;
-    if (tail) {
-      w[q] = a.L.N16 + j < a.N ? __ldg(a.A + a.L.N16 + j) : 0xFFFFFFFFu;
-    } else {
-      const unsigned long long src = (unsigned long long)j * stride;
-      w[q] = (active && j < a.L.n[k]) ? __ldcs(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[16^k j] (A: evict-first)
+    for (int q = 0; q < 4; ++q) {
+      const unsigned j = j0 + q;
+      if (tail) {
+        w[q] = a.L.N16 + j < a.N ? __ldg(a.A + a.L.N16 + j) : 0xFFFFFFFFu;
+      } else {
+        const unsigned long long src = (unsigned long long)j * stride;
+        w[q] = (active && j < a.L.n[k]) ? __ldcs(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[16^k j] (A: evict-first)
+      }
     }
+    const unsigned dst = tail ? a.L.tail_off + j0 : active ? a.L.off[k] + j0 : 0u;
+    rep.template commit<4, 1>(active ? 0xFu : 0u, dst, w, 0xFFFFFFF0u,
+                              [&](unsigned i, unsigned m, const unsigned* x) {
+                                if (m == 0xFu) *reinterpret_cast<uint4*>(a.lev + i) = make_uint4(x[0], x[1], x[2], x[3]);
+                              });
   }
-  const unsigned dst = tail ? a.L.tail_off + j0 : active ? a.L.off[k] + j0 : 0u;
-  rep.template commit<4, 1>(active ? 0xFu : 0u, dst, w, 0xFFFFFFF0u,
-                            [&](unsigned i, unsigned m, const unsigned* x) {
-                              if (m == 0xFu) *reinterpret_cast<uint4*>(a.lev + i) = make_uint4(x[0], x[1], x[2], x[3]);
-                            });
   rep.finish();
 }
 
@@ -140,96 +142,98 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 3 : 4) 
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned j0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * VEC;
-  unsigned key[VEC];
-  unsigned mask = 0;
-  if (j0 + VEC <= a.Q) {
-    uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.q + j0));
-    key[0] = w.x; key[1] = w.y; key[2] = w.z; key[3] = w.w;
-    mask = 0xFu;
-  } else {
+  for (; rep.active(); rep.advance()) {
+    const unsigned j0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * VEC;
+    unsigned key[VEC];
+    unsigned mask = 0;
+    if (j0 + VEC <= a.Q) {
+      uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.q + j0));
+      key[0] = w.x; key[1] = w.y; key[2] = w.z; key[3] = w.w;
+      mask = 0xFu;
+    } else {
 #pragma unroll
-    for (int k = 0; k < VEC; ++k) {
-      const bool in = j0 + k < a.Q;
-      key[k] = in ? a.q[j0 + k] : 0u;
-      mask |= (in ? 1u : 0u) << k;
-    }
-  }
-  if constexpr (M == M_FAULT) {
-#pragma unroll
-    for (int k = 0; k < VEC; ++k) key[k] = rep.fault(SITE_LOAD, (long long)j0 + k, key[k]);
-  }
-  // Groups of 4 logical lanes descend together: for each of the group's 16
-  // queries the 4 members load one 16-B quarter of the same 64-B block, so a
-  // warp-wide load touches one cache line per query (1 L1 wavefront instead
-  // of 4).  Each lane tracks the block base of its OWN 4 queries and fetches the
-  // other members' bases by shuffle.
-  const int gm = rep.llane & 3;
-  const int g0 = rep.llane & ~3;
-  unsigned K[4][VEC];
-#pragma unroll
-  for (int i = 0; i < 4; ++i)
-#pragma unroll
-    for (int s = 0; s < VEC; ++s) K[i][s] = rep.lshfl_idx(key[s], g0 + i);
-  unsigned jj[VEC];
-#pragma unroll
-  for (int s = 0; s < VEC; ++s) jj[s] = a.N ? 1u : 0u;  // "block 0" of the top level
-  // one level: J <- 16 (max(J,1) - 1) + #{block < key}.  When J = 0 (key <= every
-  // entry) block 0 counts 0, so J stays 0 with no special case.
-  const unsigned* tailp = a.lev + a.L.tail_off - a.L.N16;  // tailp[N16 + i] = T[i]
-  // per-lane quarter pointers: element (base + 4 gm) of level P is Pq + 16 base bytes
-  auto level = [&](const unsigned* P, bool last) {
-    const unsigned* Pq = P + 4 * gm;
-    const unsigned* Tq = tailp + 4 * gm;
-#pragma unroll
-    for (int s = 0; s < VEC; ++s) {
-      const unsigned mybase = (max(jj[s], 1u) - 1u) * FAN;
-      unsigned packed = 0;
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const unsigned base = rep.lshfl_idx(mybase, g0 + i);
-        uint4 w;
-        if (!last) {  // sample levels: keep them L2-resident (default policy)
-          w = __ldg(reinterpret_cast<const uint4*>(wide_addr(Pq, base)));
-        } else {  // the caller's A: random 64-B blocks, evict-first; the ragged
-                  // last block comes from the padded copy (a block never straddles N16)
-          w = __ldcs(reinterpret_cast<const uint4*>(wide_addr(base >= a.L.N16 ? Tq : Pq, base)));
-        }
-        packed += count_ge(w, K[i][s]) << (8 * i);
+      for (int k = 0; k < VEC; ++k) {
+        const bool in = j0 + k < a.Q;
+        key[k] = in ? a.q[j0 + k] : 0u;
+        mask |= (in ? 1u : 0u) << k;
       }
-      packed += rep.lshfl_xor(packed, 1);  // sum the 4 quarters (bytes <= 16: no carries)
-      packed += rep.lshfl_xor(packed, 2);
-      jj[s] = mybase + FAN - ((packed >> (8 * gm)) & 0xFFu);  // #{block < key} = 16 - #{block >= key}
     }
-  };
-  for (int lv = a.L.T; lv >= 1; --lv) {  // padded sample levels: no bounds checks
     if constexpr (M == M_FAULT) {
-      if (lv == a.L.T - 1) {  // control-flow fault: a flipped block index, kept in range
+#pragma unroll
+      for (int k = 0; k < VEC; ++k) key[k] = rep.fault(SITE_LOAD, (long long)j0 + k, key[k]);
+    }
+    // Groups of 4 logical lanes descend together: for each of the group's 16
+    // queries the 4 members load one 16-B quarter of the same 64-B block, so a
+    // warp-wide load touches one cache line per query (1 L1 wavefront instead
+    // of 4).  Each lane tracks the block base of its OWN 4 queries and fetches the
+    // other members' bases by shuffle.
+    const int gm = rep.llane & 3;
+    const int g0 = rep.llane & ~3;
+    unsigned K[4][VEC];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int s = 0; s < VEC; ++s) K[i][s] = rep.lshfl_idx(key[s], g0 + i);
+    unsigned jj[VEC];
+#pragma unroll
+    for (int s = 0; s < VEC; ++s) jj[s] = a.N ? 1u : 0u;  // "block 0" of the top level
+    // one level: J <- 16 (max(J,1) - 1) + #{block < key}.  When J = 0 (key <= every
+    // entry) block 0 counts 0, so J stays 0 with no special case.
+    const unsigned* tailp = a.lev + a.L.tail_off - a.L.N16;  // tailp[N16 + i] = T[i]
+    // per-lane quarter pointers: element (base + 4 gm) of level P is Pq + 16 base bytes
+    auto level = [&](const unsigned* P, bool last) {
+      const unsigned* Pq = P + 4 * gm;
+      const unsigned* Tq = tailp + 4 * gm;
+#pragma unroll
+      for (int s = 0; s < VEC; ++s) {
+        const unsigned mybase = (max(jj[s], 1u) - 1u) * FAN;
+        unsigned packed = 0;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const unsigned base = rep.lshfl_idx(mybase, g0 + i);
+          uint4 w;
+          if (!last) {  // sample levels: keep them L2-resident (default policy)
+            w = __ldg(reinterpret_cast<const uint4*>(wide_addr(Pq, base)));
+          } else {  // the caller's A: random 64-B blocks, evict-first; the ragged
+                    // last block comes from the padded copy (a block never straddles N16)
+            w = __ldcs(reinterpret_cast<const uint4*>(wide_addr(base >= a.L.N16 ? Tq : Pq, base)));
+          }
+          packed += count_ge(w, K[i][s]) << (8 * i);
+        }
+        packed += rep.lshfl_xor(packed, 1);  // sum the 4 quarters (bytes <= 16: no carries)
+        packed += rep.lshfl_xor(packed, 2);
+        jj[s] = mybase + FAN - ((packed >> (8 * gm)) & 0xFFu);  // #{block < key} = 16 - #{block >= key}
+      }
+    };
+    for (int lv = a.L.T; lv >= 1; --lv) {  // padded sample levels: no bounds checks
+      if constexpr (M == M_FAULT) {
+        if (lv == a.L.T - 1) {  // control-flow fault: a flipped block index, kept in range
+#pragma unroll
+          for (int s = 0; s < VEC; ++s) {
+            const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, jj[s]);
+            jj[s] = f > a.L.n[lv + 1] ? a.L.n[lv + 1] : f;
+          }
+        }
+      }
+      level(a.lev + a.L.off[lv], false);
+    }
+    if constexpr (M == M_FAULT) {
+      if (a.L.T == 1) {
 #pragma unroll
         for (int s = 0; s < VEC; ++s) {
           const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, jj[s]);
-          jj[s] = f > a.L.n[lv + 1] ? a.L.n[lv + 1] : f;
+          jj[s] = f > a.L.n[1] ? a.L.n[1] : f;
         }
       }
     }
-    level(a.lev + a.L.off[lv], false);
+    level(a.A, true);  // the caller's A
+    rep.template commit<VEC, 0>(mask, j0, jj, a.Q, [&](unsigned i, unsigned m, const unsigned* w) {
+      if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.idx + i), make_uint4(w[0], w[1], w[2], w[3]));
+      else
+        for (int k = 0; k < VEC; ++k)
+          if ((m >> k) & 1u) a.idx[i + k] = w[k];
+    });
   }
-  if constexpr (M == M_FAULT) {
-    if (a.L.T == 1) {
-#pragma unroll
-      for (int s = 0; s < VEC; ++s) {
-        const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, jj[s]);
-        jj[s] = f > a.L.n[1] ? a.L.n[1] : f;
-      }
-    }
-  }
-  level(a.A, true);  // the caller's A
-  rep.template commit<VEC, 0>(mask, j0, jj, a.Q, [&](unsigned i, unsigned m, const unsigned* w) {
-    if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.idx + i), make_uint4(w[0], w[1], w[2], w[3]));
-    else
-      for (int k = 0; k < VEC; ++k)
-        if ((m >> k) & 1u) a.idx[i + k] = w[k];
-  });
   rep.finish();
 }
 

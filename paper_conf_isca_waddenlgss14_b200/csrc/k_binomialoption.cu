@@ -40,54 +40,56 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bo_kernel(BoArgs a, Ctx c) 
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned lw = (unsigned)rep.ltid / LW;
-  const unsigned o0 = 4u * ((unsigned)rep.lblock * NLW + lw);  // first of this warp's 4 options
-  unsigned res[4] = {0u, 0u, 0u, 0u};
+  for (; rep.active(); rep.advance()) {
+    const unsigned lw = (unsigned)rep.ltid / LW;
+    const unsigned o0 = 4u * ((unsigned)rep.lblock * NLW + lw);  // first of this warp's 4 options
+    unsigned res[4] = {0u, 0u, 0u, 0u};
 #pragma unroll 1
-  for (int o = 0; o < 4; ++o) {
-    const unsigned opt = o0 + o;
-    if (opt >= a.n) break;  // uniform over the logical warp
-    float r = __ldg(a.r + opt);
-    if constexpr (M == M_FAULT) r = rep.faultf(SITE_LOAD, (long long)opt, r);
-    const float om = __fsub_rn(1.0f, r);
-    const float S = __fadd_rn(__fmul_rn(5.0f, om), __fmul_rn(30.0f, r));
-    const float K = __fadd_rn(om, __fmul_rn(100.0f, r));
-    const float T = __fadd_rn(__fmul_rn(0.25f, om), __fmul_rn(10.0f, r));
-    const float dt = __fdiv_rn(T, (float)NSTEPS);
-    const float vsdt = __fmul_rn(VOL, __fsqrt_rn(dt));
-    const float rdt = __fmul_rn(RFREE, dt);
-    const float em_up = expm1f(vsdt), em_dn = expm1f(-vsdt);
-    float pu = __fdiv_rn(__fsub_rn(expm1f(rdt), em_dn), __fsub_rn(em_up, em_dn));
-    if constexpr (M == M_FAULT) pu = rep.faultf(SITE_COMPUTE, (long long)opt, pu);
-    const float disc = expf(-rdt);
-    const float pur = __fmul_rn(pu, disc), pdr = __fmul_rn(__fsub_rn(1.0f, pu), disc);
-    float v[P];
+    for (int o = 0; o < 4; ++o) {
+      const unsigned opt = o0 + o;
+      if (opt >= a.n) break;  // uniform over the logical warp
+      float r = __ldg(a.r + opt);
+      if constexpr (M == M_FAULT) r = rep.faultf(SITE_LOAD, (long long)opt, r);
+      const float om = __fsub_rn(1.0f, r);
+      const float S = __fadd_rn(__fmul_rn(5.0f, om), __fmul_rn(30.0f, r));
+      const float K = __fadd_rn(om, __fmul_rn(100.0f, r));
+      const float T = __fadd_rn(__fmul_rn(0.25f, om), __fmul_rn(10.0f, r));
+      const float dt = __fdiv_rn(T, (float)NSTEPS);
+      const float vsdt = __fmul_rn(VOL, __fsqrt_rn(dt));
+      const float rdt = __fmul_rn(RFREE, dt);
+      const float em_up = expm1f(vsdt), em_dn = expm1f(-vsdt);
+      float pu = __fdiv_rn(__fsub_rn(expm1f(rdt), em_dn), __fsub_rn(em_up, em_dn));
+      if constexpr (M == M_FAULT) pu = rep.faultf(SITE_COMPUTE, (long long)opt, pu);
+      const float disc = expf(-rdt);
+      const float pur = __fmul_rn(pu, disc), pdr = __fmul_rn(__fsub_rn(1.0f, pu), disc);
+      float v[P];
 #pragma unroll
-    for (int t = 0; t < P; ++t) {
-      const int i = rep.llane * P + t;  // leaf index
-      const float price = __fmul_rn(S, expf(__fmul_rn(vsdt, (float)(2 * i - NSTEPS))));
-      v[t] = i <= NSTEPS ? fmaxf(__fsub_rn(price, K), 0.0f) : 0.0f;
-    }
-    // backward induction: V_i <- pur V_{i+1} + pdr V_i (nodes >= j are dead and never feed V_0)
+      for (int t = 0; t < P; ++t) {
+        const int i = rep.llane * P + t;  // leaf index
+        const float price = __fmul_rn(S, expf(__fmul_rn(vsdt, (float)(2 * i - NSTEPS))));
+        v[t] = i <= NSTEPS ? fmaxf(__fsub_rn(price, K), 0.0f) : 0.0f;
+      }
+      // backward induction: V_i <- pur V_{i+1} + pdr V_i (nodes >= j are dead and never feed V_0)
 #pragma unroll 2
-    for (int j = NSTEPS; j > 0; --j) {
-      const float nxt = __shfl_down_sync(0xffffffffu, v[0], DUP);  // logical lane + 1, same replica
+      for (int j = NSTEPS; j > 0; --j) {
+        const float nxt = __shfl_down_sync(0xffffffffu, v[0], DUP);  // logical lane + 1, same replica
 #pragma unroll
-      for (int t = 0; t < P - 1; ++t) v[t] = __fmaf_rn(pur, v[t + 1], __fmul_rn(pdr, v[t]));
-      v[P - 1] = __fmaf_rn(pur, nxt, __fmul_rn(pdr, v[P - 1]));
+        for (int t = 0; t < P - 1; ++t) v[t] = __fmaf_rn(pur, v[t + 1], __fmul_rn(pdr, v[t]));
+        v[P - 1] = __fmaf_rn(pur, nxt, __fmul_rn(pdr, v[P - 1]));
+      }
+      res[o] = __float_as_uint(v[0]);  // meaningful in logical lane 0
     }
-    res[o] = __float_as_uint(v[0]);  // meaningful in logical lane 0
+    const unsigned nval = a.n > o0 ? min(4u, a.n - o0) : 0u;
+    const unsigned mask = (rep.llane == 0) ? ((1u << nval) - 1u) : 0u;
+    rep.template commit<4, 0>(mask, mask ? o0 : 0u, res, a.n, [&](unsigned idx, unsigned m, const unsigned* w) {
+      if (m == 0xFu)
+        *reinterpret_cast<float4*>(a.call + idx) =
+            make_float4(__uint_as_float(w[0]), __uint_as_float(w[1]), __uint_as_float(w[2]), __uint_as_float(w[3]));
+      else
+        for (int k = 0; k < 4; ++k)
+          if ((m >> k) & 1u) a.call[idx + k] = __uint_as_float(w[k]);
+    });
   }
-  const unsigned nval = a.n > o0 ? min(4u, a.n - o0) : 0u;
-  const unsigned mask = (rep.llane == 0) ? ((1u << nval) - 1u) : 0u;
-  rep.template commit<4, 0>(mask, mask ? o0 : 0u, res, a.n, [&](unsigned idx, unsigned m, const unsigned* w) {
-    if (m == 0xFu)
-      *reinterpret_cast<float4*>(a.call + idx) =
-          make_float4(__uint_as_float(w[0]), __uint_as_float(w[1]), __uint_as_float(w[2]), __uint_as_float(w[3]));
-    else
-      for (int k = 0; k < 4; ++k)
-        if ((m >> k) & 1u) a.call[idx + k] = __uint_as_float(w[k]);
-  });
   rep.finish();
 }
 

@@ -184,85 +184,87 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bitonic_kernel(BitArgs a, C
   __shared__ unsigned tilebuf[Geom<V>::SMDUP == 2 ? PLANE + SM_WORDS : SM_WORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned tile = (unsigned)rep.lblock;
-  const int te = 1 << a.tb;
-  unsigned* const tp = &rep.template smp<PLANE>(tilebuf, 0);
+  for (; rep.active(); rep.advance()) {
+    const unsigned tile = (unsigned)rep.lblock;
+    const int te = 1 << a.tb;
+    unsigned* const tp = &rep.template smp<PLANE>(tilebuf, 0);
 
-  // ---- load (16-B vectors; padding keys beyond N are +inf)
-  {
-    constexpr int IT = TE_MAX / (4 * BL);
-    uint4 f[IT];
+    // ---- load (16-B vectors; padding keys beyond N are +inf)
+    {
+      constexpr int IT = TE_MAX / (4 * BL);
+      uint4 f[IT];
 #pragma unroll
-    for (int it = 0; it < IT; ++it) {
-      const int e0 = 4 * (rep.ltid + it * BL);
-      const unsigned g = gidx(a, tile, (unsigned)e0);
-      if (e0 < te && g + 3 < a.N) {
-        f[it] = __ldcs(reinterpret_cast<const uint4*>(a.src + g));
-      } else {
-        unsigned w[4];
+      for (int it = 0; it < IT; ++it) {
+        const int e0 = 4 * (rep.ltid + it * BL);
+        const unsigned g = gidx(a, tile, (unsigned)e0);
+        if (e0 < te && g + 3 < a.N) {
+          f[it] = __ldcs(reinterpret_cast<const uint4*>(a.src + g));
+        } else {
+          unsigned w[4];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) w[k] = (e0 + k < te && g + k < a.N) ? a.src[g + k] : 0xFFFFFFFFu;
-        f[it] = make_uint4(w[0], w[1], w[2], w[3]);
+          for (int k = 0; k < 4; ++k) w[k] = (e0 + k < te && g + k < a.N) ? a.src[g + k] : 0xFFFFFFFFu;
+          f[it] = make_uint4(w[0], w[1], w[2], w[3]);
+        }
       }
-    }
 #pragma unroll
-    for (int it = 0; it < IT; ++it) {
-      const int e0 = 4 * (rep.ltid + it * BL);
-      if (e0 < te) {
-        unsigned w[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
-        if constexpr (M == M_FAULT) {
-          if (a.first) {
-            const unsigned g = gidx(a, tile, (unsigned)e0);
+      for (int it = 0; it < IT; ++it) {
+        const int e0 = 4 * (rep.ltid + it * BL);
+        if (e0 < te) {
+          unsigned w[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
+          if constexpr (M == M_FAULT) {
+            if (a.first) {
+              const unsigned g = gidx(a, tile, (unsigned)e0);
 #pragma unroll
-            for (int k = 0; k < 4; ++k) w[k] = rep.fault(SITE_LOAD, (long long)g + k, w[k]);
+              for (int k = 0; k < 4; ++k) w[k] = rep.fault(SITE_LOAD, (long long)g + k, w[k]);
+            }
+          }
+          if (rep.template sts_ok<4>(w, (unsigned)e0)) {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) tp[phys(e0 + k)] = w[k];
           }
         }
-        if (rep.template sts_ok<4>(w, (unsigned)e0)) {
-#pragma unroll
-          for (int k = 0; k < 4; ++k) tp[phys(e0 + k)] = w[k];
-        }
       }
     }
-  }
-  __syncthreads();
-
-  // ---- register rounds
-  for (int ri = 0; ri < a.nr; ++ri) {
-    const BitRound R = a.r[ri];
-    switch (R.q) {
-      case 0: bit_round<0>(rep, a, tp, tile, R, ri); break;
-      case 1: bit_round<1>(rep, a, tp, tile, R, ri); break;
-      case 2: bit_round<2>(rep, a, tp, tile, R, ri); break;
-      case 3: bit_round<3>(rep, a, tp, tile, R, ri); break;
-      case 4: bit_round<4>(rep, a, tp, tile, R, ri); break;
-      case 5: bit_round<5>(rep, a, tp, tile, R, ri); break;
-      case 6: bit_round<6>(rep, a, tp, tile, R, ri); break;
-      case 7: bit_round<7>(rep, a, tp, tile, R, ri); break;
-      default: bit_round<8>(rep, a, tp, tile, R, ri); break;
-    }
     __syncthreads();
-  }
 
-  // ---- store: one vector commit per 4 keys
-#pragma unroll 1
-  for (int it = 0; it < TE_MAX / (4 * BL); ++it) {
-    const int e0 = 4 * rep.ltid + it * 4 * BL;
-    const unsigned g = e0 < te ? gidx(a, tile, (unsigned)e0) : 0u;
-    unsigned w[4];
-    unsigned mask = 0;
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const bool in = e0 + k < te && g + k < a.N;
-      w[k] = in ? tp[phys(e0 + k)] : 0u;
-      mask |= (in ? 1u : 0u) << k;
+    // ---- register rounds
+    for (int ri = 0; ri < a.nr; ++ri) {
+      const BitRound R = a.r[ri];
+      switch (R.q) {
+        case 0: bit_round<0>(rep, a, tp, tile, R, ri); break;
+        case 1: bit_round<1>(rep, a, tp, tile, R, ri); break;
+        case 2: bit_round<2>(rep, a, tp, tile, R, ri); break;
+        case 3: bit_round<3>(rep, a, tp, tile, R, ri); break;
+        case 4: bit_round<4>(rep, a, tp, tile, R, ri); break;
+        case 5: bit_round<5>(rep, a, tp, tile, R, ri); break;
+        case 6: bit_round<6>(rep, a, tp, tile, R, ri); break;
+        case 7: bit_round<7>(rep, a, tp, tile, R, ri); break;
+        default: bit_round<8>(rep, a, tp, tile, R, ri); break;
+      }
+      __syncthreads();
     }
-    rep.template commit<4, 0>(mask, mask ? g : 0u, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
-      if (m == 0xFu)
-        __stcs(reinterpret_cast<uint4*>(a.dst + idx), make_uint4(x[0], x[1], x[2], x[3]));
-      else
-        for (int k = 0; k < 4; ++k)
-          if ((m >> k) & 1u) a.dst[idx + k] = x[k];
-    }, /*defer=*/it < TE_MAX / (4 * BL) - 1);
+
+    // ---- store: one vector commit per 4 keys
+#pragma unroll 1
+    for (int it = 0; it < TE_MAX / (4 * BL); ++it) {
+      const int e0 = 4 * rep.ltid + it * 4 * BL;
+      const unsigned g = e0 < te ? gidx(a, tile, (unsigned)e0) : 0u;
+      unsigned w[4];
+      unsigned mask = 0;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const bool in = e0 + k < te && g + k < a.N;
+        w[k] = in ? tp[phys(e0 + k)] : 0u;
+        mask |= (in ? 1u : 0u) << k;
+      }
+      rep.template commit<4, 0>(mask, mask ? g : 0u, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
+        if (m == 0xFu)
+          __stcs(reinterpret_cast<uint4*>(a.dst + idx), make_uint4(x[0], x[1], x[2], x[3]));
+        else
+          for (int k = 0; k < 4; ++k)
+            if ((m >> k) & 1u) a.dst[idx + k] = x[k];
+      }, /*defer=*/it < TE_MAX / (4 * BL) - 1);
+    }
   }
   rep.finish();
 }

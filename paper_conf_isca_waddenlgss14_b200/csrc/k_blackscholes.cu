@@ -90,51 +90,53 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bs_kernel(BsArgs a, Ctx c) 
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned i0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * VEC;
-  unsigned mask = 0;
+  for (; rep.active(); rep.advance()) {
+    const unsigned i0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * VEC;
+    unsigned mask = 0;
 #pragma unroll
-  for (int k = 0; k < VEC; ++k) mask |= (i0 + k < a.n ? 1u : 0u) << k;
-  // input replication: each replica loads its own copy
-  BsParams prm[VEC];
-  if constexpr (!IND) {
-    float r4[VEC];
-    load4(a.r, i0, a.n, r4);
+    for (int k = 0; k < VEC; ++k) mask |= (i0 + k < a.n ? 1u : 0u) << k;
+    // input replication: each replica loads its own copy
+    BsParams prm[VEC];
+    if constexpr (!IND) {
+      float r4[VEC];
+      load4(a.r, i0, a.n, r4);
 #pragma unroll
-    for (int k = 0; k < VEC; ++k) prm[k] = bs_map(rep.faultf(SITE_LOAD, (long long)i0 + k, r4[k]));
-  } else {
-    const size_t pl = a.n;  // plane pitch
-    float S4[VEC], K4[VEC], T4[VEC], R4[VEC], V4[VEC];
-    load4(a.r, i0, a.n, S4);
-    load4(a.r + pl, i0, a.n, K4);
-    load4(a.r + 2 * pl, i0, a.n, T4);
-    load4(a.r + 3 * pl, i0, a.n, R4);
-    load4(a.r + 4 * pl, i0, a.n, V4);
+      for (int k = 0; k < VEC; ++k) prm[k] = bs_map(rep.faultf(SITE_LOAD, (long long)i0 + k, r4[k]));
+    } else {
+      const size_t pl = a.n;  // plane pitch
+      float S4[VEC], K4[VEC], T4[VEC], R4[VEC], V4[VEC];
+      load4(a.r, i0, a.n, S4);
+      load4(a.r + pl, i0, a.n, K4);
+      load4(a.r + 2 * pl, i0, a.n, T4);
+      load4(a.r + 3 * pl, i0, a.n, R4);
+      load4(a.r + 4 * pl, i0, a.n, V4);
 #pragma unroll
-    for (int k = 0; k < VEC; ++k)
-      prm[k] = BsParams{rep.faultf(SITE_LOAD, (long long)i0 + k, S4[k]), K4[k], T4[k], R4[k], V4[k]};
-  }
-  unsigned cv[VEC], pv[VEC];
+      for (int k = 0; k < VEC; ++k)
+        prm[k] = BsParams{rep.faultf(SITE_LOAD, (long long)i0 + k, S4[k]), K4[k], T4[k], R4[k], V4[k]};
+    }
+    unsigned cv[VEC], pv[VEC];
 #pragma unroll
-  for (int k = 0; k < VEC; ++k) {
-    float cl, pt;
-    bs_option(rep, prm[k], (long long)i0 + k, cl, pt);
-    cv[k] = __float_as_uint(cl);
-    pv[k] = __float_as_uint(pt);
-  }
-  auto store_to = [](float* base) {
-    return [base](unsigned idx, unsigned m, const unsigned* v) {
-      if (m == 0xFu) {
-        __stcs(reinterpret_cast<float4*>(base + idx),
-               make_float4(__uint_as_float(v[0]), __uint_as_float(v[1]), __uint_as_float(v[2]), __uint_as_float(v[3])));
-      } else {
+    for (int k = 0; k < VEC; ++k) {
+      float cl, pt;
+      bs_option(rep, prm[k], (long long)i0 + k, cl, pt);
+      cv[k] = __float_as_uint(cl);
+      pv[k] = __float_as_uint(pt);
+    }
+    auto store_to = [](float* base) {
+      return [base](unsigned idx, unsigned m, const unsigned* v) {
+        if (m == 0xFu) {
+          __stcs(reinterpret_cast<float4*>(base + idx),
+                 make_float4(__uint_as_float(v[0]), __uint_as_float(v[1]), __uint_as_float(v[2]), __uint_as_float(v[3])));
+        } else {
 #pragma unroll
-        for (int k = 0; k < VEC; ++k)
-          if ((m >> k) & 1u) base[idx + k] = __uint_as_float(v[k]);
-      }
+          for (int k = 0; k < VEC; ++k)
+            if ((m >> k) & 1u) base[idx + k] = __uint_as_float(v[k]);
+        }
+      };
     };
-  };
-  rep.template commit<VEC, 0>(mask, i0, cv, a.n, store_to(a.call), /*defer=*/true);
-  rep.template commit<VEC, 1>(mask, i0, pv, a.n, store_to(a.put));
+    rep.template commit<VEC, 0>(mask, i0, cv, a.n, store_to(a.call), /*defer=*/true);
+    rep.template commit<VEC, 1>(mask, i0, pv, a.n, store_to(a.put));
+  }
   rep.finish();
 }
 

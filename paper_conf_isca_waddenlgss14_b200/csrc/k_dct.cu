@@ -39,118 +39,120 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c
   __shared__ __align__(16) float Zs[Geom<V>::SMDUP == 2 ? PLANE + ZWORDS : ZWORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
-  // row pass: logical warp w = image row r of the strip, lane = block b, so a
-  // warp's loads are one contiguous 1 KiB row segment (coalesced; with the
-  // block-major mapping of the column pass below the loads touched 8 rows per
-  // instruction and L1 ran at 98%: 0.203 -> 0.154 ms at 8192^2)
-  int b = rep.ltid % BLOCKS, r = rep.ltid / BLOCKS;
-  unsigned col0 = (bx * BLOCKS + b) * 8;
-  bool active = col0 < a.W;
-  const unsigned row = by * 8 + r;
-  float x[8];
-  if (active) {
-    if (a.v8) {  // one 256-bit load: the warp's 1 KiB row segment in whole lines
-      unsigned w[8];
-      ldcs8(a.X + (size_t)row * a.W + col0, w);
+  for (; rep.active(); rep.advance()) {
+    const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
+    // row pass: logical warp w = image row r of the strip, lane = block b, so a
+    // warp's loads are one contiguous 1 KiB row segment (coalesced; with the
+    // block-major mapping of the column pass below the loads touched 8 rows per
+    // instruction and L1 ran at 98%: 0.203 -> 0.154 ms at 8192^2)
+    int b = rep.ltid % BLOCKS, r = rep.ltid / BLOCKS;
+    unsigned col0 = (bx * BLOCKS + b) * 8;
+    bool active = col0 < a.W;
+    const unsigned row = by * 8 + r;
+    float x[8];
+    if (active) {
+      if (a.v8) {  // one 256-bit load: the warp's 1 KiB row segment in whole lines
+        unsigned w[8];
+        ldcs8(a.X + (size_t)row * a.W + col0, w);
 #pragma unroll
-      for (int y = 0; y < 8; ++y) x[y] = __uint_as_float(w[y]);
-    } else {  // X only 16-B aligned (the ABI minimum)
-      const float4* src = reinterpret_cast<const float4*>(a.X + (size_t)row * a.W + col0);
-      float4 p = __ldcs(src), q = __ldcs(src + 1);
-      x[0] = p.x; x[1] = p.y; x[2] = p.z; x[3] = p.w; x[4] = q.x; x[5] = q.y; x[6] = q.z; x[7] = q.w;
-    }
-  } else {
-#pragma unroll
-    for (int y = 0; y < 8; ++y) x[y] = 0.0f;
-  }
-  if constexpr (M == M_FAULT) {
-#pragma unroll
-    for (int y = 0; y < 8; ++y) x[y] = rep.faultf(SITE_LOAD, (long long)row * a.W + col0 + y, x[y]);
-  }
-  float z[8];
-#pragma unroll
-  for (int v = 0; v < 8; ++v) {
-    float s = __fmul_rn(x[0], a.C[v][0]);
-#pragma unroll
-    for (int y = 1; y < 8; ++y) s = __fmaf_rn(x[y], a.C[v][y], s);
-    if constexpr (M == M_FAULT) s = rep.faultf(SITE_COMPUTE, (long long)row * a.W + col0 + v, s);
-    z[v] = s;
-  }
-  float* zrow = &rep.template smp<PLANE>(Zs, b * BSTRIDE + r * 8);
-  const unsigned zw[8] = {__float_as_uint(z[0]), __float_as_uint(z[1]), __float_as_uint(z[2]), __float_as_uint(z[3]),
-                          __float_as_uint(z[4]), __float_as_uint(z[5]), __float_as_uint(z[6]), __float_as_uint(z[7])};
-  if (rep.template sts_ok<8>(zw, b * BSTRIDE + r * 8)) {
-    reinterpret_cast<float4*>(zrow)[0] = make_float4(z[0], z[1], z[2], z[3]);
-    reinterpret_cast<float4*>(zrow)[1] = make_float4(z[4], z[5], z[6], z[7]);
-  }
-  __syncthreads();
-  // column pass: thread (b, u) produces output row u of block b (8 lanes per
-  // block: the smem reads of a warp broadcast over 4 blocks, one wavefront;
-  // routing the output back through smem for row-major stores was slower)
-  b = rep.ltid / 8;
-  const int u = rep.ltid % 8;
-  col0 = (bx * BLOCKS + b) * 8;
-  active = col0 < a.W;
-  float y[8];
-#pragma unroll
-  for (int v = 0; v < 8; ++v) y[v] = 0.0f;
-  const float* zb = &rep.template smp<PLANE>(Zs, b * BSTRIDE);
-#pragma unroll
-  for (int xr = 0; xr < 8; ++xr) {
-    float4 p = reinterpret_cast<const float4*>(zb + xr * 8)[0];
-    float4 q = reinterpret_cast<const float4*>(zb + xr * 8)[1];
-    float zz[8] = {p.x, p.y, p.z, p.w, q.x, q.y, q.z, q.w};
-    if constexpr (M == M_FAULT) {
-#pragma unroll
-      for (int v = 0; v < 8; ++v)
-        zz[v] = rep.faultf(SITE_SMEM, (long long)(by * 8 + xr) * a.W + col0 + v, zz[v]);
-    }
-    const float cu = a.C[u][xr];
-#pragma unroll
-    for (int v = 0; v < 8; ++v) y[v] = xr == 0 ? __fmul_rn(cu, zz[v]) : __fmaf_rn(cu, zz[v], y[v]);
-  }
-  // Stores (measured per variant at 8192^2): none, intra_reg and intra_nolds
-  // first swap one 16-B half between output rows u and u^4 of a block through
-  // a shuffle, so that store h writes rows 4h..4h+3 of the warp's blocks as
-  // whole 128-B lines (lanes u < 4: half 0 of row 4h + u; lanes u >= 4: half 1
-  // of row 4h + u - 4) -- none 0.155 -> 0.145 ms, intra_reg 0.272 -> 0.253 ms;
-  // intra_smem and the inter variants were slower with it and store their own
-  // row u directly (8 rows of half-sectors per store).
-  constexpr bool XS = (V == V_NONE || V == V_INTRA_REG || V == V_INTRA_NOLDS);
-  const bool lowu = u < 4;
-  unsigned got[4];
-  if constexpr (XS) {
-#pragma unroll
-    for (int q = 0; q < 4; ++q) got[q] = rep.lshfl_xor(__float_as_uint(lowu ? y[4 + q] : y[q]), 4);
-  }
-#pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    unsigned w[4];
-    unsigned orow, idx;
-    if constexpr (XS) {
-#pragma unroll
-      for (int q = 0; q < 4; ++q)
-        w[q] = lowu ? (h == 0 ? __float_as_uint(y[q]) : got[q]) : (h == 0 ? got[q] : __float_as_uint(y[4 + q]));
-      orow = by * 8 + (lowu ? (unsigned)u + 4u * h : (unsigned)u - 4u + 4u * h);
-      idx = orow * a.W + col0 + (lowu ? 0u : 4u);
+        for (int y = 0; y < 8; ++y) x[y] = __uint_as_float(w[y]);
+      } else {  // X only 16-B aligned (the ABI minimum)
+        const float4* src = reinterpret_cast<const float4*>(a.X + (size_t)row * a.W + col0);
+        float4 p = __ldcs(src), q = __ldcs(src + 1);
+        x[0] = p.x; x[1] = p.y; x[2] = p.z; x[3] = p.w; x[4] = q.x; x[5] = q.y; x[6] = q.z; x[7] = q.w;
+      }
     } else {
 #pragma unroll
-      for (int q = 0; q < 4; ++q) w[q] = __float_as_uint(y[4 * h + q]);
-      orow = by * 8 + u;
-      idx = orow * a.W + col0 + 4 * h;
+      for (int y = 0; y < 8; ++y) x[y] = 0.0f;
     }
-    rep.template commit<4, 0>(active ? 0xFu : 0u, active ? idx : 0u, w, a.H * a.W,
-                              [&](unsigned i, unsigned m, const unsigned* v) {
-                                if (m == 0xFu)
-                                  __stcs(reinterpret_cast<float4*>(a.Y + i),
-                                         make_float4(__uint_as_float(v[0]), __uint_as_float(v[1]),
-                                                     __uint_as_float(v[2]), __uint_as_float(v[3])));
-                                else
-                                  for (int k = 0; k < 4; ++k)
-                                    if ((m >> k) & 1u) a.Y[i + k] = __uint_as_float(v[k]);
-                              },
-                              /*defer=*/h == 0);
+    if constexpr (M == M_FAULT) {
+#pragma unroll
+      for (int y = 0; y < 8; ++y) x[y] = rep.faultf(SITE_LOAD, (long long)row * a.W + col0 + y, x[y]);
+    }
+    float z[8];
+#pragma unroll
+    for (int v = 0; v < 8; ++v) {
+      float s = __fmul_rn(x[0], a.C[v][0]);
+#pragma unroll
+      for (int y = 1; y < 8; ++y) s = __fmaf_rn(x[y], a.C[v][y], s);
+      if constexpr (M == M_FAULT) s = rep.faultf(SITE_COMPUTE, (long long)row * a.W + col0 + v, s);
+      z[v] = s;
+    }
+    float* zrow = &rep.template smp<PLANE>(Zs, b * BSTRIDE + r * 8);
+    const unsigned zw[8] = {__float_as_uint(z[0]), __float_as_uint(z[1]), __float_as_uint(z[2]), __float_as_uint(z[3]),
+                            __float_as_uint(z[4]), __float_as_uint(z[5]), __float_as_uint(z[6]), __float_as_uint(z[7])};
+    if (rep.template sts_ok<8>(zw, b * BSTRIDE + r * 8)) {
+      reinterpret_cast<float4*>(zrow)[0] = make_float4(z[0], z[1], z[2], z[3]);
+      reinterpret_cast<float4*>(zrow)[1] = make_float4(z[4], z[5], z[6], z[7]);
+    }
+    __syncthreads();
+    // column pass: thread (b, u) produces output row u of block b (8 lanes per
+    // block: the smem reads of a warp broadcast over 4 blocks, one wavefront;
+    // routing the output back through smem for row-major stores was slower)
+    b = rep.ltid / 8;
+    const int u = rep.ltid % 8;
+    col0 = (bx * BLOCKS + b) * 8;
+    active = col0 < a.W;
+    float y[8];
+#pragma unroll
+    for (int v = 0; v < 8; ++v) y[v] = 0.0f;
+    const float* zb = &rep.template smp<PLANE>(Zs, b * BSTRIDE);
+#pragma unroll
+    for (int xr = 0; xr < 8; ++xr) {
+      float4 p = reinterpret_cast<const float4*>(zb + xr * 8)[0];
+      float4 q = reinterpret_cast<const float4*>(zb + xr * 8)[1];
+      float zz[8] = {p.x, p.y, p.z, p.w, q.x, q.y, q.z, q.w};
+      if constexpr (M == M_FAULT) {
+#pragma unroll
+        for (int v = 0; v < 8; ++v)
+          zz[v] = rep.faultf(SITE_SMEM, (long long)(by * 8 + xr) * a.W + col0 + v, zz[v]);
+      }
+      const float cu = a.C[u][xr];
+#pragma unroll
+      for (int v = 0; v < 8; ++v) y[v] = xr == 0 ? __fmul_rn(cu, zz[v]) : __fmaf_rn(cu, zz[v], y[v]);
+    }
+    // Stores (measured per variant at 8192^2): none, intra_reg and intra_nolds
+    // first swap one 16-B half between output rows u and u^4 of a block through
+    // a shuffle, so that store h writes rows 4h..4h+3 of the warp's blocks as
+    // whole 128-B lines (lanes u < 4: half 0 of row 4h + u; lanes u >= 4: half 1
+    // of row 4h + u - 4) -- none 0.155 -> 0.145 ms, intra_reg 0.272 -> 0.253 ms;
+    // intra_smem and the inter variants were slower with it and store their own
+    // row u directly (8 rows of half-sectors per store).
+    constexpr bool XS = (V == V_NONE || V == V_INTRA_REG || V == V_INTRA_NOLDS);
+    const bool lowu = u < 4;
+    unsigned got[4];
+    if constexpr (XS) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) got[q] = rep.lshfl_xor(__float_as_uint(lowu ? y[4 + q] : y[q]), 4);
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      unsigned w[4];
+      unsigned orow, idx;
+      if constexpr (XS) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          w[q] = lowu ? (h == 0 ? __float_as_uint(y[q]) : got[q]) : (h == 0 ? got[q] : __float_as_uint(y[4 + q]));
+        orow = by * 8 + (lowu ? (unsigned)u + 4u * h : (unsigned)u - 4u + 4u * h);
+        idx = orow * a.W + col0 + (lowu ? 0u : 4u);
+      } else {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) w[q] = __float_as_uint(y[4 * h + q]);
+        orow = by * 8 + u;
+        idx = orow * a.W + col0 + 4 * h;
+      }
+      rep.template commit<4, 0>(active ? 0xFu : 0u, active ? idx : 0u, w, a.H * a.W,
+                                [&](unsigned i, unsigned m, const unsigned* v) {
+                                  if (m == 0xFu)
+                                    __stcs(reinterpret_cast<float4*>(a.Y + i),
+                                           make_float4(__uint_as_float(v[0]), __uint_as_float(v[1]),
+                                                       __uint_as_float(v[2]), __uint_as_float(v[3])));
+                                  else
+                                    for (int k = 0; k < 4; ++k)
+                                      if ((m >> k) & 1u) a.Y[i + k] = __uint_as_float(v[k]);
+                                },
+                                /*defer=*/h == 0);
+    }
   }
   rep.finish();
 }

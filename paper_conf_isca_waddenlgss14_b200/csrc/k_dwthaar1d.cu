@@ -53,132 +53,134 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dwt_kernel(DwtArgs a, Ctx c
   __shared__ __align__(16) float cbuf[Geom<V>::SMDUP == 2 ? PLANE + TE_MAX : TE_MAX];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned tile = (unsigned)rep.lblock;
-  const int te = 1 << a.tb;
-  const float s = __uint_as_float(S_BITS);
-  float* const cp = &rep.template smp<PLANE>(cbuf, 0);  // this replica's copy
-  const float* src = a.src + (size_t)tile * te;
+  for (; rep.active(); rep.advance()) {
+    const unsigned tile = (unsigned)rep.lblock;
+    const int te = 1 << a.tb;
+    const float s = __uint_as_float(S_BITS);
+    float* const cp = &rep.template smp<PLANE>(cbuf, 0);  // this replica's copy
+    const float* src = a.src + (size_t)tile * te;
 
-  // ---- load the tile (all of a thread's 16-B loads in flight first)
-  if (te >= 4) {
-    constexpr int IT = TE_MAX / (4 * BL);
-    const int nv = te >> 2;
-    float4 f[IT];
+    // ---- load the tile (all of a thread's 16-B loads in flight first)
+    if (te >= 4) {
+      constexpr int IT = TE_MAX / (4 * BL);
+      const int nv = te >> 2;
+      float4 f[IT];
 #pragma unroll
-    for (int it = 0; it < IT; ++it) {
-      const int vi = rep.ltid + it * BL;
-      f[it] = vi < nv ? __ldcs(reinterpret_cast<const float4*>(src) + vi) : make_float4(0.f, 0.f, 0.f, 0.f);
-    }
-#pragma unroll
-    for (int it = 0; it < IT; ++it) {
-      const int vi = rep.ltid + it * BL;
-      if (vi < nv) {  // same predicate in both replicas (a function of ltid)
-        unsigned w[4] = {__float_as_uint(f[it].x), __float_as_uint(f[it].y), __float_as_uint(f[it].z),
-                         __float_as_uint(f[it].w)};
-        if constexpr (M == M_FAULT) {
-          if (a.first) {
-#pragma unroll
-            for (int k = 0; k < 4; ++k) w[k] = rep.fault(SITE_LOAD, (long long)tile * te + 4 * vi + k, w[k]);
-          }
-        }
-        if (rep.template sts_ok<4>(w, (unsigned)(4 * vi)))
-          reinterpret_cast<float4*>(cp)[vi] =
-              make_float4(__uint_as_float(w[0]), __uint_as_float(w[1]), __uint_as_float(w[2]), __uint_as_float(w[3]));
+      for (int it = 0; it < IT; ++it) {
+        const int vi = rep.ltid + it * BL;
+        f[it] = vi < nv ? __ldcs(reinterpret_cast<const float4*>(src) + vi) : make_float4(0.f, 0.f, 0.f, 0.f);
       }
-    }
-  } else if (rep.ltid < te) {
-    unsigned w = __float_as_uint(src[rep.ltid]);
-    if constexpr (M == M_FAULT) {
-      if (a.first) w = rep.fault(SITE_LOAD, (long long)tile * te + rep.ltid, w);
-    }
-    if (rep.sts_ok1(w, (unsigned)rep.ltid)) cp[rep.ltid] = __uint_as_float(w);
-  }
-  __syncthreads();
-
-  // ---- levels 1..K: thread group g turns c[8g .. 8g+8) into 4 approximations
-  // (written back to c[4g .. 4g+4)) and 4 details (one vector commit)
-  for (int k = 1; k <= a.K; ++k) {
-    const int half = te >> k, ng = half >> 2;
-    const int nu = (ng + BL - 1) / BL;  // 1 or 2 (uniform over the CTA)
-    float av[2][4], dv[2][4];
 #pragma unroll
-    for (int u = 0; u < 2; ++u) {
-      const int g = rep.ltid + u * BL;
-      if (u < nu && g < ng) {
-        const float4 p = reinterpret_cast<const float4*>(cp)[2 * g];
-        const float4 q = reinterpret_cast<const float4*>(cp)[2 * g + 1];
-        float x[8] = {p.x, p.y, p.z, p.w, q.x, q.y, q.z, q.w};
-        if constexpr (M == M_FAULT) {
-          if (a.first && k == 2) {  // level-1 approximations read back from smem
-#pragma unroll
-            for (int t = 0; t < 8; ++t) x[t] = rep.faultf(SITE_SMEM, (long long)tile * (te >> 1) + 8 * g + t, x[t]);
-          }
-        }
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          av[u][i] = __fmul_rn(__fadd_rn(x[2 * i], x[2 * i + 1]), s);
-          dv[u][i] = __fmul_rn(__fsub_rn(x[2 * i], x[2 * i + 1]), s);
+      for (int it = 0; it < IT; ++it) {
+        const int vi = rep.ltid + it * BL;
+        if (vi < nv) {  // same predicate in both replicas (a function of ltid)
+          unsigned w[4] = {__float_as_uint(f[it].x), __float_as_uint(f[it].y), __float_as_uint(f[it].z),
+                           __float_as_uint(f[it].w)};
           if constexpr (M == M_FAULT) {
-            if (a.first && k == 1) av[u][i] = rep.faultf(SITE_COMPUTE, (long long)tile * (te >> 1) + 4 * g + i, av[u][i]);
-          }
-        }
-      }
-    }
-    __syncthreads();  // every read of this level precedes the first write-back
-    // a warp none of whose logical threads has a group this level skips the
-    // commit: the decision is the same in both replicas (a function of ltid, k)
-    const int lw0 = rep.ltid - rep.llane;  // first logical thread of this warp
+            if (a.first) {
 #pragma unroll
-    for (int u = 0; u < 2; ++u) {
-      if (u < nu && lw0 + u * BL < ng) {
-        const int g = rep.ltid + u * BL;
-        const bool act = g < ng;
-        if (act) {
-          const unsigned aw[4] = {__float_as_uint(av[u][0]), __float_as_uint(av[u][1]), __float_as_uint(av[u][2]),
-                                  __float_as_uint(av[u][3])};
-          if (rep.template sts_ok<4>(aw, (unsigned)(4 * g)))
-            reinterpret_cast<float4*>(cp)[g] = make_float4(av[u][0], av[u][1], av[u][2], av[u][3]);
+              for (int k = 0; k < 4; ++k) w[k] = rep.fault(SITE_LOAD, (long long)tile * te + 4 * vi + k, w[k]);
+            }
+          }
+          if (rep.template sts_ok<4>(w, (unsigned)(4 * vi)))
+            reinterpret_cast<float4*>(cp)[vi] =
+                make_float4(__uint_as_float(w[0]), __uint_as_float(w[1]), __uint_as_float(w[2]), __uint_as_float(w[3]));
         }
-        unsigned dw[4] = {__float_as_uint(dv[u][0]), __float_as_uint(dv[u][1]), __float_as_uint(dv[u][2]),
-                          __float_as_uint(dv[u][3])};
-        const unsigned idx = (a.M >> k) + tile * (unsigned)half + 4u * (unsigned)g;
-        rep.template commit<4, 0>(act ? 0xFu : 0u, act ? idx : 0u, dw, a.M,
-                                  [&](unsigned i, unsigned m, const unsigned* w) { st_y(a.y, i, m, w); },
-                                  /*defer=*/u + 1 < nu && lw0 + (u + 1) * BL < ng);
       }
+    } else if (rep.ltid < te) {
+      unsigned w = __float_as_uint(src[rep.ltid]);
+      if constexpr (M == M_FAULT) {
+        if (a.first) w = rep.fault(SITE_LOAD, (long long)tile * te + rep.ltid, w);
+      }
+      if (rep.sts_ok1(w, (unsigned)rep.ltid)) cp[rep.ltid] = __uint_as_float(w);
     }
     __syncthreads();
-  }
 
-  // ---- the remaining m = min(te, 4) approximations of the tile
-  if (rep.warp == 0) {
-    const int m = te >> a.K;
-    const bool me = rep.ltid == 0;
-    unsigned w[4] = {0u, 0u, 0u, 0u};
-    if (me) {
-      float c0 = cp[0], c1 = m > 1 ? cp[1] : 0.f, c2 = m > 2 ? cp[2] : 0.f, c3 = m > 3 ? cp[3] : 0.f;
-      if (!a.last) {
-        w[0] = __float_as_uint(c0); w[1] = __float_as_uint(c1); w[2] = __float_as_uint(c2); w[3] = __float_as_uint(c3);
-      } else if (m == 4) {
-        const float a0 = __fmul_rn(__fadd_rn(c0, c1), s), d0 = __fmul_rn(__fsub_rn(c0, c1), s);
-        const float a1 = __fmul_rn(__fadd_rn(c2, c3), s), d1 = __fmul_rn(__fsub_rn(c2, c3), s);
-        w[0] = __float_as_uint(__fmul_rn(__fadd_rn(a0, a1), s));
-        w[1] = __float_as_uint(__fmul_rn(__fsub_rn(a0, a1), s));
-        w[2] = __float_as_uint(d0);
-        w[3] = __float_as_uint(d1);
-      } else if (m == 2) {
-        w[0] = __float_as_uint(__fmul_rn(__fadd_rn(c0, c1), s));
-        w[1] = __float_as_uint(__fmul_rn(__fsub_rn(c0, c1), s));
-      } else {
-        w[0] = __float_as_uint(c0);
+    // ---- levels 1..K: thread group g turns c[8g .. 8g+8) into 4 approximations
+    // (written back to c[4g .. 4g+4)) and 4 details (one vector commit)
+    for (int k = 1; k <= a.K; ++k) {
+      const int half = te >> k, ng = half >> 2;
+      const int nu = (ng + BL - 1) / BL;  // 1 or 2 (uniform over the CTA)
+      float av[2][4], dv[2][4];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int g = rep.ltid + u * BL;
+        if (u < nu && g < ng) {
+          const float4 p = reinterpret_cast<const float4*>(cp)[2 * g];
+          const float4 q = reinterpret_cast<const float4*>(cp)[2 * g + 1];
+          float x[8] = {p.x, p.y, p.z, p.w, q.x, q.y, q.z, q.w};
+          if constexpr (M == M_FAULT) {
+            if (a.first && k == 2) {  // level-1 approximations read back from smem
+#pragma unroll
+              for (int t = 0; t < 8; ++t) x[t] = rep.faultf(SITE_SMEM, (long long)tile * (te >> 1) + 8 * g + t, x[t]);
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            av[u][i] = __fmul_rn(__fadd_rn(x[2 * i], x[2 * i + 1]), s);
+            dv[u][i] = __fmul_rn(__fsub_rn(x[2 * i], x[2 * i + 1]), s);
+            if constexpr (M == M_FAULT) {
+              if (a.first && k == 1) av[u][i] = rep.faultf(SITE_COMPUTE, (long long)tile * (te >> 1) + 4 * g + i, av[u][i]);
+            }
+          }
+        }
       }
+      __syncthreads();  // every read of this level precedes the first write-back
+      // a warp none of whose logical threads has a group this level skips the
+      // commit: the decision is the same in both replicas (a function of ltid, k)
+      const int lw0 = rep.ltid - rep.llane;  // first logical thread of this warp
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        if (u < nu && lw0 + u * BL < ng) {
+          const int g = rep.ltid + u * BL;
+          const bool act = g < ng;
+          if (act) {
+            const unsigned aw[4] = {__float_as_uint(av[u][0]), __float_as_uint(av[u][1]), __float_as_uint(av[u][2]),
+                                    __float_as_uint(av[u][3])};
+            if (rep.template sts_ok<4>(aw, (unsigned)(4 * g)))
+              reinterpret_cast<float4*>(cp)[g] = make_float4(av[u][0], av[u][1], av[u][2], av[u][3]);
+          }
+          unsigned dw[4] = {__float_as_uint(dv[u][0]), __float_as_uint(dv[u][1]), __float_as_uint(dv[u][2]),
+                            __float_as_uint(dv[u][3])};
+          const unsigned idx = (a.M >> k) + tile * (unsigned)half + 4u * (unsigned)g;
+          rep.template commit<4, 0>(act ? 0xFu : 0u, act ? idx : 0u, dw, a.M,
+                                    [&](unsigned i, unsigned m, const unsigned* w) { st_y(a.y, i, m, w); },
+                                    /*defer=*/u + 1 < nu && lw0 + (u + 1) * BL < ng);
+        }
+      }
+      __syncthreads();
     }
-    if (a.last) {
-      const unsigned mask = me ? ((1u << m) - 1u) : 0u;
-      rep.template commit<4, 0>(mask, 0u, w, a.M, [&](unsigned i, unsigned mm, const unsigned* x) { st_y(a.y, i, mm, x); });
-    } else {
-      rep.template commit<4, 1>(me ? 0xFu : 0u, me ? 4u * tile : 0u, w, a.M >> a.K,
-                                [&](unsigned i, unsigned mm, const unsigned* x) { st_y(a.approx, i, mm, x); });
+
+    // ---- the remaining m = min(te, 4) approximations of the tile
+    if (rep.warp == 0) {
+      const int m = te >> a.K;
+      const bool me = rep.ltid == 0;
+      unsigned w[4] = {0u, 0u, 0u, 0u};
+      if (me) {
+        float c0 = cp[0], c1 = m > 1 ? cp[1] : 0.f, c2 = m > 2 ? cp[2] : 0.f, c3 = m > 3 ? cp[3] : 0.f;
+        if (!a.last) {
+          w[0] = __float_as_uint(c0); w[1] = __float_as_uint(c1); w[2] = __float_as_uint(c2); w[3] = __float_as_uint(c3);
+        } else if (m == 4) {
+          const float a0 = __fmul_rn(__fadd_rn(c0, c1), s), d0 = __fmul_rn(__fsub_rn(c0, c1), s);
+          const float a1 = __fmul_rn(__fadd_rn(c2, c3), s), d1 = __fmul_rn(__fsub_rn(c2, c3), s);
+          w[0] = __float_as_uint(__fmul_rn(__fadd_rn(a0, a1), s));
+          w[1] = __float_as_uint(__fmul_rn(__fsub_rn(a0, a1), s));
+          w[2] = __float_as_uint(d0);
+          w[3] = __float_as_uint(d1);
+        } else if (m == 2) {
+          w[0] = __float_as_uint(__fmul_rn(__fadd_rn(c0, c1), s));
+          w[1] = __float_as_uint(__fmul_rn(__fsub_rn(c0, c1), s));
+        } else {
+          w[0] = __float_as_uint(c0);
+        }
+      }
+      if (a.last) {
+        const unsigned mask = me ? ((1u << m) - 1u) : 0u;
+        rep.template commit<4, 0>(mask, 0u, w, a.M, [&](unsigned i, unsigned mm, const unsigned* x) { st_y(a.y, i, mm, x); });
+      } else {
+        rep.template commit<4, 1>(me ? 0xFu : 0u, me ? 4u * tile : 0u, w, a.M >> a.K,
+                                  [&](unsigned i, unsigned mm, const unsigned* x) { st_y(a.approx, i, mm, x); });
+      }
     }
   }
   rep.finish();

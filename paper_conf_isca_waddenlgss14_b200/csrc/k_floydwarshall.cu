@@ -42,14 +42,16 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_init_kernel(FwArgs a, Ct
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned e0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * 4;
-  const unsigned nn = a.n * a.n;
-  unsigned w[4];
-  unsigned i = e0 / a.n;
+  for (; rep.active(); rep.advance()) {
+    const unsigned e0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * 4;
+    const unsigned nn = a.n * a.n;
+    unsigned w[4];
+    unsigned i = e0 / a.n;
 #pragma unroll
-  for (int q = 0; q < 4; ++q) w[q] = i;
-  rep.template commit<4, 2>(e0 < nn ? 0xFu : 0u, e0 < nn ? e0 : 0u, w, nn,
-                            [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
+    for (int q = 0; q < 4; ++q) w[q] = i;
+    rep.template commit<4, 2>(e0 < nn ? 0xFu : 0u, e0 < nn ? e0 : 0u, w, nn,
+                              [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
+  }
   rep.finish();
 }
 
@@ -77,54 +79,56 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ct
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned nn = a.n * a.n;
-  // logical CTA = (row i, column chunk of BL*4*VPT words): the row and chunk
-  // are CTA-uniform (no per-thread division)
-  const unsigned cpr = (a.n + BL * 4 * VPT - 1) / (BL * 4 * VPT);
-  const unsigned i = (unsigned)rep.lblock / cpr;
-  const unsigned jc = ((unsigned)rep.lblock - i * cpr) * (BL * 4 * VPT);
-  const unsigned dik0 = a.D[(size_t)i * a.n + a.k];  // one broadcast word per CTA row
-  // all VPT vector pairs in flight before the first use (L2 latency-bound:
-  // an intra warp carries half the distinct bytes of an unprotected warp)
-  uint4 dkj[VPT], dij[VPT];
+  for (; rep.active(); rep.advance()) {
+    const unsigned nn = a.n * a.n;
+    // logical CTA = (row i, column chunk of BL*4*VPT words): the row and chunk
+    // are CTA-uniform (no per-thread division)
+    const unsigned cpr = (a.n + BL * 4 * VPT - 1) / (BL * 4 * VPT);
+    const unsigned i = (unsigned)rep.lblock / cpr;
+    const unsigned jc = ((unsigned)rep.lblock - i * cpr) * (BL * 4 * VPT);
+    const unsigned dik0 = a.D[(size_t)i * a.n + a.k];  // one broadcast word per CTA row
+    // all VPT vector pairs in flight before the first use (L2 latency-bound:
+    // an intra warp carries half the distinct bytes of an unprotected warp)
+    uint4 dkj[VPT], dij[VPT];
 #pragma unroll
-  for (int it = 0; it < VPT; ++it) {
-    const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
-    dkj[it] = make_uint4(0, 0, 0, 0);
-    dij[it] = make_uint4(0, 0, 0, 0);
-    if (j < a.n) {
-      dkj[it] = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
-      dij[it] = *reinterpret_cast<const uint4*>(a.D + i * a.n + j);
+    for (int it = 0; it < VPT; ++it) {
+      const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
+      dkj[it] = make_uint4(0, 0, 0, 0);
+      dij[it] = make_uint4(0, 0, 0, 0);
+      if (j < a.n) {
+        dkj[it] = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
+        dij[it] = *reinterpret_cast<const uint4*>(a.D + i * a.n + j);
+      }
     }
-  }
 #pragma unroll
-  for (int it = 0; it < VPT; ++it) {
-    const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
-    const bool active = j < a.n;
-    const unsigned e0 = i * a.n + j;
-    unsigned dik = dik0;
-    unsigned kj[4] = {dkj[it].x, dkj[it].y, dkj[it].z, dkj[it].w};
-    unsigned ij[4] = {dij[it].x, dij[it].y, dij[it].z, dij[it].w};
-    if constexpr (M == M_FAULT) {
-      dik = rep.fault(SITE_LOAD, (long long)i * a.n + a.k, dik);
+    for (int it = 0; it < VPT; ++it) {
+      const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
+      const bool active = j < a.n;
+      const unsigned e0 = i * a.n + j;
+      unsigned dik = dik0;
+      unsigned kj[4] = {dkj[it].x, dkj[it].y, dkj[it].z, dkj[it].w};
+      unsigned ij[4] = {dij[it].x, dij[it].y, dij[it].z, dij[it].w};
+      if constexpr (M == M_FAULT) {
+        dik = rep.fault(SITE_LOAD, (long long)i * a.n + a.k, dik);
 #pragma unroll
-      for (int q = 0; q < 4; ++q) ij[q] = rep.fault(SITE_LOAD, (long long)e0 + q, ij[q]);
+        for (int q = 0; q < 4; ++q) ij[q] = rep.fault(SITE_LOAD, (long long)e0 + q, ij[q]);
+      }
+      unsigned nd[4], np[4], mask = 0;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        unsigned cand = dik + kj[q];
+        if constexpr (M == M_FAULT) cand = rep.fault(SITE_COMPUTE, (long long)e0 + q, cand);
+        const bool better = active && cand < ij[q];
+        mask |= (better ? 1u : 0u) << q;
+        nd[q] = cand;
+        np[q] = a.k;
+      }
+      rep.template commit<4, 0, false, true>(mask, active ? e0 : 0u, nd, nn,
+                                [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); },
+                                /*defer=*/true);
+      rep.template commit<4, 1, false, true>(mask, active ? e0 : 0u, np, nn,
+                                [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
     }
-    unsigned nd[4], np[4], mask = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      unsigned cand = dik + kj[q];
-      if constexpr (M == M_FAULT) cand = rep.fault(SITE_COMPUTE, (long long)e0 + q, cand);
-      const bool better = active && cand < ij[q];
-      mask |= (better ? 1u : 0u) << q;
-      nd[q] = cand;
-      np[q] = a.k;
-    }
-    rep.template commit<4, 0, false, true>(mask, active ? e0 : 0u, nd, nn,
-                              [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); },
-                              /*defer=*/true);
-    rep.template commit<4, 1, false, true>(mask, active ? e0 : 0u, np, nn,
-                              [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
   }
   rep.finish();
 }

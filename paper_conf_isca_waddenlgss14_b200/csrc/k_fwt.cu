@@ -209,100 +209,102 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
   __shared__ float tile[Geom<V>::SMDUP == 2 ? PLANE + S::WORDS : S::WORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned tileid = (unsigned)rep.lblock;
-  const int te = KIND != 0 ? TE_MAX : 1 << a.tb;  // full tiles in the specialised passes
-  float* const tp = &rep.template smp<PLANE>(tile, 0);  // this replica's plane
-  // load: 16-B vectors, contiguous in both the tile and global memory
-  auto put4 = [&](int e0, unsigned g, float (&w)[4]) {
-    unsigned xw[4];
+  for (; rep.active(); rep.advance()) {
+    const unsigned tileid = (unsigned)rep.lblock;
+    const int te = KIND != 0 ? TE_MAX : 1 << a.tb;  // full tiles in the specialised passes
+    float* const tp = &rep.template smp<PLANE>(tile, 0);  // this replica's plane
+    // load: 16-B vectors, contiguous in both the tile and global memory
+    auto put4 = [&](int e0, unsigned g, float (&w)[4]) {
+      unsigned xw[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      if constexpr (M == M_FAULT) {
-        if (a.s0 == 0 && e0 + k < te) w[k] = rep.faultf(SITE_LOAD, (long long)g + k, w[k]);
+      for (int k = 0; k < 4; ++k) {
+        if constexpr (M == M_FAULT) {
+          if (a.s0 == 0 && e0 + k < te) w[k] = rep.faultf(SITE_LOAD, (long long)g + k, w[k]);
+        }
+        xw[k] = __float_as_uint(w[k]);
       }
-      xw[k] = __float_as_uint(w[k]);
-    }
-    if (rep.template sts_ok<4>(xw, (unsigned)e0)) {
+      if (rep.template sts_ok<4>(xw, (unsigned)e0)) {
 #pragma unroll
-      for (int k = 0; k < 4; ++k)
-        if (KIND != 0 || e0 + k < te) tp[S::phys(e0 + k)] = w[k];
-    }
-  };
-  if constexpr (KIND != 0) {
-    // full tile: all of this thread's loads in flight before the first use
-    constexpr int IT = TE_MAX / (4 * BL);
-    float4 f[IT];
-#pragma unroll
-    for (int it = 0; it < IT; ++it)
-      f[it] = *reinterpret_cast<const float4*>(a.src + gindex_k<KIND>(a, tileid, (unsigned)(4 * rep.ltid + it * 4 * BL)));
-#pragma unroll
-    for (int it = 0; it < IT; ++it) {
-      const int e0 = 4 * rep.ltid + it * 4 * BL;
-      float w[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
-      put4(e0, gindex_k<KIND>(a, tileid, (unsigned)e0), w);
-    }
-  } else {
-    for (int e0 = 4 * rep.ltid; e0 < te; e0 += 4 * BL) {
-      const unsigned g = gindex(a, tileid, (unsigned)e0);
-      float w[4];
-      if (te >= 4) {
-        float4 f = *reinterpret_cast<const float4*>(a.src + g);
-        w[0] = f.x; w[1] = f.y; w[2] = f.z; w[3] = f.w;
-      } else {
-#pragma unroll
-        for (int k = 0; k < 4; ++k) w[k] = e0 + k < te ? a.src[g + k] : 0.0f;
-      }
-      put4(e0, g, w);
-    }
-  }
-  __syncthreads();
-  // stages [s0, s0 + b) live at tile bits [c, c + b); rounds of <= 4 stages
-  if constexpr (KIND == 1) {
-    fwt_round_ct<4, 0>(rep, tp, a, tileid, 0);
-    __syncthreads();
-    fwt_round_ct<4, 4>(rep, tp, a, tileid, 1);
-    __syncthreads();
-    fwt_round_ct<4, 8>(rep, tp, a, tileid, 2);
-    __syncthreads();
-  } else if constexpr (KIND == 2) {
-    fwt_round_ct<4, 5>(rep, tp, a, tileid, 0);
-    __syncthreads();
-    fwt_round_ct<3, 9>(rep, tp, a, tileid, 1);
-    __syncthreads();
-  } else {
-    int round_no = 0;
-    for (int q = a.c; q < a.c + a.b; q += 4, ++round_no) {
-      const int nb = min(4, a.c + a.b - q);
-      switch (nb) {
-        case 4: fwt_round<4>(rep, tp, q, te, a, tileid, round_no); break;
-        case 3: fwt_round<3>(rep, tp, q, te, a, tileid, round_no); break;
-        case 2: fwt_round<2>(rep, tp, q, te, a, tileid, round_no); break;
-        default: fwt_round<1>(rep, tp, q, te, a, tileid, round_no); break;
-      }
-      __syncthreads();
-    }
-  }
-  // store: one vector commit per 4 elements
-#pragma unroll 1
-  for (int it = 0; it < TE_MAX / (4 * BL); ++it) {
-    const int e0 = 4 * rep.ltid + it * 4 * BL;
-    unsigned w[4];
-    unsigned mask = 0;
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const bool in = KIND != 0 || e0 + k < te;  // specialised passes: full tiles
-      w[k] = in ? __float_as_uint(tp[S::phys(e0 + k)]) : 0u;
-      mask |= (in ? 1u : 0u) << k;
-    }
-    const unsigned g = e0 < te ? gindex_k<KIND>(a, tileid, (unsigned)e0) : 0u;
-    rep.template commit<4, 0>(mask, g, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
-      if (m == 0xFu)
-        *reinterpret_cast<float4*>(a.dst + idx) =
-            make_float4(__uint_as_float(x[0]), __uint_as_float(x[1]), __uint_as_float(x[2]), __uint_as_float(x[3]));
-      else
         for (int k = 0; k < 4; ++k)
-          if ((m >> k) & 1u) a.dst[idx + k] = __uint_as_float(x[k]);
-    }, /*defer=*/it < TE_MAX / (4 * BL) - 1);
+          if (KIND != 0 || e0 + k < te) tp[S::phys(e0 + k)] = w[k];
+      }
+    };
+    if constexpr (KIND != 0) {
+      // full tile: all of this thread's loads in flight before the first use
+      constexpr int IT = TE_MAX / (4 * BL);
+      float4 f[IT];
+#pragma unroll
+      for (int it = 0; it < IT; ++it)
+        f[it] = *reinterpret_cast<const float4*>(a.src + gindex_k<KIND>(a, tileid, (unsigned)(4 * rep.ltid + it * 4 * BL)));
+#pragma unroll
+      for (int it = 0; it < IT; ++it) {
+        const int e0 = 4 * rep.ltid + it * 4 * BL;
+        float w[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
+        put4(e0, gindex_k<KIND>(a, tileid, (unsigned)e0), w);
+      }
+    } else {
+      for (int e0 = 4 * rep.ltid; e0 < te; e0 += 4 * BL) {
+        const unsigned g = gindex(a, tileid, (unsigned)e0);
+        float w[4];
+        if (te >= 4) {
+          float4 f = *reinterpret_cast<const float4*>(a.src + g);
+          w[0] = f.x; w[1] = f.y; w[2] = f.z; w[3] = f.w;
+        } else {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) w[k] = e0 + k < te ? a.src[g + k] : 0.0f;
+        }
+        put4(e0, g, w);
+      }
+    }
+    __syncthreads();
+    // stages [s0, s0 + b) live at tile bits [c, c + b); rounds of <= 4 stages
+    if constexpr (KIND == 1) {
+      fwt_round_ct<4, 0>(rep, tp, a, tileid, 0);
+      __syncthreads();
+      fwt_round_ct<4, 4>(rep, tp, a, tileid, 1);
+      __syncthreads();
+      fwt_round_ct<4, 8>(rep, tp, a, tileid, 2);
+      __syncthreads();
+    } else if constexpr (KIND == 2) {
+      fwt_round_ct<4, 5>(rep, tp, a, tileid, 0);
+      __syncthreads();
+      fwt_round_ct<3, 9>(rep, tp, a, tileid, 1);
+      __syncthreads();
+    } else {
+      int round_no = 0;
+      for (int q = a.c; q < a.c + a.b; q += 4, ++round_no) {
+        const int nb = min(4, a.c + a.b - q);
+        switch (nb) {
+          case 4: fwt_round<4>(rep, tp, q, te, a, tileid, round_no); break;
+          case 3: fwt_round<3>(rep, tp, q, te, a, tileid, round_no); break;
+          case 2: fwt_round<2>(rep, tp, q, te, a, tileid, round_no); break;
+          default: fwt_round<1>(rep, tp, q, te, a, tileid, round_no); break;
+        }
+        __syncthreads();
+      }
+    }
+    // store: one vector commit per 4 elements
+#pragma unroll 1
+    for (int it = 0; it < TE_MAX / (4 * BL); ++it) {
+      const int e0 = 4 * rep.ltid + it * 4 * BL;
+      unsigned w[4];
+      unsigned mask = 0;
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const bool in = KIND != 0 || e0 + k < te;  // specialised passes: full tiles
+        w[k] = in ? __float_as_uint(tp[S::phys(e0 + k)]) : 0u;
+        mask |= (in ? 1u : 0u) << k;
+      }
+      const unsigned g = e0 < te ? gindex_k<KIND>(a, tileid, (unsigned)e0) : 0u;
+      rep.template commit<4, 0>(mask, g, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
+        if (m == 0xFu)
+          *reinterpret_cast<float4*>(a.dst + idx) =
+              make_float4(__uint_as_float(x[0]), __uint_as_float(x[1]), __uint_as_float(x[2]), __uint_as_float(x[3]));
+        else
+          for (int k = 0; k < 4; ++k)
+            if ((m >> k) & 1u) a.dst[idx + k] = __uint_as_float(x[k]);
+      }, /*defer=*/it < TE_MAX / (4 * BL) - 1);
+    }
   }
   rep.finish();
 }
@@ -354,77 +356,79 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, C
   __shared__ __align__(16) float tile[DUPL ? P1_PLANE + P1_WORDS : P1_WORDS];
   R rep(c);
   rep.init(mb);
-  const unsigned tileid = (unsigned)rep.lblock;
-  const unsigned gbase = tileid << TB_MAX;
-  float* const tp = tile + (DUPL ? P1_PLANE * rep.r : 0);  // this replica's plane
-  const int t = rep.ltid;
-  // load: 8 coalesced float4 per thread, all in flight before the first use
-  float4 f[8];
+  for (; rep.active(); rep.advance()) {
+    const unsigned tileid = (unsigned)rep.lblock;
+    const unsigned gbase = tileid << TB_MAX;
+    float* const tp = tile + (DUPL ? P1_PLANE * rep.r : 0);  // this replica's plane
+    const int t = rep.ltid;
+    // load: 8 coalesced float4 per thread, all in flight before the first use
+    float4 f[8];
 #pragma unroll
-  for (int it = 0; it < 8; ++it) f[it] = *reinterpret_cast<const float4*>(a.src + gbase + 4 * t + 512 * it);
-  float* const ps = tp + p1_phys(4 * t);  // + p1_phys(512 it) + k: compile-time offsets
+    for (int it = 0; it < 8; ++it) f[it] = *reinterpret_cast<const float4*>(a.src + gbase + 4 * t + 512 * it);
+    float* const ps = tp + p1_phys(4 * t);  // + p1_phys(512 it) + k: compile-time offsets
 #pragma unroll
-  for (int it = 0; it < 8; ++it) {
-    const int e0 = 4 * t + 512 * it;
-    float v[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
-    if constexpr (M == M_FAULT) {
+    for (int it = 0; it < 8; ++it) {
+      const int e0 = 4 * t + 512 * it;
+      float v[4] = {f[it].x, f[it].y, f[it].z, f[it].w};
+      if constexpr (M == M_FAULT) {
 #pragma unroll
-      for (int k = 0; k < 4; ++k) v[k] = rep.faultf(SITE_LOAD, (long long)gbase + e0 + k, v[k]);
-    }
-    butterflies<2>(v);  // stages 0, 1 (element bits 0, 1)
-    unsigned w[4];
+        for (int k = 0; k < 4; ++k) v[k] = rep.faultf(SITE_LOAD, (long long)gbase + e0 + k, v[k]);
+      }
+      butterflies<2>(v);  // stages 0, 1 (element bits 0, 1)
+      unsigned w[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_COMPUTE, (long long)gbase + e0 + k, v[k]);
-      w[k] = __float_as_uint(v[k]);
-    }
-    if (rep.template sts_ok<4>(w, (unsigned)e0)) {
-      if constexpr (PAD) {
-        *reinterpret_cast<float4*>(ps + p1_phys(512 * it)) = make_float4(v[0], v[1], v[2], v[3]);
-      } else {
+      for (int k = 0; k < 4; ++k) {
+        if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_COMPUTE, (long long)gbase + e0 + k, v[k]);
+        w[k] = __float_as_uint(v[k]);
+      }
+      if (rep.template sts_ok<4>(w, (unsigned)e0)) {
+        if constexpr (PAD) {
+          *reinterpret_cast<float4*>(ps + p1_phys(512 * it)) = make_float4(v[0], v[1], v[2], v[3]);
+        } else {
 #pragma unroll
-        for (int k = 0; k < 4; ++k) tp[p1x(e0 + k)] = v[k];
+          for (int k = 0; k < 4; ++k) tp[p1x(e0 + k)] = v[k];
+        }
       }
     }
-  }
-  __syncthreads();
-  {  // round A: stages 2..6 on elements ebase + 4k
-    const int ebase = (t & 3) | ((t >> 2) << 7);
-    float* const pb = tp + p1_phys(ebase);  // + p1_phys(4k): compile-time offsets
-    auto at = [&](int k) -> float& { return PAD ? pb[p1_phys(4 * k)] : tp[p1x(ebase + 4 * k)]; };
+    __syncthreads();
+    {  // round A: stages 2..6 on elements ebase + 4k
+      const int ebase = (t & 3) | ((t >> 2) << 7);
+      float* const pb = tp + p1_phys(ebase);  // + p1_phys(4k): compile-time offsets
+      auto at = [&](int k) -> float& { return PAD ? pb[p1_phys(4 * k)] : tp[p1x(ebase + 4 * k)]; };
+      float v[32];
+#pragma unroll
+      for (int k = 0; k < 32; ++k) {
+        v[k] = at(k);
+        if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_SMEM, (long long)gbase + ebase + 4 * k, v[k]);
+      }
+      butterflies<5>(v);
+      unsigned w[32];
+#pragma unroll
+      for (int k = 0; k < 32; ++k) w[k] = __float_as_uint(v[k]);
+      // each thread reads and rewrites its own 32 elements: no barrier inside the round
+      if (rep.template sts_ok<32>(w, (unsigned)ebase)) {
+#pragma unroll
+        for (int k = 0; k < 32; ++k) at(k) = v[k];
+      }
+    }
+    __syncthreads();
+    // round B: stages 7..11 on elements t + 128k, then 8 strided commits
+    float* const pt = tp + p1_phys(t);
     float v[32];
 #pragma unroll
-    for (int k = 0; k < 32; ++k) {
-      v[k] = at(k);
-      if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_SMEM, (long long)gbase + ebase + 4 * k, v[k]);
-    }
+    for (int k = 0; k < 32; ++k) v[k] = PAD ? pt[p1_phys(128 * k)] : tp[p1x(t + 128 * k)];
     butterflies<5>(v);
-    unsigned w[32];
 #pragma unroll
-    for (int k = 0; k < 32; ++k) w[k] = __float_as_uint(v[k]);
-    // each thread reads and rewrites its own 32 elements: no barrier inside the round
-    if (rep.template sts_ok<32>(w, (unsigned)ebase)) {
+    for (int j = 0; j < 8; ++j) {
+      unsigned w[4];
 #pragma unroll
-      for (int k = 0; k < 32; ++k) at(k) = v[k];
+      for (int u = 0; u < 4; ++u) w[u] = __float_as_uint(v[4 * j + u]);
+      rep.template commit<4, 0>(0xFu, gbase + t + 512 * j, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if ((m >> u) & 1u) a.dst[idx + 128 * u] = __uint_as_float(x[u]);
+      }, /*defer=*/j < 7, /*stride=*/128u);
     }
-  }
-  __syncthreads();
-  // round B: stages 7..11 on elements t + 128k, then 8 strided commits
-  float* const pt = tp + p1_phys(t);
-  float v[32];
-#pragma unroll
-  for (int k = 0; k < 32; ++k) v[k] = PAD ? pt[p1_phys(128 * k)] : tp[p1x(t + 128 * k)];
-  butterflies<5>(v);
-#pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    unsigned w[4];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) w[u] = __float_as_uint(v[4 * j + u]);
-    rep.template commit<4, 0>(0xFu, gbase + t + 512 * j, w, a.N, [&](unsigned idx, unsigned m, const unsigned* x) {
-#pragma unroll
-      for (int u = 0; u < 4; ++u)
-        if ((m >> u) & 1u) a.dst[idx + 128 * u] = __uint_as_float(x[u]);
-    }, /*defer=*/j < 7, /*stride=*/128u);
   }
   rep.finish();
 }
@@ -440,46 +444,48 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_ps_kernel(FwtArgs a, C
   __shared__ float tile[TE_MAX * Geom<V>::SMDUP];
   R rep(c);
   rep.init(mb);
-  const unsigned tileid = (unsigned)rep.lblock;
-  const int t = rep.ltid;
-  const int col = t & 31, g = t >> 5;
-  // this replica's plane, column pre-applied (bank bit 4 flipped for replica 1):
-  // element (col, row) is tc[row << 5], a compile-time offset from a per-thread base
-  float* const tc = tile + (DUPL ? TE_MAX * rep.r : 0) + (col ^ (DUPL && rep.r ? 16 : 0));
-  // global index of tile element (col, row): row bits land at s0.. (gindex_k<2>)
-  const int midb = a.s0 - 5;
-  const unsigned gcol = ((tileid >> midb) << (a.s0 + 7)) | ((tileid & ((1u << midb) - 1u)) << 5) | (unsigned)col;
-  // rows 32 g + i, i = 0..31: one 128-B row per warp load
-  float v[32];
+  for (; rep.active(); rep.advance()) {
+    const unsigned tileid = (unsigned)rep.lblock;
+    const int t = rep.ltid;
+    const int col = t & 31, g = t >> 5;
+    // this replica's plane, column pre-applied (bank bit 4 flipped for replica 1):
+    // element (col, row) is tc[row << 5], a compile-time offset from a per-thread base
+    float* const tc = tile + (DUPL ? TE_MAX * rep.r : 0) + (col ^ (DUPL && rep.r ? 16 : 0));
+    // global index of tile element (col, row): row bits land at s0.. (gindex_k<2>)
+    const int midb = a.s0 - 5;
+    const unsigned gcol = ((tileid >> midb) << (a.s0 + 7)) | ((tileid & ((1u << midb) - 1u)) << 5) | (unsigned)col;
+    // rows 32 g + i, i = 0..31: one 128-B row per warp load
+    float v[32];
 #pragma unroll
-  for (int i = 0; i < 32; ++i) v[i] = a.src[gcol + ((unsigned)(32 * g + i) << a.s0)];
-  butterflies<5>(v);  // stages s0 .. s0+4 (row bits 0..4)
-  unsigned w[32];
+    for (int i = 0; i < 32; ++i) v[i] = a.src[gcol + ((unsigned)(32 * g + i) << a.s0)];
+    butterflies<5>(v);  // stages s0 .. s0+4 (row bits 0..4)
+    unsigned w[32];
 #pragma unroll
-  for (int i = 0; i < 32; ++i) w[i] = __float_as_uint(v[i]);
-  if (rep.template sts_ok<32>(w, (unsigned)(col | (32 * g) << 5))) {
+    for (int i = 0; i < 32; ++i) w[i] = __float_as_uint(v[i]);
+    if (rep.template sts_ok<32>(w, (unsigned)(col | (32 * g) << 5))) {
 #pragma unroll
-    for (int i = 0; i < 32; ++i) tc[(32 * g + i) << 5] = v[i];
-  }
-  __syncthreads();
-  // stages s0+5, s0+6 (row bits 5, 6): 8 groups of 4 rows {rlo + 32 k}
+      for (int i = 0; i < 32; ++i) tc[(32 * g + i) << 5] = v[i];
+    }
+    __syncthreads();
+    // stages s0+5, s0+6 (row bits 5, 6): 8 groups of 4 rows {rlo + 32 k}
 #pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const int rlo = g + 4 * j;
-    float q[4];
+    for (int j = 0; j < 8; ++j) {
+      const int rlo = g + 4 * j;
+      float q[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) q[k] = tc[(rlo + 32 * k) << 5];
-    butterflies<2>(q);
-    unsigned x[4];
+      for (int k = 0; k < 4; ++k) q[k] = tc[(rlo + 32 * k) << 5];
+      butterflies<2>(q);
+      unsigned x[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) x[k] = __float_as_uint(q[k]);
-    const unsigned stride = 1u << (a.s0 + 5);
-    rep.template commit<4, 0>(0xFu, gcol + ((unsigned)rlo << a.s0), x, a.N,
-                              [&](unsigned idx, unsigned m, const unsigned* y) {
+      for (int k = 0; k < 4; ++k) x[k] = __float_as_uint(q[k]);
+      const unsigned stride = 1u << (a.s0 + 5);
+      rep.template commit<4, 0>(0xFu, gcol + ((unsigned)rlo << a.s0), x, a.N,
+                                [&](unsigned idx, unsigned m, const unsigned* y) {
 #pragma unroll
-                                for (int k = 0; k < 4; ++k)
-                                  if ((m >> k) & 1u) a.dst[idx + stride * k] = __uint_as_float(y[k]);
-                              }, /*defer=*/j < 7, stride);
+                                  for (int k = 0; k < 4; ++k)
+                                    if ((m >> k) & 1u) a.dst[idx + stride * k] = __uint_as_float(y[k]);
+                                }, /*defer=*/j < 7, stride);
+    }
   }
   rep.finish();
 }

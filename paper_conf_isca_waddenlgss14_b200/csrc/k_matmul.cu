@@ -311,7 +311,8 @@ int matmul_run(Launch& L) {
   const unsigned G = (M / BM) * (N / BN);
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, Mo = decltype(vm)::M;
-    return launch_std<V>(L, mm_kernel<V, Mo>, mm_kernel<V_NONE, M_NORMAL>, G, BL, MmCfg<V>::SMEM, a, "matmul");
+    return launch_std<V>(L, mm_kernel<V, Mo>, mm_kernel<V_NONE, M_NORMAL>, G, BL, MmCfg<V>::SMEM, a, "matmul",
+                         /*persistent=*/false);
   });
 }
 

@@ -58,47 +58,49 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_reduce_kernel(PsArgs a, 
   __shared__ unsigned sw[(BL / (32 / DUP)) * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned ch = (unsigned)rep.lblock;
-  const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
-  unsigned s = 0;
-  // 16-B coalesced loads, 4 in flight per thread (chunk starts are 16-B aligned)
-  // blocks of 16 BL elements visited from the END of the chunk: the scan pass
-  // reads each chunk from its start, which is then what L2 still holds
-  const unsigned nblk = hi > lo ? (hi - lo + 16 * BL - 1) / (16 * BL) : 0u;
+  for (; rep.active(); rep.advance()) {
+    const unsigned ch = (unsigned)rep.lblock;
+    const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
+    unsigned s = 0;
+    // 16-B coalesced loads, 4 in flight per thread (chunk starts are 16-B aligned)
+    // blocks of 16 BL elements visited from the END of the chunk: the scan pass
+    // reads each chunk from its start, which is then what L2 still holds
+    const unsigned nblk = hi > lo ? (hi - lo + 16 * BL - 1) / (16 * BL) : 0u;
 #pragma unroll 1
-  for (unsigned b = nblk; b-- > 0;) {
-    const unsigned e = lo + b * 16 * BL + 4 * rep.ltid;
-    uint4 v[4];
+    for (unsigned b = nblk; b-- > 0;) {
+      const unsigned e = lo + b * 16 * BL + 4 * rep.ltid;
+      uint4 v[4];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const unsigned f = e + u * 4 * BL;
-      if (f + 4 <= hi) {
-        v[u] = __ldg(reinterpret_cast<const uint4*>(a.x + f));
-      } else {  // ragged tail of the array
-        v[u].x = f < hi ? a.x[f] : 0u;
-        v[u].y = f + 1 < hi ? a.x[f + 1] : 0u;
-        v[u].z = f + 2 < hi ? a.x[f + 2] : 0u;
-        v[u].w = 0u;
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      if constexpr (M == M_FAULT) {
+      for (int u = 0; u < 4; ++u) {
         const unsigned f = e + u * 4 * BL;
-        v[u].x = rep.fault(SITE_LOAD, (long long)f, v[u].x);
-        v[u].y = rep.fault(SITE_LOAD, (long long)f + 1, v[u].y);
-        v[u].z = rep.fault(SITE_LOAD, (long long)f + 2, v[u].z);
-        v[u].w = rep.fault(SITE_LOAD, (long long)f + 3, v[u].w);
+        if (f + 4 <= hi) {
+          v[u] = __ldg(reinterpret_cast<const uint4*>(a.x + f));
+        } else {  // ragged tail of the array
+          v[u].x = f < hi ? a.x[f] : 0u;
+          v[u].y = f + 1 < hi ? a.x[f + 1] : 0u;
+          v[u].z = f + 2 < hi ? a.x[f + 2] : 0u;
+          v[u].w = 0u;
+        }
       }
-      s += v[u].x + v[u].y + v[u].z + v[u].w;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        if constexpr (M == M_FAULT) {
+          const unsigned f = e + u * 4 * BL;
+          v[u].x = rep.fault(SITE_LOAD, (long long)f, v[u].x);
+          v[u].y = rep.fault(SITE_LOAD, (long long)f + 1, v[u].y);
+          v[u].z = rep.fault(SITE_LOAD, (long long)f + 2, v[u].z);
+          v[u].w = rep.fault(SITE_LOAD, (long long)f + 3, v[u].w);
+        }
+        s += v[u].x + v[u].y + v[u].z + v[u].w;
+      }
     }
-  }
-  s = rep.fault(SITE_COMPUTE, (long long)ch * BL + rep.ltid, s);
-  const unsigned t = block_sum_u32(rep, s, sw);
-  if (rep.warp == 0) {  // one store per CTA leaves the SoR ("ghost" warps)
-    unsigned w[1] = {t};
-    rep.template commit<1, 2>(rep.llane == 0 ? 1u : 0u, ch, w, a.nch,
-                              [&](unsigned i, unsigned, const unsigned* x) { a.partial[i] = x[0]; });
+    s = rep.fault(SITE_COMPUTE, (long long)ch * BL + rep.ltid, s);
+    const unsigned t = block_sum_u32(rep, s, sw);
+    if (rep.warp == 0) {  // one store per CTA leaves the SoR ("ghost" warps)
+      unsigned w[1] = {t};
+      rep.template commit<1, 2>(rep.llane == 0 ? 1u : 0u, ch, w, a.nch,
+                                [&](unsigned i, unsigned, const unsigned* x) { a.partial[i] = x[0]; });
+    }
   }
   rep.finish();
 }
@@ -123,134 +125,136 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_k
   __shared__ unsigned sw[NQ * NLW * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned ch = a.nch - 1u - (unsigned)rep.lblock;  // reverse order: L2-hot chunks first
-  // carry-in: sum of the partials of all earlier chunks (L2-resident)
-  unsigned cs = 0;
-  for (unsigned i = rep.ltid; i < ch; i += BL) cs += __ldcg(a.partial + i);
-  unsigned carry = a.carry_in + block_sum_u32(rep, cs, sw);
-  const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
-  const int lw = rep.ltid / LW;
-  // Register double buffer: the next tile's loads are in flight while this
-  // tile is scanned and stored.  v[q * RUN + k] = x[t0 + q SUB + ltid RUN + k].
-  auto load_tile = [&](unsigned t0, unsigned (&v)[ITEMS]) {
+  for (; rep.active(); rep.advance()) {
+    const unsigned ch = a.nch - 1u - (unsigned)rep.lblock;  // reverse order: L2-hot chunks first
+    // carry-in: sum of the partials of all earlier chunks (L2-resident)
+    unsigned cs = 0;
+    for (unsigned i = rep.ltid; i < ch; i += BL) cs += __ldcg(a.partial + i);
+    unsigned carry = a.carry_in + block_sum_u32(rep, cs, sw);
+    const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
+    const int lw = rep.ltid / LW;
+    // Register double buffer: the next tile's loads are in flight while this
+    // tile is scanned and stored.  v[q * RUN + k] = x[t0 + q SUB + ltid RUN + k].
+    auto load_tile = [&](unsigned t0, unsigned (&v)[ITEMS]) {
 #pragma unroll
-    for (int q = 0; q < NQ; ++q) {
-      const unsigned e = t0 + q * SUB + RUN * (unsigned)rep.ltid;
-      if (e + RUN <= hi) {
-        if (RUN % 8 == 0 && a.v8) {  // 256-bit loads: 32 B per lane, whole lines per instruction
+      for (int q = 0; q < NQ; ++q) {
+        const unsigned e = t0 + q * SUB + RUN * (unsigned)rep.ltid;
+        if (e + RUN <= hi) {
+          if (RUN % 8 == 0 && a.v8) {  // 256-bit loads: 32 B per lane, whole lines per instruction
 #pragma unroll
-          for (int j = 0; j < RUN / 8; ++j) {
-            unsigned w[8];
-            ldcs8(a.x + e + 8 * j, w);
+            for (int j = 0; j < RUN / 8; ++j) {
+              unsigned w[8];
+              ldcs8(a.x + e + 8 * j, w);
 #pragma unroll
-            for (int k = 0; k < 8; ++k) v[q * RUN + 8 * j + k] = w[k];
+              for (int k = 0; k < 8; ++k) v[q * RUN + 8 * j + k] = w[k];
+            }
+          } else {
+#pragma unroll
+            for (int j = 0; j < RUN / 4; ++j) {
+              uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.x + e) + j);
+              v[q * RUN + 4 * j] = w.x; v[q * RUN + 4 * j + 1] = w.y;
+              v[q * RUN + 4 * j + 2] = w.z; v[q * RUN + 4 * j + 3] = w.w;
+            }
           }
         } else {
 #pragma unroll
-          for (int j = 0; j < RUN / 4; ++j) {
-            uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.x + e) + j);
-            v[q * RUN + 4 * j] = w.x; v[q * RUN + 4 * j + 1] = w.y;
-            v[q * RUN + 4 * j + 2] = w.z; v[q * RUN + 4 * j + 3] = w.w;
-          }
+          for (int k = 0; k < RUN; ++k) v[q * RUN + k] = e + k < hi ? a.x[e + k] : 0u;
         }
-      } else {
-#pragma unroll
-        for (int k = 0; k < RUN; ++k) v[q * RUN + k] = e + k < hi ? a.x[e + k] : 0u;
       }
-    }
-  };
-  unsigned nxt[ITEMS];
-  if (lo < hi) load_tile(lo, nxt);
+    };
+    unsigned nxt[ITEMS];
+    if (lo < hi) load_tile(lo, nxt);
 #pragma unroll 1
-  for (unsigned t0 = lo; t0 < hi; t0 += TILE) {  // uniform trip count per CTA
-    unsigned v[ITEMS];
+    for (unsigned t0 = lo; t0 < hi; t0 += TILE) {  // uniform trip count per CTA
+      unsigned v[ITEMS];
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) v[i] = nxt[i];
-    if (t0 + TILE < hi) load_tile(t0 + TILE, nxt);
-    if constexpr (M == M_FAULT) {
+      for (int i = 0; i < ITEMS; ++i) v[i] = nxt[i];
+      if (t0 + TILE < hi) load_tile(t0 + TILE, nxt);
+      if constexpr (M == M_FAULT) {
 #pragma unroll
-      for (int i = 0; i < ITEMS; ++i)
-        v[i] = rep.fault(SITE_LOAD, (long long)t0 + (i / RUN) * SUB + RUN * rep.ltid + (i % RUN), v[i]);
-    }
-    unsigned tsum[NQ], ws[NQ];
-#pragma unroll
-    for (int q = 0; q < NQ; ++q) {  // thread-local inclusive scans
-#pragma unroll
-      for (int k = 1; k < RUN; ++k) v[q * RUN + k] += v[q * RUN + k - 1];
-      tsum[q] = ws[q] = v[q * RUN + RUN - 1];
-    }
-#pragma unroll
-    for (int d = 1; d < LW; d <<= 1) {  // logical-warp scans, NQ independent chains
-#pragma unroll
-      for (int q = 0; q < NQ; ++q) {
-        const unsigned u = rep.lshfl_up(ws[q], d);
-        if (rep.llane >= d) ws[q] += u;
+        for (int i = 0; i < ITEMS; ++i)
+          v[i] = rep.fault(SITE_LOAD, (long long)t0 + (i / RUN) * SUB + RUN * rep.ltid + (i % RUN), v[i]);
       }
-    }
+      unsigned tsum[NQ], ws[NQ];
 #pragma unroll
-    for (int q = 0; q < NQ; ++q)  // warp totals, sub-tile-major
-      if (rep.llane == LW - 1 && rep.sts_ok1(ws[q], q * NLW + lw)) rep.sm(sw, q * NLW + lw) = ws[q];
-    __syncthreads();
-    unsigned pre[NQ];  // exclusive prefix of this thread's sub-tile-q run within the tile
-    unsigned total;
-    if constexpr (FLAT) {
-      // lane l holds total l = (sub-tile l / NLW, warp l % NLW): one scan over the lanes
-      unsigned wt = rep.sm(sw, rep.llane);
-      if constexpr (M == M_FAULT) wt = rep.fault(SITE_SMEM, (long long)ch * BL + rep.llane, wt);
-      unsigned winc = wt;
+      for (int q = 0; q < NQ; ++q) {  // thread-local inclusive scans
 #pragma unroll
-      for (int d = 1; d < LW; d <<= 1) {
-        const unsigned u = rep.lshfl_up(winc, d);
-        if (rep.llane >= d) winc += u;
-      }
-      const unsigned wex = winc - wt;
-#pragma unroll
-      for (int q = 0; q < NQ; ++q) pre[q] = rep.lshfl_idx(wex, q * NLW + lw);
-      total = rep.lshfl_idx(winc, LW - 1);
-    } else {
-      unsigned wt[NQ], winc[NQ];
-#pragma unroll
-      for (int q = 0; q < NQ; ++q) {
-        wt[q] = rep.llane < NLW ? rep.sm(sw, q * NLW + rep.llane) : 0u;
-        if constexpr (M == M_FAULT) wt[q] = rep.fault(SITE_SMEM, (long long)ch * BL + q * NLW + rep.llane, wt[q]);
-        winc[q] = wt[q];
+        for (int k = 1; k < RUN; ++k) v[q * RUN + k] += v[q * RUN + k - 1];
+        tsum[q] = ws[q] = v[q * RUN + RUN - 1];
       }
 #pragma unroll
-      for (int d = 1; d < NLW; d <<= 1) {
+      for (int d = 1; d < LW; d <<= 1) {  // logical-warp scans, NQ independent chains
 #pragma unroll
         for (int q = 0; q < NQ; ++q) {
-          const unsigned u = rep.lshfl_up(winc[q], d);
-          if (rep.llane >= d) winc[q] += u;
+          const unsigned u = rep.lshfl_up(ws[q], d);
+          if (rep.llane >= d) ws[q] += u;
         }
       }
-      total = 0;
 #pragma unroll
-      for (int q = 0; q < NQ; ++q) {
-        pre[q] = total + rep.lshfl_idx(winc[q] - wt[q], lw);
-        total += rep.lshfl_idx(winc[q], NLW - 1);
+      for (int q = 0; q < NQ; ++q)  // warp totals, sub-tile-major
+        if (rep.llane == LW - 1 && rep.sts_ok1(ws[q], q * NLW + lw)) rep.sm(sw, q * NLW + lw) = ws[q];
+      __syncthreads();
+      unsigned pre[NQ];  // exclusive prefix of this thread's sub-tile-q run within the tile
+      unsigned total;
+      if constexpr (FLAT) {
+        // lane l holds total l = (sub-tile l / NLW, warp l % NLW): one scan over the lanes
+        unsigned wt = rep.sm(sw, rep.llane);
+        if constexpr (M == M_FAULT) wt = rep.fault(SITE_SMEM, (long long)ch * BL + rep.llane, wt);
+        unsigned winc = wt;
+#pragma unroll
+        for (int d = 1; d < LW; d <<= 1) {
+          const unsigned u = rep.lshfl_up(winc, d);
+          if (rep.llane >= d) winc += u;
+        }
+        const unsigned wex = winc - wt;
+#pragma unroll
+        for (int q = 0; q < NQ; ++q) pre[q] = rep.lshfl_idx(wex, q * NLW + lw);
+        total = rep.lshfl_idx(winc, LW - 1);
+      } else {
+        unsigned wt[NQ], winc[NQ];
+#pragma unroll
+        for (int q = 0; q < NQ; ++q) {
+          wt[q] = rep.llane < NLW ? rep.sm(sw, q * NLW + rep.llane) : 0u;
+          if constexpr (M == M_FAULT) wt[q] = rep.fault(SITE_SMEM, (long long)ch * BL + q * NLW + rep.llane, wt[q]);
+          winc[q] = wt[q];
+        }
+#pragma unroll
+        for (int d = 1; d < NLW; d <<= 1) {
+#pragma unroll
+          for (int q = 0; q < NQ; ++q) {
+            const unsigned u = rep.lshfl_up(winc[q], d);
+            if (rep.llane >= d) winc[q] += u;
+          }
+        }
+        total = 0;
+#pragma unroll
+        for (int q = 0; q < NQ; ++q) {
+          pre[q] = total + rep.lshfl_idx(winc[q] - wt[q], lw);
+          total += rep.lshfl_idx(winc[q], NLW - 1);
+        }
       }
-    }
-    __syncthreads();  // sw is reused by the next tile
+      __syncthreads();  // sw is reused by the next tile
 #pragma unroll
-    for (int i = 0; i < ITEMS / 4; ++i) {
-      const int q = (4 * i) / RUN;
-      const unsigned e0 = t0 + q * SUB + RUN * (unsigned)rep.ltid + (4 * i) % RUN;
-      const unsigned prefix = carry + pre[q] + (ws[q] - tsum[q]);
-      unsigned w[4];
-      unsigned mask = 0;
+      for (int i = 0; i < ITEMS / 4; ++i) {
+        const int q = (4 * i) / RUN;
+        const unsigned e0 = t0 + q * SUB + RUN * (unsigned)rep.ltid + (4 * i) % RUN;
+        const unsigned prefix = carry + pre[q] + (ws[q] - tsum[q]);
+        unsigned w[4];
+        unsigned mask = 0;
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        w[k] = prefix + v[4 * i + k];
-        mask |= (e0 + k < hi ? 1u : 0u) << k;
+        for (int k = 0; k < 4; ++k) {
+          w[k] = prefix + v[4 * i + k];
+          mask |= (e0 + k < hi ? 1u : 0u) << k;
+        }
+        rep.template commit<4, 0>(mask, mask ? e0 : 0u, w, a.n, [&](unsigned idx, unsigned m, const unsigned* x) {
+          if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.y + idx), make_uint4(x[0], x[1], x[2], x[3]));
+          else
+            for (int k = 0; k < 4; ++k)
+              if ((m >> k) & 1u) a.y[idx + k] = x[k];
+        }, /*defer=*/i < ITEMS / 4 - 1);
       }
-      rep.template commit<4, 0>(mask, mask ? e0 : 0u, w, a.n, [&](unsigned idx, unsigned m, const unsigned* x) {
-        if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.y + idx), make_uint4(x[0], x[1], x[2], x[3]));
-        else
-          for (int k = 0; k < 4; ++k)
-            if ((m >> k) & 1u) a.y[idx + k] = x[k];
-      }, /*defer=*/i < ITEMS / 4 - 1);
+      carry += total;
     }
-    carry += total;
   }
   rep.finish();
 }

@@ -56,39 +56,41 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) red_partial_kernel(RedArgs 
   __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned T = (unsigned)c.nblocks * BL;  // logical threads in the grid
-  const unsigned gt = (unsigned)rep.lblock * BL + rep.ltid;
-  unsigned long long s = 0;
-  const unsigned nvec = a.n / 4;
-  for (unsigned base = 0; base < nvec; base += T * UNROLL) {
-    uint4 v[UNROLL];
+  for (; rep.active(); rep.advance()) {
+    const unsigned T = (unsigned)c.nblocks * BL;  // logical threads in the grid
+    const unsigned gt = (unsigned)rep.lblock * BL + rep.ltid;
+    unsigned long long s = 0;
+    const unsigned nvec = a.n / 4;
+    for (unsigned base = 0; base < nvec; base += T * UNROLL) {
+      uint4 v[UNROLL];
 #pragma unroll
-    for (int u = 0; u < UNROLL; ++u) {
-      unsigned vi = base + u * T + gt;
-      v[u] = vi < nvec ? __ldcs(reinterpret_cast<const uint4*>(a.x) + vi) : make_uint4(0, 0, 0, 0);
-    }
-#pragma unroll
-    for (int u = 0; u < UNROLL; ++u) {
-      unsigned e = (base + u * T + gt) * 4;
-      if constexpr (M == M_FAULT) {
-        v[u].x = rep.fault(SITE_LOAD, (long long)e, v[u].x);
-        v[u].y = rep.fault(SITE_LOAD, (long long)e + 1, v[u].y);
-        v[u].z = rep.fault(SITE_LOAD, (long long)e + 2, v[u].z);
-        v[u].w = rep.fault(SITE_LOAD, (long long)e + 3, v[u].w);
+      for (int u = 0; u < UNROLL; ++u) {
+        unsigned vi = base + u * T + gt;
+        v[u] = vi < nvec ? __ldcs(reinterpret_cast<const uint4*>(a.x) + vi) : make_uint4(0, 0, 0, 0);
       }
-      s += (unsigned long long)v[u].x + v[u].y + (unsigned long long)v[u].z + v[u].w;
+#pragma unroll
+      for (int u = 0; u < UNROLL; ++u) {
+        unsigned e = (base + u * T + gt) * 4;
+        if constexpr (M == M_FAULT) {
+          v[u].x = rep.fault(SITE_LOAD, (long long)e, v[u].x);
+          v[u].y = rep.fault(SITE_LOAD, (long long)e + 1, v[u].y);
+          v[u].z = rep.fault(SITE_LOAD, (long long)e + 2, v[u].z);
+          v[u].w = rep.fault(SITE_LOAD, (long long)e + 3, v[u].w);
+        }
+        s += (unsigned long long)v[u].x + v[u].y + (unsigned long long)v[u].z + v[u].w;
+      }
     }
-  }
-  // ragged tail (< 4 elements), indexed in 64 bits: n may be within T of 2^32
-  for (unsigned long long e = (unsigned long long)nvec * 4 + gt; e < a.n; e += T)
-    s += rep.fault(SITE_LOAD, (long long)e, a.x[e]);
-  s = (s & 0xffffffff00000000ull) | rep.fault(SITE_COMPUTE, (long long)gt, (unsigned)s);
-  unsigned long long t = block_sum(rep, s, sm_warp);
-  if (rep.warp == 0) {  // warp-uniform: only warp 0 holds the CTA's store (P:809 ghost warps)
-    unsigned v[2] = {(unsigned)t, (unsigned)(t >> 32)};
-    unsigned mask = rep.llane == 0 ? 3u : 0u;
-    rep.template commit<2, 0>(mask, 2u * (unsigned)rep.lblock, v, 2u * (unsigned)c.nblocks,
-                              [&](unsigned idx, unsigned m, const unsigned* w) { store_u64(a.out, idx, m, w); });
+    // ragged tail (< 4 elements), indexed in 64 bits: n may be within T of 2^32
+    for (unsigned long long e = (unsigned long long)nvec * 4 + gt; e < a.n; e += T)
+      s += rep.fault(SITE_LOAD, (long long)e, a.x[e]);
+    s = (s & 0xffffffff00000000ull) | rep.fault(SITE_COMPUTE, (long long)gt, (unsigned)s);
+    unsigned long long t = block_sum(rep, s, sm_warp);
+    if (rep.warp == 0) {  // warp-uniform: only warp 0 holds the CTA's store (P:809 ghost warps)
+      unsigned v[2] = {(unsigned)t, (unsigned)(t >> 32)};
+      unsigned mask = rep.llane == 0 ? 3u : 0u;
+      rep.template commit<2, 0>(mask, 2u * (unsigned)rep.lblock, v, 2u * (unsigned)c.nblocks,
+                                [&](unsigned idx, unsigned m, const unsigned* w) { store_u64(a.out, idx, m, w); });
+    }
   }
   rep.finish();
 }
@@ -100,14 +102,16 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) red_final_kernel(RedArgs a,
   __shared__ unsigned long long sm_warp[(BL / (32 / DUP)) * Geom<V>::SMDUP];
   Rep<V, M> rep(c);
   rep.init(mb);
-  unsigned long long s = 0;
-  for (unsigned i = rep.ltid; i < a.n; i += BL) s += a.partials[i];
-  unsigned long long t = block_sum(rep, s, sm_warp);
-  if (rep.warp == 0) {
-    unsigned v[2] = {(unsigned)t, (unsigned)(t >> 32)};
-    unsigned mask = rep.llane == 0 ? 3u : 0u;
-    rep.template commit<2, 1>(mask, 0u, v, 2u,
-                              [&](unsigned idx, unsigned m, const unsigned* w) { store_u64(a.out, idx, m, w); });
+  for (; rep.active(); rep.advance()) {
+    unsigned long long s = 0;
+    for (unsigned i = rep.ltid; i < a.n; i += BL) s += a.partials[i];
+    unsigned long long t = block_sum(rep, s, sm_warp);
+    if (rep.warp == 0) {
+      unsigned v[2] = {(unsigned)t, (unsigned)(t >> 32)};
+      unsigned mask = rep.llane == 0 ? 3u : 0u;
+      rep.template commit<2, 1>(mask, 0u, v, 2u,
+                                [&](unsigned idx, unsigned m, const unsigned* w) { store_u64(a.out, idx, m, w); });
+    }
   }
   rep.finish();
 }

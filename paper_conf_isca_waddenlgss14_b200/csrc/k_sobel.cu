@@ -130,71 +130,73 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) sobel_kernel(SobArgs a, Ctx
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
-  const unsigned x0 = (bx * BL + (unsigned)rep.ltid) * 4;
-  const bool active = x0 < a.W;
-  const int y0 = (int)(by * RY);
-  unsigned xin = 0;  // interior columns among this thread's 4 pixels (loop-invariant)
+  for (; rep.active(); rep.advance()) {
+    const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
+    const unsigned x0 = (bx * BL + (unsigned)rep.ltid) * 4;
+    const bool active = x0 < a.W;
+    const int y0 = (int)(by * RY);
+    unsigned xin = 0;  // interior columns among this thread's 4 pixels (loop-invariant)
 #pragma unroll
-  for (int p = 0; p < 4; ++p) xin |= ((x0 + p >= 1 && x0 + p < a.W - 1) ? 1u : 0u) << p;
-  // one output row from the window (t = y-1, m = y, b = y+1)
-  auto row_out = [&](int y, const Row& t, const Row& m, const Row& b) {
-    unsigned vs_lo[6], vs_hi[6], vd_lo[6], vd_hi[6];
+    for (int p = 0; p < 4; ++p) xin |= ((x0 + p >= 1 && x0 + p < a.W - 1) ? 1u : 0u) << p;
+    // one output row from the window (t = y-1, m = y, b = y+1)
+    auto row_out = [&](int y, const Row& t, const Row& m, const Row& b) {
+      unsigned vs_lo[6], vs_hi[6], vd_lo[6], vd_hi[6];
 #pragma unroll
-    for (int k = 0; k < 6; ++k) {
-      vs_lo[k] = t.lo[k] + 2u * m.lo[k] + b.lo[k];   // <= 1020 per lane
-      vs_hi[k] = t.hi[k] + 2u * m.hi[k] + b.hi[k];
-      vd_lo[k] = t.lo[k] + 0x01000100u - b.lo[k];    // 256 + (top - bot)
-      vd_hi[k] = t.hi[k] + 0x01000100u - b.hi[k];
-    }
-    const bool yin = y >= 1 && y < (int)a.H - 1;
-    unsigned out[4];
+      for (int k = 0; k < 6; ++k) {
+        vs_lo[k] = t.lo[k] + 2u * m.lo[k] + b.lo[k];   // <= 1020 per lane
+        vs_hi[k] = t.hi[k] + 2u * m.hi[k] + b.hi[k];
+        vd_lo[k] = t.lo[k] + 0x01000100u - b.lo[k];    // 256 + (top - bot)
+        vd_hi[k] = t.hi[k] + 0x01000100u - b.hi[k];
+      }
+      const bool yin = y >= 1 && y < (int)a.H - 1;
+      unsigned out[4];
 #pragma unroll
-    for (int p = 0; p < 4; ++p) {
-      const int w = p + 1;
-      // biased by 1024 per 16-bit lane
-      unsigned gx_lo = vd_lo[w - 1] + 2u * vd_lo[w] + vd_lo[w + 1];
-      const unsigned gx_hi = vd_hi[w - 1] + 2u * vd_hi[w] + vd_hi[w + 1];
-      const unsigned gy_lo = vs_lo[w - 1] + 0x04000400u - vs_lo[w + 1];
-      const unsigned gy_hi = vs_hi[w - 1] + 0x04000400u - vs_hi[w + 1];
-      if constexpr (M == M_FAULT) gx_lo = rep.fault(SITE_COMPUTE, (long long)y * a.W + x0 + p, gx_lo);
-      unsigned m0, m2, m1, m3;
-      sobel_mag2(gx_lo, gy_lo, m0, m2);  // channels 0, 2
-      sobel_mag2(gx_hi, gy_hi, m1, m3);  // channels 1, 3
-      // two channels per 16-bit lane pair, saturated with one VIMNMX.U16x2 each
-      const unsigned h01 = __vminu2(__byte_perm(m0, m1, 0x5410), 0x00FF00FFu);
-      const unsigned h23 = __vminu2(__byte_perm(m2, m3, 0x5410), 0x00FF00FFu);
-      const unsigned px = __byte_perm(h01, h23, 0x6420);
-      out[p] = (yin && ((xin >> p) & 1u)) ? px : 0u;
-    }
-    const unsigned mask = (active && y < (int)a.H) ? 0xFu : 0u;
-    rep.template commit<4, 0>(mask, (unsigned)y * a.W + x0, out, a.H * a.W,
-                              [&](unsigned idx, unsigned mm, const unsigned* w) {
-                                if (mm == 0xFu)
-                                  __stcs(reinterpret_cast<uint4*>(a.O + idx), make_uint4(w[0], w[1], w[2], w[3]));
-                                else
-                                  for (int k = 0; k < 4; ++k)
-                                    if ((mm >> k) & 1u) a.O[idx + k] = w[k];
-                              });
-  };
-  // rolling 3-row window; the raw words of the row after next are in flight
-  // while the current row is filtered (one row of prefetch distance)
-  Row top, mid, bot;
-  unsigned raw[6], nxt[6];
-  load_raw(rep, a, y0 - 1, x0, active, raw);
-  unpack_row(rep, a, y0 - 1, x0, raw, top);
-  load_raw(rep, a, y0, x0, active, raw);
-  load_raw(rep, a, y0 + 1, x0, active, nxt);
-  unpack_row(rep, a, y0, x0, raw, mid);
+      for (int p = 0; p < 4; ++p) {
+        const int w = p + 1;
+        // biased by 1024 per 16-bit lane
+        unsigned gx_lo = vd_lo[w - 1] + 2u * vd_lo[w] + vd_lo[w + 1];
+        const unsigned gx_hi = vd_hi[w - 1] + 2u * vd_hi[w] + vd_hi[w + 1];
+        const unsigned gy_lo = vs_lo[w - 1] + 0x04000400u - vs_lo[w + 1];
+        const unsigned gy_hi = vs_hi[w - 1] + 0x04000400u - vs_hi[w + 1];
+        if constexpr (M == M_FAULT) gx_lo = rep.fault(SITE_COMPUTE, (long long)y * a.W + x0 + p, gx_lo);
+        unsigned m0, m2, m1, m3;
+        sobel_mag2(gx_lo, gy_lo, m0, m2);  // channels 0, 2
+        sobel_mag2(gx_hi, gy_hi, m1, m3);  // channels 1, 3
+        // two channels per 16-bit lane pair, saturated with one VIMNMX.U16x2 each
+        const unsigned h01 = __vminu2(__byte_perm(m0, m1, 0x5410), 0x00FF00FFu);
+        const unsigned h23 = __vminu2(__byte_perm(m2, m3, 0x5410), 0x00FF00FFu);
+        const unsigned px = __byte_perm(h01, h23, 0x6420);
+        out[p] = (yin && ((xin >> p) & 1u)) ? px : 0u;
+      }
+      const unsigned mask = (active && y < (int)a.H) ? 0xFu : 0u;
+      rep.template commit<4, 0>(mask, (unsigned)y * a.W + x0, out, a.H * a.W,
+                                [&](unsigned idx, unsigned mm, const unsigned* w) {
+                                  if (mm == 0xFu)
+                                    __stcs(reinterpret_cast<uint4*>(a.O + idx), make_uint4(w[0], w[1], w[2], w[3]));
+                                  else
+                                    for (int k = 0; k < 4; ++k)
+                                      if ((mm >> k) & 1u) a.O[idx + k] = w[k];
+                                });
+    };
+    // rolling 3-row window; the raw words of the row after next are in flight
+    // while the current row is filtered (one row of prefetch distance)
+    Row top, mid, bot;
+    unsigned raw[6], nxt[6];
+    load_raw(rep, a, y0 - 1, x0, active, raw);
+    unpack_row(rep, a, y0 - 1, x0, raw, top);
+    load_raw(rep, a, y0, x0, active, raw);
+    load_raw(rep, a, y0 + 1, x0, active, nxt);
+    unpack_row(rep, a, y0, x0, raw, mid);
 #pragma unroll 1
-  for (int y = y0; y < y0 + RY; ++y) {
+    for (int y = y0; y < y0 + RY; ++y) {
 #pragma unroll
-    for (int k = 0; k < 6; ++k) raw[k] = nxt[k];
-    load_raw(rep, a, y + 2, x0, active, nxt);
-    unpack_row(rep, a, y + 1, x0, raw, bot);
-    row_out(y, top, mid, bot);
-    top = mid;
-    mid = bot;
+      for (int k = 0; k < 6; ++k) raw[k] = nxt[k];
+      load_raw(rep, a, y + 2, x0, active, nxt);
+      unpack_row(rep, a, y + 1, x0, raw, bot);
+      row_out(y, top, mid, bot);
+      top = mid;
+      mid = bot;
+    }
   }
   rep.finish();
 }

@@ -36,51 +36,53 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) tr_kernel(TrArgs a, Ctx c) 
   __shared__ unsigned tile[Geom<V>::SMDUP == 2 ? PLANE + SWORDS : SWORDS];
   Rep<V, M> rep(c);
   rep.init(mb);
-  const unsigned ty = (unsigned)rep.lblock / a.nsx, sx = (unsigned)rep.lblock % a.nsx;
-  const unsigned r = rep.ltid / 8, l4 = (rep.ltid % 8) * 4;
-  // load phase: A row ty*32 + r, columns sx*128 + 32t + l4 .. +3
-  uint4 v[NT];
-  const unsigned gi = ty * TS + r;
+  for (; rep.active(); rep.advance()) {
+    const unsigned ty = (unsigned)rep.lblock / a.nsx, sx = (unsigned)rep.lblock % a.nsx;
+    const unsigned r = rep.ltid / 8, l4 = (rep.ltid % 8) * 4;
+    // load phase: A row ty*32 + r, columns sx*128 + 32t + l4 .. +3
+    uint4 v[NT];
+    const unsigned gi = ty * TS + r;
 #pragma unroll
-  for (int t = 0; t < NT; ++t) {
-    const unsigned gj = sx * (NT * TS) + t * TS + l4;
-    v[t] = (gi < a.H && gj < a.W) ? __ldcs(reinterpret_cast<const uint4*>(a.A + (size_t)gi * a.W + gj))
-                                  : make_uint4(0, 0, 0, 0);
-  }
-#pragma unroll
-  for (int t = 0; t < NT; ++t) {
-    unsigned w[4] = {v[t].x, v[t].y, v[t].z, v[t].w};
-    const unsigned gj = sx * (NT * TS) + t * TS + l4;
-    if constexpr (M == M_FAULT) {
-#pragma unroll
-      for (int k = 0; k < 4; ++k) w[k] = rep.fault(SITE_LOAD, (long long)gi * a.W + gj + k, w[k]);
+    for (int t = 0; t < NT; ++t) {
+      const unsigned gj = sx * (NT * TS) + t * TS + l4;
+      v[t] = (gi < a.H && gj < a.W) ? __ldcs(reinterpret_cast<const uint4*>(a.A + (size_t)gi * a.W + gj))
+                                    : make_uint4(0, 0, 0, 0);
     }
-    if (rep.template sts_ok<4>(w, t * TWORDS + r * PITCH + l4)) {
 #pragma unroll
-      for (int k = 0; k < 4; ++k) rep.template smp<PLANE>(tile, t * TWORDS + r * PITCH + l4 + k) = w[k];
+    for (int t = 0; t < NT; ++t) {
+      unsigned w[4] = {v[t].x, v[t].y, v[t].z, v[t].w};
+      const unsigned gj = sx * (NT * TS) + t * TS + l4;
+      if constexpr (M == M_FAULT) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) w[k] = rep.fault(SITE_LOAD, (long long)gi * a.W + gj + k, w[k]);
+      }
+      if (rep.template sts_ok<4>(w, t * TWORDS + r * PITCH + l4)) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k) rep.template smp<PLANE>(tile, t * TWORDS + r * PITCH + l4 + k) = w[k];
+      }
     }
-  }
-  __syncthreads();
-  // store phase: B row sx*128 + 32t + c (= a column of A), columns ty*32 + l4 .. +3
-  const unsigned cc = rep.ltid / 8;
+    __syncthreads();
+    // store phase: B row sx*128 + 32t + c (= a column of A), columns ty*32 + l4 .. +3
+    const unsigned cc = rep.ltid / 8;
 #pragma unroll
-  for (int t = 0; t < NT; ++t) {
-    const unsigned bi = sx * (NT * TS) + t * TS + cc, bj = ty * TS + l4;
-    unsigned w[4];
+    for (int t = 0; t < NT; ++t) {
+      const unsigned bi = sx * (NT * TS) + t * TS + cc, bj = ty * TS + l4;
+      unsigned w[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      w[k] = rep.template smp<PLANE>(tile, t * TWORDS + (l4 + k) * PITCH + cc);
-      if constexpr (M == M_FAULT) w[k] = rep.fault(SITE_SMEM, (long long)bi * a.H + bj + k, w[k]);
+      for (int k = 0; k < 4; ++k) {
+        w[k] = rep.template smp<PLANE>(tile, t * TWORDS + (l4 + k) * PITCH + cc);
+        if constexpr (M == M_FAULT) w[k] = rep.fault(SITE_SMEM, (long long)bi * a.H + bj + k, w[k]);
+      }
+      const unsigned mask = (bi < a.W && bj < a.H) ? 0xFu : 0u;
+      rep.template commit<4, 0>(mask, mask ? bi * a.H + bj : 0u, w, a.H * a.W,
+                                [&](unsigned idx, unsigned m, const unsigned* x) {
+                                  if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.B + idx), make_uint4(x[0], x[1], x[2], x[3]));
+                                  else
+                                    for (int k = 0; k < 4; ++k)
+                                      if ((m >> k) & 1u) a.B[idx + k] = x[k];
+                                },
+                                /*defer=*/t < NT - 1);
     }
-    const unsigned mask = (bi < a.W && bj < a.H) ? 0xFu : 0u;
-    rep.template commit<4, 0>(mask, mask ? bi * a.H + bj : 0u, w, a.H * a.W,
-                              [&](unsigned idx, unsigned m, const unsigned* x) {
-                                if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.B + idx), make_uint4(x[0], x[1], x[2], x[3]));
-                                else
-                                  for (int k = 0; k < 4; ++k)
-                                    if ((m >> k) & 1u) a.B[idx + k] = x[k];
-                              },
-                              /*defer=*/t < NT - 1);
   }
   rep.finish();
 }

@@ -158,6 +158,15 @@ int run_dup(Launch& L0, const KEntry& e, char* ws, bool armed, const FaultDesc& 
 
 void set_error(const std::string& msg) { g_err = msg; }
 
+#ifdef RMT_TRACE
+// experiment builds: a device buffer of 2^17 x 8 u64 milestones (Rep RMT_TR)
+unsigned long long* trace_buf() {
+  static unsigned long long* p = nullptr;
+  if (!p && cudaMalloc(&p, (size_t)(1u << 17) * 8 * 8) == cudaSuccess) cudaMemset(p, 0, (size_t)(1u << 17) * 64);
+  return p;
+}
+#endif
+
 int cuda_check(cudaError_t e, const char* what) {
   if (e == cudaSuccess) return RMT_OK;
   set_error(std::string(what) + ": " + cudaGetErrorString(e));
@@ -227,6 +236,9 @@ int rmt_launch(int kernel, int variant, const rmt_bufs_t* bufs, int64_t n, unsig
   L.ctx.wd = g_stress.wd ? g_stress.wd : WATCHDOG_CYCLES;
   L.ctx.stress = g_stress.flags;
   L.ctx.skew_ns = g_stress.skew_ns;
+#ifdef RMT_TRACE
+  L.ctx.trace = trace_buf();
+#endif
   L.cl_depth = (variant == RMT_INTER_CLUSTER) ? g_stress.depth : 0;
   char* ws = (char*)workspace;
   if (variant == RMT_INTER_GROUP) {
@@ -371,6 +383,13 @@ int rmt_set_ablation(int mode) {
 }
 
 int rmt_last_launch_count(void) { return g_last_launches; }
+
+#ifdef RMT_TRACE
+int rmt_trace_copy(void* host, size_t bytes) {  // experiment builds only
+  cudaDeviceSynchronize();
+  return cuda_check(cudaMemcpy(host, trace_buf(), bytes, cudaMemcpyDeviceToHost), "trace copy");
+}
+#endif
 
 int rmt_set_stress(int depth, int flags, int skew_ns, long long watchdog_cycles) {
   if (depth < 0 || depth > INTER_S || (depth & (depth - 1)) != 0 || flags < 0 ||

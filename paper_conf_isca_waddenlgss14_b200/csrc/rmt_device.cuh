@@ -75,9 +75,12 @@ struct Ctx {
   unsigned* payload;        // inter: R*W*S records of RING_WORDS*32 words
   int R, W, S;              // inter queue geometry (regions, warps per CTA, slots in use: 1..INTER_S)
   int nblocks;              // logical CTAs in this launch
+  int pairs;                // inter/cluster: physical replica pairs launched (2 * pairs CTAs)
+  int lstride;              // inter/cluster: logical-CTA stride of a pair (0: one logical CTA per pair)
   unsigned long long wd;    // watchdog bound in clock64 cycles (WATCHDOG_CYCLES unless a stress test lowers it)
   int stress;               // M_STRESS: STRESS_* bits
   unsigned skew_ns;         // M_STRESS: maximum random sleep (ns) per CTA start / per commit
+  unsigned long long* trace;  // RMT_TRACE experiment builds only: per-CTA globaltimer milestones
   FaultDesc f;
 };
 
@@ -161,6 +164,17 @@ __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
+// Inter queue publication/free (experiment knobs):
+// RMT_PUB_FENCE_SC=1 the producer's batch fence is fence.sc.gpu (else
+// fence.acq_rel.gpu); RMT_FREE_RELAXED=1 the consumer frees consumed slots with
+// relaxed stores issued after the warp ballot that consumed every loaded word
+// (else st.release.gpu, which also waits for the consumer's own output stores).
+#ifndef RMT_PUB_FENCE_SC
+#define RMT_PUB_FENCE_SC 1
+#endif
+#ifndef RMT_FREE_RELAXED
+#define RMT_FREE_RELAXED 0
+#endif
 #ifndef RMT_SPIN_NS0
 #define RMT_SPIN_NS0 32     // first back-off sleep of a queue wait (0: pure spin)
 #endif
@@ -203,6 +217,26 @@ __device__ __forceinline__ bool spin_cl(unsigned addr, unsigned want, const Ctx&
   }
 }
 
+// Experiment instrumentation (-DRMT_TRACE builds only): thread 0 of inter CTA
+// `ticket` stores globaltimer at milestone k (0 start, 1 after ticket + region
+// turn, 2 first commit entry, 3 first commit done, 4 finish entry, 5 finish
+// exit, 6 SM id, 7 role).
+#ifdef RMT_TRACE
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define RMT_TR(k, v)                                                                        \
+  do {                                                                                      \
+    if (c.trace && threadIdx.x == 0 && tr_id < (1u << 17)) c.trace[(size_t)tr_id * 8 + (k)] = (v); \
+  } while (0)
+#else
+#define RMT_TR(k, v) \
+  do {               \
+  } while (0)
+#endif
+
 // 32-bit mixer (stress skew and record tags): lowbias32
 __device__ __forceinline__ unsigned mix32(unsigned x) {
   x ^= x >> 16;
@@ -236,13 +270,38 @@ struct Rep {
   int lblock;     // logical CTA id
   int lane, warp, llane;
   unsigned j;     // records this warp has committed (inter)
+  int lstride;    // logical CTAs advance by this (0: this CTA runs one logical CTA)
   unsigned nerr;  // intra: mismatching commits of this (consumer) lane, added to *err at finish()
   unsigned pend;  // inter: records not yet published (producer) / freed (consumer)
   unsigned region, epoch;
   unsigned* mbox;  // intra_smem: this warp's mailbox
+  unsigned tr_id;  // RMT_TRACE: trace row (inter ticket)
   unsigned cl_pay, cl_full;  // inter_cluster: this warp's mailbox / flags in the consumer CTA (shared::cluster)
 
-  __device__ __forceinline__ explicit Rep(const Ctx& ctx) : c(ctx), j(0), nerr(0), pend(0), region(0), epoch(0), mbox(nullptr), cl_pay(0), cl_full(0) {}
+  __device__ __forceinline__ explicit Rep(const Ctx& ctx)
+      : c(ctx), j(0), lstride(0), nerr(0), pend(0), region(0), epoch(0), mbox(nullptr), cl_pay(0), cl_full(0) {}
+
+  // ---- logical-CTA loop.  Kernel bodies are written
+  //        rep.init(mb);
+  //        for (; rep.active(); rep.advance()) { ... body of logical CTA rep.lblock ... }
+  //        rep.finish();
+  // none / intra: one logical CTA per physical CTA (one iteration).  inter_group
+  // and inter_cluster launch a resident set of replica pairs once, and each pair
+  // walks the logical CTAs pair, pair + P, pair + 2P, ... (persistent pairs: the
+  // ticket, region and exit bookkeeping are paid once per pair instead of once
+  // per logical CTA; both replicas walk the same sequence, so their commit
+  // sequences stay in lockstep).  advance() is CTA-uniform and ends with a
+  // barrier before the next logical CTA reuses shared memory (every body's last
+  // commit is non-deferred, so no record is pending across it).
+  __device__ __forceinline__ bool active() const { return lblock < c.nblocks; }
+  __device__ __forceinline__ void advance() {
+    if (lstride == 0) {
+      lblock = c.nblocks;
+    } else {
+      __syncthreads();
+      lblock += lstride;
+    }
+  }
 
   // Must be called by every thread of the CTA, first thing (may __syncthreads).
   // mbox_smem: MBOX_WORDS * (blockDim/32) words of shared memory (intra_smem only).
@@ -265,16 +324,31 @@ struct Rep {
       if constexpr (V == V_INTRA_SMEM) mbox = mbox_smem + warp * MBOX_WORDS;
     } else if constexpr (INTER) {
       __shared__ unsigned s_ticket;
+#ifdef RMT_TRACE
+      const unsigned long long tr0 = gtimer();
+#endif
       if (threadIdx.x == 0) s_ticket = atomicAdd(c.ctrl, 1u);  // P:679-681 global counter
       __syncthreads();
       unsigned t = s_ticket;
-      lblock = (int)(t >> 1);  // P:681 mask the low bit -> identical pair
+      tr_id = t;
+#ifdef RMT_TRACE
+      RMT_TR(0, tr0);
+      {
+        unsigned smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        RMT_TR(6, smid);
+        RMT_TR(7, t & 1u);
+      }
+#endif
+      const unsigned pair = t >> 1;  // P:681 mask the low bit -> identical pair
+      lblock = (int)pair;            // first logical CTA of the pair
+      lstride = c.lstride;
       r = (int)(t & 1u);
       consumer = (r == 1);     // even ticket = producer (reading R-RMT2)
       ltid = threadIdx.x;
       llane = lane;
-      region = (unsigned)lblock % (unsigned)c.R;
-      epoch = (unsigned)lblock / (unsigned)c.R;
+      region = pair % (unsigned)c.R;
+      epoch = pair / (unsigned)c.R;
       if constexpr (STRESS) {  // random per-CTA start skew: perturbs which role runs ahead
         if (c.stress & STRESS_SKEW) __nanosleep(mix32(t * 0x9E3779B9u + 1u) % (c.skew_ns + 1u));
       }
@@ -284,6 +358,9 @@ struct Rep {
         if (threadIdx.x == 0 && epoch != 0) spin_until(c.ctrl + CTRL_TURN + region, epoch, c);
         __syncthreads();
       }
+#ifdef RMT_TRACE
+      RMT_TR(1, gtimer());
+#endif
     } else if constexpr (CLUSTER) {
       // The pair is a 2-CTA thread-block cluster: hardware co-schedules both
       // CTAs, so no ticket or turn is needed (the B200 form of P:679's
@@ -296,6 +373,7 @@ struct Rep {
       r = (int)cluster_ctarank();
       consumer = (r == 1);
       lblock = (int)cluster_id_x();
+      lstride = c.lstride;
       ltid = threadIdx.x;
       llane = lane;
       if constexpr (STRESS) {
@@ -349,12 +427,20 @@ struct Rep {
       if (pend == 0u) return;
       const unsigned first = j - pend;
       if (!consumer) {
+#if RMT_PUB_FENCE_SC
         asm volatile("fence.sc.gpu;" ::: "memory");
+#else
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#endif
         __syncwarp();
         if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), 1u);
       } else {
         __syncwarp();
+#if RMT_FREE_RELAXED
+        if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), 0u);
+#else
         if ((unsigned)lane < pend) st_release(c.flags + slot_index(first + lane), 0u);
+#endif
       }
       pend = 0u;
     }
@@ -370,13 +456,16 @@ struct Rep {
     }
     if constexpr (INTER) {
       __shared__ unsigned s_last;
+#ifdef RMT_TRACE
+      RMT_TR(4, gtimer());
+#endif
       flush();
       __syncthreads();
       if (threadIdx.x == 0) {
         if (consumer && !NOCOMM) st_release(c.ctrl + CTRL_TURN + region, epoch + 1);
         __threadfence();
         unsigned d = atomicAdd(c.ctrl + 1, 1u);
-        s_last = (d == 2u * (unsigned)c.nblocks - 1u);
+        s_last = (d == 2u * (unsigned)c.pairs - 1u);
       }
       __syncthreads();
       if (s_last) {  // self-reset: the next launch starts from zero
@@ -395,6 +484,9 @@ struct Rep {
           c.ctrl[CTRL_DONE] = 0;
         }
       }
+#ifdef RMT_TRACE
+      RMT_TR(5, gtimer());
+#endif
     }
   }
 
@@ -635,6 +727,9 @@ struct Rep {
           for (int k = 0; k < NW; ++k) pv[k] = (!COND || ((mask >> k) & 1u)) ? ld_cl(pa + (1 + k) * 32 * 4) : 0u;
         }
       } else {  // V_INTER: per-(region, warp) queue of S records
+#ifdef RMT_TRACE
+        if (j == 0) RMT_TR(2, gtimer());
+#endif
         const size_t fi = slot_index(j);
         unsigned* fl = c.flags + fi;
         unsigned* pl = c.payload + fi * (RING_WORDS * 32);
@@ -695,6 +790,9 @@ struct Rep {
         ++j;
         ++pend;
         if (!defer) flush();  // publish (producer) / free the buffers (consumer)
+#ifdef RMT_TRACE
+        if (INTER && j == 1) RMT_TR(3, gtimer());
+#endif
       }
     }
   }

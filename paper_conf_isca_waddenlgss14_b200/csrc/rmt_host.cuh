@@ -4,6 +4,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <stdlib.h>
+
 #include <string>
 
 #include "../../include/rmt.h"
@@ -141,12 +143,70 @@ size_t pad_for_occupancy(K kn, int bn, size_t sn, int target) {
 // Standard launch of one RMT kernel instance: logical grid G of BL-thread
 // logical CTAs, `smem` dynamic shared bytes.  kr = the variant's kernel,
 // kn = the V_NONE kernel (used for the INFLATE ablation).
+// inter_group / inter_cluster launch a resident set of P replica pairs (P <=
+// the pairs that fit on the GPU at once, <= INTER_R queue regions, <= G) and
+// each pair walks the logical CTAs pair, pair + P, ... (Rep::active/advance);
+// `persistent = false` keeps one logical CTA per pair (kernels whose body is not
+// written as the logical-CTA loop).
+// Resident pairs per pair slot.  Measured on the suite (DESIGN.md section 7,
+// "Persistent pairs"): persistent DSMEM pairs help inter_cluster (transpose
+// 3.03 -> 2.68x, FWT 4.12 -> 3.94x), but persistent L2-queue pairs run in
+// lockstep with two L2 round trips per record on the consumer side and lose
+// (transpose 3.1 -> 4.4x), so inter_group keeps one logical CTA per pair.
+// Experiment knob RMT_INTER_PAIRS_MULT (k > 0: k x resident pairs for both; 0: none).
+inline int inter_pairs_mult(bool cluster) {
+  static int m = [] {
+    const char* e = getenv("RMT_INTER_PAIRS_MULT");
+    return e ? atoi(e) : -1;
+  }();
+  return m >= 0 ? m : (cluster ? 1 : 0);
+}
+
+template <int V, class Args>
+unsigned inter_pairs(void (*kr)(Args, Ctx), int block, size_t dyn_smem, unsigned G, bool cluster) {
+  if (inter_pairs_mult(cluster) <= 0) return G;
+  int occ = 0;
+  if (cluster) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = dyn_smem;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int ncl = 0;
+    if (cudaOccupancyMaxActiveClusters(&ncl, kr, &cfg) != cudaSuccess || ncl < 1) {
+      cudaGetLastError();
+      ncl = 148;
+    }
+    occ = ncl;  // resident clusters = pairs
+  } else {
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kr, block, dyn_smem) != cudaSuccess || per_sm < 1) {
+      cudaGetLastError();
+      per_sm = 2;
+    }
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    occ = per_sm * nsm / 2;
+  }
+  unsigned P = (unsigned)(occ < 1 ? 1 : occ) * (unsigned)inter_pairs_mult(cluster);
+  return P < G ? P : G;
+}
+
 template <int V, class Args>
 int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned G, int BL, size_t smem,
-               const Args& a, const char* what) {
+               const Args& a, const char* what, bool persistent = true) {
   if (G == 0) return RMT_OK;
   Ctx c = L.ctx;
   c.nblocks = (int)G;
+  c.pairs = (int)G;
+  c.lstride = 0;
   if (L.inflate) {
     // run the original kernel with the RMT version's per-SM footprint
     // (inter: the footprint of two RMT groups).
@@ -169,8 +229,12 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
       dyn = (size_t)c.R + (size_t)(BL / 32) * c.S * (RING_WORDS * 32 + 1) * 4;
     }
     cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+    if (persistent) {
+      c.pairs = (int)inter_pairs<V>(kr, Geom<V>::block(BL), dyn, G, true);
+      c.lstride = c.pairs;
+    }
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(Geom<V>::grid(G));
+    cfg.gridDim = dim3(Geom<V>::grid((unsigned)c.pairs));
     cfg.blockDim = dim3(Geom<V>::block(BL));
     cfg.dynamicSmemBytes = dyn;
     cfg.stream = L.stream;
@@ -187,10 +251,14 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
     if (e != cudaSuccess) return cuda_check(e, what);
   } else {
     if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (V == V_INTER && persistent) {
+      c.pairs = (int)inter_pairs<V>(kr, Geom<V>::block(BL), smem, G, false);
+      c.lstride = c.pairs;
+    }
     // programmatic dependent launch: the grid is scheduled while the previous
     // kernel drains; Rep::init waits (griddepcontrol.wait) before any access
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(Geom<V>::grid(G));
+    cfg.gridDim = dim3(Geom<V>::grid(V == V_INTER ? (unsigned)c.pairs : G));
     cfg.blockDim = dim3(Geom<V>::block(BL));
     cfg.dynamicSmemBytes = smem;
     cfg.stream = L.stream;
