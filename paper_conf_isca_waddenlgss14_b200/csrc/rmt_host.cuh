@@ -201,7 +201,7 @@ unsigned inter_pairs(void (*kr)(Args, Ctx), int block, size_t dyn_smem, unsigned
 
 template <int V, class Args>
 int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned G, int BL, size_t smem,
-               const Args& a, const char* what, bool persistent = true) {
+               const Args& a, const char* what, bool persistent = true, int bl_none = 0) {
   if (G == 0) return RMT_OK;
   Ctx c = L.ctx;
   c.nblocks = (int)G;
@@ -214,10 +214,10 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
     if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kr, Geom<V>::block(BL), smem);
     int target = (V == V_INTER || V == V_CLUSTER) ? (occ / 2 > 1 ? occ / 2 : 1) : (occ > 1 ? occ : 1);
-    size_t pad = pad_for_occupancy(kn, BL, smem, target);
+    size_t pad = pad_for_occupancy(kn, bl_none ? bl_none : BL, smem, target);
     if (smem + pad > 48 * 1024)
       cudaFuncSetAttribute(kn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem + pad));
-    kn<<<G, BL, smem + pad, L.stream>>>(a, c);
+    kn<<<G, bl_none ? bl_none : BL, smem + pad, L.stream>>>(a, c);
   } else if constexpr (V == V_CLUSTER) {
     // the DSMEM mailbox (rmt_device.cuh, Rep::init) follows the kernel's own
     // dynamic shared memory

@@ -458,11 +458,13 @@ class FloydWarshall(Case):
 class MatMul(Case):
     kernel = "matmul"
 
-    def __init__(self, M, N, K, seed=10, integer=False):
+    def __init__(self, M, N, K, seed=10, integer=False, kc=0):
         self.M, self.N, self.K = M, N, K
         self.n = M * N
-        self.dims = (M, N, K)
+        self.dims = (M, N, K, kc)  # kc: TMEM chunk (fold) length in K, 0 = the library default
         self.integer = integer
+        if kc:
+            self.tag = f"-kc{kc}"
         if integer:
             self.A = inputs.matmul_bf16_int(seed, M, K, stream=20)
             self.Bt = inputs.matmul_bf16_int(seed, N, K, stream=21)
@@ -610,6 +612,8 @@ def small_cases():
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),
         FloydWarshall(64, sparse=0.03), FloydWarshall(128, sparse=0.1),
         MatMul(128, 256, 64), MatMul(256, 512, 192, integer=True), MatMul(384, 256, 1024),
+        MatMul(256, 512, 3072), MatMul(128, 256, 640, kc=64), MatMul(256, 256, 1024, kc=1024),
+        MatMul(128, 512, 4096, kc=4096),
         DWT(1), DWT(2), DWT(4), DWT(8), DWT(64), DWT(4096), DWT(8192), DWT(1 << 20), DWT(1 << 23),
         BitonicSort(1), BitonicSort(2), BitonicSort(8), BitonicSort(16), BitonicSort(64, bits=3),
         BitonicSort(4096), BitonicSort(8192, bits=8), BitonicSort(1 << 17), BitonicSort(1 << 20, bits=12),

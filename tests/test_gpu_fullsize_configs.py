@@ -202,10 +202,12 @@ def test_matmul_16384_fullsize(integer):
     if integer:
         xi = rng.integers(-3, 4, N).astype(np.float64)  # exact in fp64 (|terms| < 2^53)
         assert np.array_equal(C.astype(np.float64) @ xi, Af @ (Bf.T @ xi))
-    # DESIGN.md R-MM4: the tensor pipe's fp32 accumulation drifts ~1.9e-5
-    # normwise at K = 16384 (not RN); the rigorous check is the elementwise
-    # gamma-type bound below
-    assert np.linalg.norm(lhs - rhs) <= 1e-4 * np.linalg.norm(rhs) + 1e-30
+    # R-MM2: normwise 1e-5 (BASELINE.json).  R-MM4: the tensor pipe's own fp32
+    # accumulation is not round-to-nearest (1.9e-5 at K = 16384 in one TMEM
+    # accumulator); the kernel accumulates K in chunks of 1024 and adds them RN
+    rel = np.linalg.norm(lhs - rhs) / np.linalg.norm(rhs)
+    print(f"matmul 16384^3 normwise error (Freivalds projection): {rel:.3e}")
+    assert rel <= 1e-5
     rows = rng.integers(0, M, 4096)
     cols = rng.integers(0, N, 4096)
     want, absw = oracle.matmul_bf16_sampled(A.reshape(M, K), Bt.reshape(N, K), rows, cols)
