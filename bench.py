@@ -323,37 +323,50 @@ def main():
         else:
             dist.init_process_group(args.dist_backend)
     variants = [v for v in args.variants.split(",") if v]
-    jobs = workloads.config_jobs(args.config, rank)
+    jobs = workloads.config_jobs(args.config, rank, world)
+    scaling = "strong" if args.config in workloads.STRONG_CONFIGS else "weak"
     stream = torch.cuda.current_stream()
     err = torch.zeros(1, dtype=torch.int64, device="cuda")
     ws = {}
-    ws_red = {}
+    ws_aux = {}
     for j in jobs:
         j.device_buffers()
         for v in variants:
             ws[(j.kernel, v)] = rmt.make_workspace(j.kernel, v, j.n, j.dims)
-            if j.kernel == "prefixsum":
-                ws_red[v] = rmt.make_workspace("reduction", v, j.n)
+            if world > 1 and j.kernel == "prefixsum":
+                ws_aux[(j.kernel, v)] = rmt.make_workspace("reduction", v, j.n)
+            if world > 1 and j.kernel == "fwt":
+                ws_aux[(j.kernel, v)] = rmt.make_workspace("fwt", v, j.n, (1, 0))
     torch.cuda.synchronize()
 
     launches = [(j, v) for j in jobs for v in variants]
     ev = {(j.kernel, v): [] for j, v in launches}
     counts = {"gpu_launches": 0}
+    # multi-GPU exchange buffers: PrefixSum totals, FWT partner shard
     s_tmp = torch.zeros(2, dtype=torch.int32, device="cuda")
+    totals = torch.zeros(world, dtype=torch.int64, device="cuda")
+    fwt_n = max([j.n for j in jobs if j.kernel == "fwt"] or [0])
+    fwt_recv = torch.empty(fwt_n if world > 1 else 0, dtype=torch.float32, device="cuda")
+    fwt_tmp = torch.empty_like(fwt_recv)
 
     def one(j, v):
         """One launch of job j under variant v; for N > 1 the kernels that need a
-        cross-shard exchange do it here."""
+        cross-shard exchange do it here (parallel.py)."""
         if world > 1 and j.kernel == "prefixsum":
-            # local total (Reduction kernel) -> all-gather -> carry-in -> scan
-            parallel.global_prefixsum(j.dev[0], j.dev[1], s_tmp, err, rmt, variant=v,
-                                      ws_red=ws_red[v], ws_ps=ws[(j.kernel, v)])
-            return 2
-        nk = rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=ws[(j.kernel, v)],
-                        stream=stream.cuda_stream)
+            # local total (Reduction kernel) -> device all-gather -> device carry -> scan
+            return parallel.global_prefixsum(j.dev[0], j.dev[1], s_tmp, totals, err, rmt, variant=v,
+                                             ws_red=ws_aux[(j.kernel, v)], ws_ps=ws[(j.kernel, v)]) + 1
+        if world > 1 and j.kernel == "fwt":
+            # local transform + log2 G cross-shard butterfly stages (send/recv + combine kernel)
+            return parallel.global_fwt(j.dev[0], j.dev[1].view(torch.float32), fwt_recv, fwt_tmp, err, rmt,
+                                       variant=v, workspace=ws[(j.kernel, v)], ws_comb=ws_aux[(j.kernel, v)])
         if world > 1 and j.kernel == "reduction":
+            rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=ws[(j.kernel, v)],
+                       stream=stream.cuda_stream)
             parallel.allreduce_sum_(j.dev[1].view(torch.int64))
-        return nk
+            return rmt.last_launch_count()
+        return rmt.launch(j.kernel, v, j.dev, j.n, err, dims=j.dims, workspace=ws[(j.kernel, v)],
+                          stream=stream.cuda_stream)
 
     def step(timed):
         for j, v in launches:
@@ -420,7 +433,7 @@ def main():
     rest = {}
     if not args.no_rest10 and args.config == "suite" and "none" in variants:
         err_r = torch.zeros(1, dtype=torch.int64, device="cuda")
-        for j in workloads.config_jobs("rest10", rank):
+        for j in workloads.config_jobs("rest10", rank, world):
             j.device_buffers()
             d = {"bound": j.bound}
             for v in variants:
@@ -646,11 +659,11 @@ def main():
         line = {
             "metric": METRIC, "value": round(value, 1) if value else None, "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_total / args.steps, 3),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32/u8x4",
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u32/f32/u8x4",
             "data": "synthetic",
             "config": {"workload": workloads.CONFIG_TITLES[args.config], "preset": args.config,
                        "variants": variants, "l2": "every input > 126 MB L2 (no flush needed)",
-                       "parallelism": f"dp{world} (data-sharded, weak)",
+                       "parallelism": f"dp{world} (data-sharded, {scaling})",
                        "value": "baseline (none) HBM GB/s: sum of algorithmic bytes / sum of none launch times"},
             "step_gbs_all_variants": round(step_bytes * args.steps * world / (ms_total * 1e-3) / 1e9, 1),
             "slowdown_geomean": slowdown_geomean, "baseline_frac": baseline_frac,

@@ -117,9 +117,14 @@ typedef struct {
  *                 mode 0: one draw r per option, (S,K,T,R,sigma) from r with S == K (DESIGN.md R-BS1)
  *                 mode 1: buf[0] = params:F32[5n], planes S | K | T | R | sigma, n%4 = 0 (R-BS4)
  *   BINARYSEARCH  buf {A:U32[N] sorted, q:U32[Q], idx:U32[Q]}       n = Q, dims {N, Q}
- *   FWT           buf {x:F32[N], y:F32[N]}                          n = N = 2^m
+ *   FWT           buf {x:F32[N], y:F32[N]}                          n = N = 2^m, dims {0}
+ *                 dims {1, upper}: one cross-shard butterfly stage of a multi-GPU FWT,
+ *                 buf {x: this shard, y: out, p: the partner shard} F32[N]; y = x + p (lower
+ *                 rank of the pair) or p - x (upper) -- the single-GPU stage's fp32 operations
  *   PREFIXSUM     buf {x:U32[n], y:U32[n]}  inclusive, mod 2^32     n, dims {carry_in} (u32 added
- *                 to every y: the exclusive prefix of earlier shards in a multi-GPU scan; 0 = none)
+ *                 to every y: the exclusive prefix of earlier shards in a multi-GPU scan; 0 = none);
+ *                 optional buf[2] totals:U64[G] (every rank's total, all-gathered on the device)
+ *                 with dims {carry_in, rank}: totals[0 .. rank) are added too (no host round trip)
  *   REDUCTION     buf {x:U32[n], s:U64[1]}                          n
  *   TRANSPOSE     buf {A:U32|F32[H*W], B:same[W*H]}                 n = H*W, dims {H, W}, H%4 = W%4 = 0
  *   SOBEL         buf {I:U8X4[H*W], O:U8X4[H*W]}                    n = H*W, dims {H, W}, W%4 = 0

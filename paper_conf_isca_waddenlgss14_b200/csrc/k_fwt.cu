@@ -490,6 +490,63 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_ps_kernel(FwtArgs a, C
   rep.finish();
 }
 
+// Cross-shard butterfly stage of a multi-GPU FWT (local FWHT of
+// N/G, then log2 G stages whose pairs (i, i + h) sit on two GPUs): this rank
+// holds x = its shard, p = the partner shard; the lower rank of the pair keeps
+// a + b = x + p, the upper keeps a - b = p - x, the same fp32 operations (and
+// operand order) as the single-GPU stage h, so the sharded result is bitwise the
+// single-GPU one.  Logical thread = 4 consecutive elements, one vector commit.
+struct FwtCombArgs {
+  const float* x;
+  const float* p;
+  float* y;
+  unsigned n;
+  unsigned upper;
+};
+
+constexpr int BLC = 256;
+
+template <int V, int M>
+__global__ void __launch_bounds__(BLC * Geom<V>::DUP) fwt_combine_kernel(FwtCombArgs a, Ctx c) {
+  __shared__ unsigned mb[mbox_words<V>(BLC * Geom<V>::DUP)];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  for (; rep.active(); rep.advance()) {
+    const unsigned i0 = ((unsigned)rep.lblock * BLC + (unsigned)rep.ltid) * 4u;
+    unsigned w[4];
+    unsigned mask = 0;
+    if (i0 + 4 <= a.n) {  // input replication: each replica loads both operands itself
+      const float4 xv = __ldcs(reinterpret_cast<const float4*>(a.x + i0));
+      const float4 pv = __ldcs(reinterpret_cast<const float4*>(a.p + i0));
+      const float xs[4] = {xv.x, xv.y, xv.z, xv.w}, ps[4] = {pv.x, pv.y, pv.z, pv.w};
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const float xk = rep.faultf(SITE_LOAD, (long long)i0 + k, xs[k]);
+        w[k] = __float_as_uint(a.upper ? __fsub_rn(ps[k], xk) : __fadd_rn(xk, ps[k]));
+      }
+      mask = 0xFu;
+    } else {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const bool in = i0 + k < a.n;
+        const float xk = rep.faultf(SITE_LOAD, (long long)i0 + k, in ? a.x[i0 + k] : 0.0f);
+        const float pk = in ? a.p[i0 + k] : 0.0f;
+        w[k] = __float_as_uint(a.upper ? __fsub_rn(pk, xk) : __fadd_rn(xk, pk));
+        mask |= (in ? 1u : 0u) << k;
+      }
+    }
+    rep.template commit<4, 0>(mask, i0, w, a.n, [&](unsigned idx, unsigned m, const unsigned* v) {
+      if (m == 0xFu)
+        __stcs(reinterpret_cast<float4*>(a.y + idx),
+               make_float4(__uint_as_float(v[0]), __uint_as_float(v[1]), __uint_as_float(v[2]), __uint_as_float(v[3])));
+      else
+        for (int k = 0; k < 4; ++k)
+          if ((m >> k) & 1u) a.y[idx + k] = __uint_as_float(v[k]);
+    });
+  }
+  rep.finish();
+}
+
 int log2u(int64_t n) {
   int m = 0;
   while ((1LL << m) < n) ++m;
@@ -499,9 +556,12 @@ int log2u(int64_t n) {
 }  // namespace
 
 int fwt_validate(const rmt_bufs_t* b, int64_t n) {
+  const int64_t mode = b->dims[0];
   if (b->nbuf < 2 || n < 1 || n > (1LL << 30) || (n & (n - 1)) || !buf_ok(b->buf[0], RMT_F32, n) ||
-      !buf_ok(b->buf[1], RMT_F32, n)) {
-    set_error("fwt: expected {x,y} F32[N], N a power of two in [1, 2^30]");
+      !buf_ok(b->buf[1], RMT_F32, n) || (mode != 0 && mode != 1) ||
+      (mode == 1 && (b->nbuf < 3 || !buf_ok(b->buf[2], RMT_F32, n) || (b->dims[1] != 0 && b->dims[1] != 1)))) {
+    set_error("fwt: expected {x,y} F32[N], N a power of two in [1, 2^30] (dims[0] = 0); or the cross-shard stage "
+              "{x, y, p} F32[N] with dims {1, upper}");
     return RMT_EINVAL;
   }
   return RMT_OK;
@@ -510,6 +570,16 @@ size_t fwt_scratch(int64_t, const int64_t*) { return 0; }
 int fwt_inter_warps(int64_t, const int64_t*) { return BL / 32; }
 
 int fwt_run(Launch& L) {
+  if (L.bufs->dims[0] == 1) {  // cross-shard butterfly stage (multi-GPU)
+    FwtCombArgs a{(const float*)L.bufs->buf[0].ptr, (const float*)L.bufs->buf[2].ptr, (float*)L.bufs->buf[1].ptr,
+                  (unsigned)L.n, (unsigned)L.bufs->dims[1]};
+    const unsigned G = (unsigned)((L.n + 4 * BLC - 1) / (4 * BLC));
+    return dispatch(L.variant, L.mode, [&](auto vm) {
+      constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+      return launch_std<V>(L, fwt_combine_kernel<V, M>, fwt_combine_kernel<V_NONE, M_NORMAL>, G, BLC, 0, a,
+                           "fwt/combine");
+    });
+  }
   const int m = log2u(L.n);
   const int tb = m < TB_MAX ? m : TB_MAX;
   const float* x = (const float*)L.bufs->buf[0].ptr;

@@ -33,6 +33,8 @@ struct PsArgs {
   unsigned nch;        // chunks actually used
   unsigned carry_in;   // added to every output (multi-GPU shard offset)
   unsigned v8;         // x is 32-B aligned: 256-bit loads where a thread's run allows
+  const unsigned long long* totals;  // multi-GPU: every rank's total (all-gathered on the device), or null
+  unsigned rank;       // totals[0 .. rank) are added to the carry (mod 2^32)
 };
 
 // u32 sum over the logical CTA (logical warps + duplicated smem)
@@ -130,6 +132,8 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_k
     // carry-in: sum of the partials of all earlier chunks (L2-resident)
     unsigned cs = 0;
     for (unsigned i = rep.ltid; i < ch; i += BL) cs += __ldcg(a.partial + i);
+    if (a.totals)  // exclusive prefix of the lower ranks' totals: no host round trip
+      for (unsigned i = rep.ltid; i < a.rank; i += BL) cs += (unsigned)__ldcg(a.totals + i);
     unsigned carry = a.carry_in + block_sum_u32(rep, cs, sw);
     const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
     const int lw = rep.ltid / LW;
@@ -262,8 +266,12 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_k
 }  // namespace
 
 int prefixsum_validate(const rmt_bufs_t* b, int64_t n) {
-  if (b->nbuf < 2 || n < 0 || n >= (1LL << 30) || !buf_ok(b->buf[0], RMT_U32, n) || !buf_ok(b->buf[1], RMT_U32, n)) {
-    set_error("prefixsum: expected {x,y} U32[n], n < 2^30");
+  const bool tot = b->nbuf >= 3 && b->buf[2].ptr != nullptr;
+  if (b->nbuf < 2 || n < 0 || n >= (1LL << 30) || !buf_ok(b->buf[0], RMT_U32, n) || !buf_ok(b->buf[1], RMT_U32, n) ||
+      (tot && (b->buf[2].dtype != RMT_U64 || ((uintptr_t)b->buf[2].ptr % 16) != 0 || b->dims[1] < 0 ||
+               b->dims[1] > b->buf[2].numel))) {
+    set_error("prefixsum: expected {x,y} U32[n], n < 2^30, dims {carry_in}; optionally totals:U64[G] with dims "
+              "{carry_in, rank}");
     return RMT_EINVAL;
   }
   return RMT_OK;
@@ -279,7 +287,8 @@ int prefixsum_run(Launch& L) {
   const unsigned chunk = tiles_per_chunk * TILE;
   const unsigned nch = (n + chunk - 1) / chunk;
   PsArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, (unsigned*)L.scratch, n, chunk, nch,
-           (unsigned)(L.bufs->dims[0] & 0xFFFFFFFFu), ((uintptr_t)L.bufs->buf[0].ptr % 32) == 0 ? 1u : 0u};
+           (unsigned)(L.bufs->dims[0] & 0xFFFFFFFFu), ((uintptr_t)L.bufs->buf[0].ptr % 32) == 0 ? 1u : 0u,
+           L.bufs->nbuf >= 3 ? (const unsigned long long*)L.bufs->buf[2].ptr : nullptr, (unsigned)L.bufs->dims[1]};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     int rc = launch_std<V>(L, ps_reduce_kernel<V, M>, ps_reduce_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a,

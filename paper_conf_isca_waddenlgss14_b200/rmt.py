@@ -44,6 +44,9 @@ SCHEMA = {
     "bitonicsort": (U32, U32),
     "binomialoption": (F32, F32),
 }
+# optional trailing buffers: the FWT cross-shard stage's partner shard, the
+# PrefixSum all-gathered rank totals (include/rmt.h)
+SCHEMA_EXTRA = {"fwt": (F32,), "prefixsum": (U64,)}
 
 
 class RmtError(RuntimeError):
@@ -129,7 +132,9 @@ def _ptr(t):
 def make_bufs(kernel: str, tensors, dims=()) -> _Bufs:
     schema = SCHEMA[kernel]
     if len(tensors) != len(schema):
-        raise RmtError(f"{kernel}: expected {len(schema)} buffers, got {len(tensors)}")
+        schema = schema + SCHEMA_EXTRA.get(kernel, ())
+        if len(tensors) != len(schema):
+            raise RmtError(f"{kernel}: expected {len(SCHEMA[kernel])} buffers, got {len(tensors)}")
     b = _Bufs()
     b.nbuf = len(tensors)
     for i, (t, dt) in enumerate(zip(tensors, schema)):

@@ -127,29 +127,37 @@ def job_transpose(H, W, seed=3, rank=0):
                alg_bytes=8 * H * W, unit="elements")
 
 
-def job_sobel(H, W, seed=7, rank=0):
-    I = inputs.sobel_image(seed, H, W, rank * H).view(np.uint32).reshape(-1)
-    return Job("sobel", H * W, (H, W), [I, None], [(1, 4 * H * W)], alg_bytes=8 * H * W, unit="pixels")
+def job_sobel(H, W, seed=7, rank=0, world=1):
+    """Rank `rank` of `world` owns rows [rank H, (rank + 1) H) of a (world H)-row
+    image; with world > 1 its input carries one halo row above / below
+    (parallel.sobel_halo_rows), whose output rows are not part of the result."""
+    r0 = rank * H
+    lo, hi = (r0, r0 + H) if world == 1 else (max(0, r0 - 1), min(world * H, r0 + H + 1))
+    I = inputs.sobel_image(seed, hi - lo, W, lo).view(np.uint32).reshape(-1)
+    return Job("sobel", (hi - lo) * W, (hi - lo, W), [I, None], [(1, 4 * (hi - lo) * W)], alg_bytes=8 * H * W,
+               unit="pixels", note="" if world == 1 else f"rows [{r0}, {r0 + H}) + halo rows [{lo}, {hi})")
 
 
-def job_blackscholes(n, seed=1, rank=0, device_gen=False):
+def job_blackscholes(n, seed=1, rank=0, device_gen=False, offset=None):
+    off = rank * n if offset is None else offset
     if device_gen:  # 2^30 options: generated in HBM (inputs.blackscholes_r_t, the same bits)
         return Job("blackscholes", n, (0,), [None, None, None], [(1, 4 * n), (2, 4 * n)], alg_bytes=12 * n,
                    unit="options", bound="mufu",
-                   dev_gen=lambda i: inputs.blackscholes_r_t(seed, n, rank * n))
-    return Job("blackscholes", n, (0,), [inputs.blackscholes_r(seed, n, rank * n), None, None],
+                   dev_gen=lambda i: inputs.blackscholes_r_t(seed, n, off))
+    return Job("blackscholes", n, (0,), [inputs.blackscholes_r(seed, n, off), None, None],
                [(1, 4 * n), (2, 4 * n)], alg_bytes=12 * n, unit="options", bound="mufu")
 
 
-def job_matmul(M, N, K, seed=10, rank=0, device_gen=False):
+def job_matmul(M, N, K, seed=10, rank=0, device_gen=False, row_offset=None):
     note = f"{2 * M * N * K:.3e} flop"
+    ro = rank * M if row_offset is None else row_offset
     if device_gen:
-        gen = {0: lambda: inputs.matmul_bf16_normal_t(seed, M, K, stream=22, row_offset=rank * M),
+        gen = {0: lambda: inputs.matmul_bf16_normal_t(seed, M, K, stream=22, row_offset=ro),
                1: lambda: inputs.matmul_bf16_normal_t(seed, N, K, stream=24)}
         return Job("matmul", M * N, (M, N, K), [None, None, None], [(2, 4 * M * N)],
                    alg_bytes=2 * (M * K + N * K) + 4 * M * N, unit="C elements", bound="tensor", note=note,
                    dev_gen=lambda i: gen[i]())
-    A = inputs.matmul_bf16_normal(seed, M, K, stream=22, row_offset=rank * M)
+    A = inputs.matmul_bf16_normal(seed, M, K, stream=22, row_offset=ro)
     Bt = inputs.matmul_bf16_normal(seed, N, K, stream=24)
     return Job("matmul", M * N, (M, N, K), [A, Bt, None], [(2, 4 * M * N)],
                alg_bytes=2 * (M * K + N * K) + 4 * M * N, unit="C elements", bound="tensor", note=note)
@@ -191,28 +199,47 @@ def job_binomialoption(n, seed=12, rank=0):
 
 # ---------------------------------------------------------------- BASELINE.json configs
 
-def config_jobs(name: str, rank: int = 0):
+STRONG_CONFIGS = ("bs30", "mm16k")  # BASELINE.json configs[4]: a fixed global problem split over the GPUs
+
+
+def _bs_strong(n_total, rank, world):
+    off, cnt = strong_range(n_total, world, rank, 4)
+    return job_blackscholes(cnt, rank=rank, device_gen=True, offset=off)
+
+
+def _mm_strong(M, N, K, rank, world):
+    off, cnt = strong_range(M, world, rank, 128)
+    return job_matmul(cnt, N, K, rank=rank, device_gen=True, row_offset=off)
+
+
+def strong_range(n_total: int, world: int, rank: int, align: int = 1):
+    units = n_total // align
+    lo, hi = units * rank // world, units * (rank + 1) // world
+    return lo * align, (hi - lo) * align
+
+
+def config_jobs(name: str, rank: int = 0, world: int = 1):
     if ":" in name:          # "<config>:<kernel>[,<kernel>]" -- a subset of a config (quick timing)
         base, ks = name.split(":", 1)
         keep = set(ks.split(","))
-        return [j for j in config_jobs(base, rank) if j.kernel in keep]
-    if name == "suite":      # configs[1]: the APP SDK-style suite, "paper's sizes"
+        return [j for j in config_jobs(base, rank, world) if j.kernel in keep]
+    if name == "suite":      # configs[1]: the APP SDK-style suite, "paper's sizes"; weak scaling
         return [job_binarysearch(1 << 26, 1 << 24, rank=rank), job_fwt(1 << 26, rank=rank),
                 job_prefixsum(1 << 26, rank=rank), job_reduction(1 << 26, rank=rank),
-                job_transpose(8192, 8192, rank=rank), job_sobel(8192, 8192, rank=rank)]
+                job_transpose(8192, 8192, rank=rank), job_sobel(8192, 8192, rank=rank, world=world)]
     if name == "suite28":    # configs[2]: 2^28 elements
         return [job_binarysearch(1 << 28, 1 << 26, rank=rank), job_fwt(1 << 28, rank=rank),
                 job_prefixsum(1 << 28, rank=rank), job_reduction(1 << 28, rank=rank),
-                job_transpose(16384, 16384, rank=rank), job_sobel(16384, 16384, rank=rank)]
+                job_transpose(16384, 16384, rank=rank), job_sobel(16384, 16384, rank=rank, world=world)]
     if name == "bs16":       # configs[0]
         return [job_blackscholes(1 << 16, rank=rank)]
-    if name == "bs30":       # configs[4] (BlackScholes part)
-        return [job_blackscholes(1 << 30, rank=rank, device_gen=True)]
-    if name == "mm16k":      # configs[4] (MatrixMultiplication part)
-        return [job_matmul(16384, 16384, 16384, rank=rank, device_gen=True)]
+    if name == "bs30":       # configs[4] (BlackScholes part): 2^30 options split over the GPUs (strong)
+        return [_bs_strong(1 << 30, rank, world)]
+    if name == "mm16k":      # configs[4] (MatrixMultiplication part): rows of 16384^3 split (strong)
+        return [_mm_strong(16384, 16384, 16384, rank, world)]
     if name == "rest10":     # the four BASELINE.json kernels outside configs[1] (bench.py's all-10 geomean)
-        return [job_blackscholes(1 << 30, rank=rank, device_gen=True), job_floydwarshall(4096),
-                job_dct(8192, 8192, rank=rank), job_matmul(16384, 16384, 16384, rank=rank, device_gen=True)]
+        return [_bs_strong(1 << 30, rank, world), job_floydwarshall(4096),
+                job_dct(8192, 8192, rank=rank), _mm_strong(16384, 16384, 16384, rank, world)]
     if name == "mm8k":
         return [job_matmul(8192, 8192, 8192, rank=rank)]
     if name == "fwdct":      # configs[3]
