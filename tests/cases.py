@@ -53,6 +53,13 @@ class Case:
         """True if a suppressed store feeds later computation (multi-pass, in place)."""
         return False
 
+    def flipped_oracle(self, elem, bit):
+        """Outputs the oracle predicts when input word `elem` (the kernel's LOAD
+        fault site) has bit `bit` flipped -- an independent liveness prediction
+        (SURVEY 8(c) C-FI); None where the site is not an input word or the
+        oracle is not exact."""
+        return None
+
     def commit_group(self, e):
         """Word indices of the first output buffer stored by the same commit as
         word e (one commit per store instruction; vector stores are 4 words)."""
@@ -69,6 +76,14 @@ def _nan_aware_equal(got_bits, ref_bits):
     r = ref_bits.view(np.float32)
     gn, rn = np.isnan(g), np.isnan(r)
     return np.array_equal(gn, rn) and np.array_equal(got_bits[~gn], ref_bits[~rn])
+
+
+def _flip(a, elem, bit):
+    """Copy of array a with bit `bit` of 32-bit word `elem` flipped."""
+    b = np.array(a, copy=True)
+    w = b.reshape(-1).view(np.uint32)
+    w[elem] ^= np.uint32(1 << bit)
+    return b
 
 
 class BlackScholes(Case):
@@ -167,6 +182,9 @@ class Reduction(Case):
         x = self.x if x is None else x
         assert int(outs[0][0]) == oracle.reduction_u32(x)
 
+    def flipped_oracle(self, elem, bit):
+        return [np.array([oracle.reduction_u32(_flip(self.x, elem, bit))], np.uint64)]
+
     def out_elems(self):
         return 1, 1
 
@@ -197,6 +215,9 @@ class Transpose(Case):
         A = self.A if A is None else A
         assert np.array_equal(outs[0], oracle.transpose_u32(A))
 
+    def flipped_oracle(self, elem, bit):
+        return [oracle.transpose_u32(_flip(self.A, elem, bit))]
+
     def out_elems(self):
         return 1, self.n
 
@@ -221,6 +242,9 @@ class PrefixSum(Case):
     def check(self, outs, x=None):
         x = self.x if x is None else x
         assert np.array_equal(outs[0], oracle.prefixsum_u32(x))
+
+    def flipped_oracle(self, elem, bit):
+        return [oracle.prefixsum_u32(_flip(self.x, elem, bit))]
 
     def out_elems(self):
         return 1, self.n
@@ -265,6 +289,9 @@ class FWT(Case):
 
     def out_elems(self):
         return 1, self.n
+
+    def flipped_oracle(self, elem, bit):  # R-FWT2: the fp32 DAG is exact
+        return [oracle.fwt_f32dag(_flip(self.x, elem, bit)).view(np.uint32)]
 
     def commit_group(self, e):
         # the final pass's 4-word commit holding word e (k_fwt.cu): the pass-1
@@ -320,6 +347,9 @@ class BinarySearch(Case):
         q = self.q if q is None else q
         assert np.array_equal(outs[0], oracle.binarysearch(A, q))
 
+    def flipped_oracle(self, elem, bit):  # LOAD = the query word
+        return [oracle.binarysearch(self.A, _flip(self.q, elem, bit))]
+
     def out_elems(self):
         return 2, self.Q
 
@@ -350,6 +380,9 @@ class Sobel(Case):
         I = self.I if I is None else I
         ref = oracle.sobel(I).view(np.uint32).reshape(-1)
         assert np.array_equal(outs[0], ref), f"{np.sum(outs[0] != ref)} pixels differ"
+
+    def flipped_oracle(self, elem, bit):  # LOAD = the 4-channel pixel word
+        return [oracle.sobel(_flip(self.I, elem, bit)).view(np.uint32).reshape(-1)]
 
     def out_elems(self):
         return 1, self.n
@@ -533,6 +566,9 @@ class DWT(Case):
     def out_elems(self):
         return 1, self.n
 
+    def flipped_oracle(self, elem, bit):  # R-DWT2: the fp32 DAG is exact
+        return [oracle.dwthaar1d_f32dag(_flip(self.x, elem, bit)).view(np.uint32)]
+
 
 class BitonicSort(Case):
     kernel = "bitonicsort"
@@ -555,6 +591,9 @@ class BitonicSort(Case):
     def check(self, outs, keys=None):
         keys = self.keys if keys is None else keys
         assert np.array_equal(outs[0], oracle.sort_u32(keys))  # R-BIT1: the unique sorted sequence
+
+    def flipped_oracle(self, elem, bit):
+        return [oracle.sort_u32(_flip(self.keys, elem, bit))]
 
     def out_elems(self):
         return 1, self.n

@@ -28,9 +28,13 @@ CAMPAIGN = [
                                            "store_val": lambda c: c.Q, "store_addr": lambda c: c.Q}),
     (lambda: FWT(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n, "smem": lambda c: c.n,
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
+    # PrefixSum SMEM = warp total i of chunk ch (element ch*256 + i): the unprotected
+    # scan reads 32 (sub-tile, warp) totals per chunk, the intra variants 16 (warp)
+    # totals, so i < 16 is a site every variant has
     (lambda: PrefixSum(4096 * 9 + 5), {"load": lambda c: c.n, "compute": lambda c: 256 * 10,
-                                       "smem": lambda c: 256 * 10, "store_val": lambda c: c.n,
-                                       "store_addr": lambda c: c.n}),
+                                       "smem": lambda c: (lambda rng: 256 * int(rng.integers(0, 10)) +
+                                                          int(rng.integers(0, 16))),
+                                       "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
     (lambda: Reduction(300007), {"load": lambda c: c.n, "compute": lambda c: 1184 * 256,
                                  "smem": lambda c: 1184 * 8, "store_val": lambda c: 1, "store_addr": lambda c: 1}),
     (lambda: Transpose(96, 160), {"load": lambda c: c.n, "smem": lambda c: c.n, "store_val": lambda c: c.n,
@@ -53,7 +57,7 @@ CAMPAIGN = [
     (lambda: DWT(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n // 2, "smem": lambda c: c.n // 2,
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
 ]
-SAMPLES = 6
+SAMPLES = 24  # live faults per (kernel, site)
 
 
 def _silent_by_design(kernel, variant, site):
@@ -88,15 +92,25 @@ def test_fault_campaign(idx):
     rng = np.random.default_rng(1000 + idx)
     report = {}
     for site, bound in sites.items():
-        live = detected = 0
+        live = detected = predicted = 0
         for _ in range(SAMPLES * (40 if case.kernel == "floydwarshall" else 4)):
             if live >= SAMPLES:
                 break
-            elem = int(rng.integers(0, bound(case)))
+            b = bound(case)
+            elem = int(b(rng)) if callable(b) else int(rng.integers(0, b))
             bit = int(rng.integers(0, 32))
             if site == "store_addr":
                 pass  # any of the 32 index bits: out-of-range or misaligned flips are dropped by none (liveness)
             _, o0 = _with_fault(case, "none", 0, site, bit, elem)
+            pred = case.flipped_oracle(elem, bit) if site == "load" else None
+            if pred is not None:
+                # LOAD liveness predicted by the oracle on the flipped input word
+                # (independent of the kernel): the unprotected kernel's faulted
+                # output must be exactly that
+                for a, b in zip(o0, pred):
+                    assert np.array_equal(np.asarray(a).reshape(-1), np.asarray(b).reshape(-1)), \
+                        f"{case.kernel}: none with a flipped input word != oracle on the flipped input"
+                predicted += 1
             if all(np.array_equal(a, b) for a, b in zip(o0, ref)):
                 continue  # masked by the computation: not an SDC, nothing to detect
             live += 1
@@ -116,6 +130,6 @@ def test_fault_campaign(idx):
                     elif site.startswith("store") and case.kernel not in ("floydwarshall",):
                         assert err == 1, f"{case.kernel}/{variant}: {site} flip must corrupt exactly one commit"
                     detected += 1
-        report[site] = (live, detected)
+        report[site] = (live, detected, predicted)
         assert live > 0, f"{case.kernel}/{site}: no live fault found (vacuous)"
     print(case.kernel, report)
