@@ -175,6 +175,13 @@ __device__ __forceinline__ void cluster_sync_all() {
 #ifndef RMT_FREE_RELAXED
 #define RMT_FREE_RELAXED 0
 #endif
+// Inter queue group flags: a producer publishing
+// a group of g records behind one fence stores g, g-1, ..., 1 into their slot
+// flags, so a consumer that acquires the flag of the group's first record knows
+// the rest are visible too and reads their payloads without a flag round trip.
+#ifndef RMT_GROUP_FLAGS
+#define RMT_GROUP_FLAGS 1
+#endif
 #ifndef RMT_SPIN_NS0
 #define RMT_SPIN_NS0 32     // first back-off sleep of a queue wait (0: pure spin)
 #endif
@@ -199,6 +206,27 @@ __device__ __forceinline__ bool spin_until(const unsigned* p, unsigned want, con
         atomicExch(c.ctrl + CTRL_WATCHDOG, 1u);
       }
       return false;
+    }
+  }
+}
+
+// Spin until *p != 0 (acquire); returns the value seen, 0 after a watchdog timeout.
+__device__ __forceinline__ unsigned spin_nonzero(const unsigned* p, const Ctx& c, bool count) {
+  unsigned v = ld_acquire(p);
+  if (v != 0u) return v;
+  unsigned long long t0 = clock64();
+  unsigned ns = RMT_SPIN_NS0;
+  while (true) {
+    if (ns) __nanosleep(ns);
+    v = ld_acquire(p);
+    if (v != 0u) return v;
+    if (ns && ns < RMT_SPIN_NSMAX) ns <<= 1;
+    if (clock64() - t0 > c.wd) {
+      if (count) {
+        atomicAdd(c.err, 1ull);
+        atomicExch(c.ctrl + CTRL_WATCHDOG, 1u);
+      }
+      return 0u;
     }
   }
 }
@@ -274,12 +302,14 @@ struct Rep {
   unsigned nerr;  // intra: mismatching commits of this (consumer) lane, added to *err at finish()
   unsigned pend;  // inter: records not yet published (producer) / freed (consumer)
   unsigned region, epoch;
+  unsigned rdy_hi;  // inter consumer: records below this are known to be published (group flags)
   unsigned* mbox;  // intra_smem: this warp's mailbox
   unsigned tr_id;  // RMT_TRACE: trace row (inter ticket)
   unsigned cl_pay, cl_full;  // inter_cluster: this warp's mailbox / flags in the consumer CTA (shared::cluster)
 
   __device__ __forceinline__ explicit Rep(const Ctx& ctx)
-      : c(ctx), j(0), lstride(0), nerr(0), pend(0), region(0), epoch(0), mbox(nullptr), cl_pay(0), cl_full(0) {}
+      : c(ctx), j(0), lstride(0), nerr(0), pend(0), region(0), epoch(0), rdy_hi(0), mbox(nullptr), cl_pay(0),
+        cl_full(0) {}
 
   // ---- logical-CTA loop.  Kernel bodies are written
   //        rep.init(mb);
@@ -420,6 +450,7 @@ struct Rep {
       } else {
         __syncwarp();
         if ((unsigned)lane < pend) st_release_cl(cl_full + ((first + lane) & (unsigned)(c.S - 1)) * 4u, 0u);
+        __syncwarp();  // every lane's later poll of a freed slot sees the free (lane l freed slot l)
       }
       pend = 0u;
     }
@@ -433,7 +464,8 @@ struct Rep {
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
 #endif
         __syncwarp();
-        if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), 1u);
+        // group flags: record first + l gets pend - l (its distance to the group's end)
+        if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), RMT_GROUP_FLAGS ? pend - lane : 1u);
       } else {
         __syncwarp();
 #if RMT_FREE_RELAXED
@@ -441,6 +473,11 @@ struct Rep {
 #else
         if ((unsigned)lane < pend) st_release(c.flags + slot_index(first + lane), 0u);
 #endif
+        // Lane l freed the slot of record first + l; the barrier orders those
+        // stores before every lane's later poll of the same slots (a lane that
+        // polled a slot another lane had just freed could read the old record's
+        // flag and consume its stale payload)
+        __syncwarp();
       }
       pend = 0u;
     }
@@ -738,8 +775,20 @@ struct Rep {
           // free.  Publish our own pending records first, or our consumer could be
           // waiting for them while we wait for it.
           if (j >= (unsigned)c.S) {
+#if RMT_GROUP_FLAGS
+            // publish the pending group only if we must block on this slot, so
+            // that groups stay whole while the consumer keeps up.  The slot is
+            // ours only if record j - S was published and consumed: a flag of 0
+            // also marks our own unpublished records, so with S of them pending
+            // we must publish (and wait) before overwriting the oldest.
+            if (pend >= (unsigned)c.S || ld_acquire(fl) != 0u) {
+              flush();
+              spin_until(fl, 0u, c, lane == 0);
+            }
+#else
             flush();
             spin_until(fl, 0u, c, lane == 0);
+#endif
           }
           pl[lane] = key;
 #pragma unroll
@@ -750,7 +799,16 @@ struct Rep {
           // release by one lane does not order the other lanes' in-flight stores).
         } else {
           if (pend >= (unsigned)c.S) flush();  // as above: never wait on a slot we still hold
+#if RMT_GROUP_FLAGS
+          bool ok = true;
+          if (j >= rdy_hi) {  // each lane acquires the "ready" signal of the group's first record
+            const unsigned g = spin_nonzero(fl, c, lane == 0);
+            ok = g != 0u;
+            rdy_hi = j + g;  // records j .. j+g-1 were published behind one fence
+          }
+#else
           const bool ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
+#endif
           pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
 #pragma unroll
           for (int k = 0; k < NW; ++k) pv[k] = (!COND || ((mask >> k) & 1u)) ? ld_relaxed(pl + (1 + k) * 32 + lane) : 0u;

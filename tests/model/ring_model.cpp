@@ -10,12 +10,16 @@
 //   * region = pair % R; both roles wait for turn[region] == pair / R, the
 //     consumer advances it at exit;
 //   * per (region) a ring of S slots with 0/1 flags; record j lives in slot j % S;
-//   * producer: before writing record j >= S it publishes its pending records
-//     (fence + flag stores) and waits for slot j % S to be free; records are
-//     published in batches at every non-deferred commit;
+//   * producer: records are published in groups at every non-deferred commit:
+//     one fence, then record first + l gets flag value g - l (g = group size);
+//     before writing record j >= S it publishes its pending group and waits
+//     for slot j % S, but only if it must block: S records of its own pending,
+//     or the slot's flag still set (record j - S published, not yet freed);
 //   * consumer: before waiting on record j it frees its pending records if it
-//     holds S of them; waits for flag == 1 (acquire), reads, compares, and frees
-//     in batches at every non-deferred commit (release store of 0);
+//     holds S of them; for the first record of a group it waits for a nonzero
+//     flag (acquire) -- the value g says records j .. j+g-1 are visible, so
+//     those need no flag check of their own; it reads, compares, and frees in
+//     batches at every non-deferred commit (release store of 0);
 //   * the last finisher resets tickets and turns.
 // Workers (the resident CTA slots) take tickets until 2P are gone.  Checks: every
 // record is consumed exactly once, in order, with the payload its producer wrote
@@ -62,13 +66,13 @@ static void run_role(Queue& q, unsigned t, unsigned nblocks, const std::vector<b
   const unsigned region = pair % (unsigned)q.R, epoch = pair / (unsigned)q.R;
   while (q.turn[region].load(std::memory_order_acquire) != epoch) std::this_thread::yield();  // region ownership
   auto slot = [&](unsigned rec) { return (size_t)region * q.S + rec % (unsigned)q.S; };
-  unsigned j = 0, pend = 0;
+  unsigned j = 0, pend = 0, rdy_hi = 0;
   auto flush = [&]() {
     if (pend == 0) return;
     const unsigned first = j - pend;
     if (!consumer) {
       std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
-      for (unsigned l = 0; l < pend; ++l) q.flag[slot(first + l)].store(1, std::memory_order_relaxed);
+      for (unsigned l = 0; l < pend; ++l) q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
     } else {
       for (unsigned l = 0; l < pend; ++l) q.flag[slot(first + l)].store(0, std::memory_order_release);
     }
@@ -78,14 +82,18 @@ static void run_role(Queue& q, unsigned t, unsigned nblocks, const std::vector<b
     jitter(rng);
     const size_t s = slot(j);
     if (!consumer) {
-      if (j >= (unsigned)q.S) {
+      if (j >= (unsigned)q.S && (pend >= (unsigned)q.S || q.flag[s].load(std::memory_order_acquire) != 0)) {
         flush();
         while (q.flag[s].load(std::memory_order_acquire) != 0) std::this_thread::yield();
       }
       q.payload[s].store(tag(pair, j), std::memory_order_relaxed);
     } else {
       if (pend >= (unsigned)q.S) flush();
-      while (q.flag[s].load(std::memory_order_acquire) != 1) std::this_thread::yield();
+      if (j >= rdy_hi) {
+        unsigned g;
+        while ((g = q.flag[s].load(std::memory_order_acquire)) == 0) std::this_thread::yield();
+        rdy_hi = j + g;
+      }
       const uint64_t got = q.payload[s].load(std::memory_order_relaxed);
       if (got != tag(pair, j)) {
         g_errors.fetch_add(1);
