@@ -41,7 +41,7 @@ def model(tmp_path_factory):
 def test_ring_protocol_model(model, S, R, workers):
     for seed in range(3):
         r = subprocess.run([model, str(S), str(R), str(workers), "48", "60", str(seed + 17 * S + R), "3"],
-                           capture_output=True, text=True, timeout=120)
+                           capture_output=True, text=True, timeout=300)
         assert r.returncode == 0, r.stderr[-2000:]
         assert r.stdout.startswith("ok")
 
