@@ -30,10 +30,12 @@ CAMPAIGN = [
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
     # PrefixSum SMEM = warp total i of chunk ch (element ch*256 + i): the unprotected
     # scan reads 32 (sub-tile, warp) totals per chunk, the intra variants 16 (warp)
-    # totals, so i < 16 is a site every variant has
+    # totals, so i < 16 is a site every variant has; the intra layout's last total
+    # (i = 15) feeds no later warp of the tile (dead there, live in none), so the
+    # sampled sites are i < 15, live in every layout
     (lambda: PrefixSum(4096 * 9 + 5), {"load": lambda c: c.n, "compute": lambda c: 256 * 10,
                                        "smem": lambda c: (lambda rng: 256 * int(rng.integers(0, 10)) +
-                                                          int(rng.integers(0, 16))),
+                                                          int(rng.integers(0, 15))),
                                        "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
     (lambda: Reduction(300007), {"load": lambda c: c.n, "compute": lambda c: 1184 * 256,
                                  "smem": lambda c: 1184 * 8, "store_val": lambda c: 1, "store_addr": lambda c: 1}),
