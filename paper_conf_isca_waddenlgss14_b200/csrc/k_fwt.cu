@@ -207,7 +207,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fwt_kernel(FwtArgs a, Ctx c
   constexpr int PLANE = S::PLANE;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
   __shared__ float tile[Geom<V>::SMDUP == 2 ? PLANE + S::WORDS : S::WORDS];
-  Rep<V, M> rep(c);
+  Rep<V, M, true> rep(c);  // group flags: up to 8 records per warp
   rep.init(mb);
   for (; rep.active(); rep.advance()) {
     const unsigned tileid = (unsigned)rep.lblock;
@@ -349,7 +349,7 @@ __device__ __forceinline__ int p1x(int e) { return e ^ ((e >> 5) & 31); }
 
 template <int V, int M>
 __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, Ctx c) {
-  using R = Rep<V, M>;
+  using R = Rep<V, M, true>;  // group flags: 8 records per warp
   constexpr bool DUPL = R::SMDUP;
   constexpr bool PAD = V != V_NONE;  // layout choice (see p1_phys / p1x): measured per variant
   __shared__ unsigned mb[mbox_words<V>(BLS * Geom<V>::DUP)];
@@ -438,7 +438,7 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, C
 // planes XOR bank bit 4 (a warp's 16 logical lanes share it).
 template <int V, int M>
 __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_ps_kernel(FwtArgs a, Ctx c) {
-  using R = Rep<V, M>;
+  using R = Rep<V, M, true>;  // group flags: 8 records per warp
   constexpr bool DUPL = R::SMDUP;
   __shared__ unsigned mb[mbox_words<V>(BLS * Geom<V>::DUP)];
   __shared__ float tile[TE_MAX * Geom<V>::SMDUP];

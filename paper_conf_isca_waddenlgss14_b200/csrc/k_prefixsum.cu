@@ -38,9 +38,9 @@ struct PsArgs {
 };
 
 // u32 sum over the logical CTA (logical warps + duplicated smem)
-template <int V, int M>
-__device__ __forceinline__ unsigned block_sum_u32(const Rep<V, M>& rep, unsigned s, unsigned* sw) {
-  constexpr int LW = Rep<V, M>::LW;
+template <class R>
+__device__ __forceinline__ unsigned block_sum_u32(const R& rep, unsigned s, unsigned* sw) {
+  constexpr int LW = R::LW;
   constexpr int NLW = BL / LW;
 #pragma unroll
   for (int m = LW / 2; m >= 1; m >>= 1) s += rep.lshfl_xor(s, m);
@@ -125,7 +125,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_k
   constexpr bool FLAT = NQ * NLW == LW;          // every (sub-tile, warp) total on its own lane
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
   __shared__ unsigned sw[NQ * NLW * Geom<V>::SMDUP];
-  Rep<V, M> rep(c);
+  Rep<V, M, true> rep(c);  // group flags: many records per warp
   rep.init(mb);
   for (; rep.active(); rep.advance()) {
     const unsigned ch = a.nch - 1u - (unsigned)rep.lblock;  // reverse order: L2-hot chunks first

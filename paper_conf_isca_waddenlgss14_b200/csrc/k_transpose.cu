@@ -34,7 +34,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) tr_kernel(TrArgs a, Ctx c) 
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
   __shared__ unsigned tile[Geom<V>::SMDUP == 2 ? PLANE + SWORDS : SWORDS];
-  Rep<V, M> rep(c);
+  Rep<V, M, true> rep(c);  // group flags: 4 records per warp
   rep.init(mb);
   for (; rep.active(); rep.advance()) {
     const unsigned ty = (unsigned)rep.lblock / a.nsx, sx = (unsigned)rep.lblock % a.nsx;

@@ -175,13 +175,11 @@ __device__ __forceinline__ void cluster_sync_all() {
 #ifndef RMT_FREE_RELAXED
 #define RMT_FREE_RELAXED 0
 #endif
-// Inter queue group flags: a producer publishing
-// a group of g records behind one fence stores g, g-1, ..., 1 into their slot
-// flags, so a consumer that acquires the flag of the group's first record knows
-// the rest are visible too and reads their payloads without a flag round trip.
-#ifndef RMT_GROUP_FLAGS
-#define RMT_GROUP_FLAGS 1
-#endif
+// Inter queue group flags (Rep<..., GROUP = true>; DESIGN.md "Inter-Group
+// queue"): a producer publishing a group of g records behind one fence stores g,
+// g-1, ..., 1 into their slot flags, so a consumer that acquires the flag of the
+// group's first record knows the rest are visible too and reads their payloads
+// without a flag round trip.
 #ifndef RMT_SPIN_NS0
 #define RMT_SPIN_NS0 32     // first back-off sleep of a queue wait (0: pure spin)
 #endif
@@ -276,7 +274,12 @@ __device__ __forceinline__ unsigned mix32(unsigned x) {
 }
 
 // ---------------------------------------------------------------- replica state
-template <int V, int MODE>
+// GROUP: inter-group queue with group flags (below); chosen per kernel -- it
+// saves the consumer a flag round trip per record of a multi-record group, but
+// costs registers (measured: PrefixSum inter 3.98 -> 2.67x,
+// FWT 3.56 -> 3.41x, Transpose 3.11 -> 2.91x; BlackScholes 5.58 -> 6.48x and DCT
+// 3.77 -> 4.25x lose a CTA per SM to the extra registers)
+template <int V, int MODE, bool GROUP = false>
 struct Rep {
   static constexpr bool INTRA = (V == V_INTRA_SMEM || V == V_INTRA_REG || V == V_INTRA_NOLDS);
   // +LDS: kernel-written shared memory duplicated per replica;
@@ -465,7 +468,7 @@ struct Rep {
 #endif
         __syncwarp();
         // group flags: record first + l gets pend - l (its distance to the group's end)
-        if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), RMT_GROUP_FLAGS ? pend - lane : 1u);
+        if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), GROUP ? pend - lane : 1u);
       } else {
         __syncwarp();
 #if RMT_FREE_RELAXED
@@ -775,20 +778,20 @@ struct Rep {
           // free.  Publish our own pending records first, or our consumer could be
           // waiting for them while we wait for it.
           if (j >= (unsigned)c.S) {
-#if RMT_GROUP_FLAGS
-            // publish the pending group only if we must block on this slot, so
-            // that groups stay whole while the consumer keeps up.  The slot is
-            // ours only if record j - S was published and consumed: a flag of 0
-            // also marks our own unpublished records, so with S of them pending
-            // we must publish (and wait) before overwriting the oldest.
-            if (pend >= (unsigned)c.S || ld_acquire(fl) != 0u) {
+            if constexpr (GROUP) {
+              // publish the pending group only if we must block on this slot, so
+              // that groups stay whole while the consumer keeps up.  The slot is
+              // ours only if record j - S was published and consumed: a flag of 0
+              // also marks our own unpublished records, so with S of them pending
+              // we must publish (and wait) before overwriting the oldest.
+              if (pend >= (unsigned)c.S || ld_acquire(fl) != 0u) {
+                flush();
+                spin_until(fl, 0u, c, lane == 0);
+              }
+            } else {
               flush();
               spin_until(fl, 0u, c, lane == 0);
             }
-#else
-            flush();
-            spin_until(fl, 0u, c, lane == 0);
-#endif
           }
           pl[lane] = key;
 #pragma unroll
@@ -799,16 +802,16 @@ struct Rep {
           // release by one lane does not order the other lanes' in-flight stores).
         } else {
           if (pend >= (unsigned)c.S) flush();  // as above: never wait on a slot we still hold
-#if RMT_GROUP_FLAGS
           bool ok = true;
-          if (j >= rdy_hi) {  // each lane acquires the "ready" signal of the group's first record
-            const unsigned g = spin_nonzero(fl, c, lane == 0);
-            ok = g != 0u;
-            rdy_hi = j + g;  // records j .. j+g-1 were published behind one fence
+          if constexpr (GROUP) {
+            if (j >= rdy_hi) {  // each lane acquires the "ready" signal of the group's first record
+              const unsigned g = spin_nonzero(fl, c, lane == 0);
+              ok = g != 0u;
+              rdy_hi = j + g;  // records j .. j+g-1 were published behind one fence
+            }
+          } else {
+            ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
           }
-#else
-          const bool ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
-#endif
           pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
 #pragma unroll
           for (int k = 0; k < NW; ++k) pv[k] = (!COND || ((mask >> k) & 1u)) ? ld_relaxed(pl + (1 + k) * 32 + lane) : 0u;
