@@ -276,7 +276,8 @@ int binarysearch_run(Launch& L) {
       rc = launch_std<V>(L, bins_index_kernel<V, M>, bins_index_kernel<V_NONE, M_NORMAL>, Gi, BL, 0, a,
                          "binarysearch/index");
     if (rc) return rc;
-    return launch_std<V>(L, bins_kernel<V, M>, bins_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "binarysearch");
+    return launch_std<V>(L, bins_kernel<V, M>, bins_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "binarysearch",
+                         /*mult_inter=*/2);
   });
 }
 

@@ -169,7 +169,8 @@ int fw_issue(Launch& L) {
       L.ctx.f = f;
       if (k == k0) L.ctx.f.elem = f.elem - (long long)k0 * nn;
       else L.ctx.f.site = -1;
-      rc = launch_std<V>(L, fw_pass_kernel<V, M>, fw_pass_kernel<V_NONE, M_NORMAL>, Gp, BL, 0, a, "fw/pass");
+      rc = launch_std<V>(L, fw_pass_kernel<V, M>, fw_pass_kernel<V_NONE, M_NORMAL>, Gp, BL, 0, a, "fw/pass",
+                          /*mult_inter=*/2);
     }
     L.ctx.f = f;
     return rc;

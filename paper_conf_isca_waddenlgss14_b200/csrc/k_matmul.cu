@@ -406,7 +406,7 @@ int matmul_run(Launch& L) {
     a.kpc = KC / BK;
     const unsigned G = (M / BM) * (N / Cfg::BN);
     return launch_std<V>(L, mm_kernel<V, Mo>, mm_kernel<V_NONE, M_NORMAL>, G, Cfg::BL, Cfg::SMEM, a, "matmul",
-                         /*persistent=*/false, /*bl_none=*/NTHR);
+                         /*mult_inter=*/0, /*mult_cluster=*/0, /*bl_none=*/NTHR);
   });
 }
 

@@ -136,7 +136,7 @@ int reduction_run(Launch& L) {
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     int rc = launch_std<V>(L, red_partial_kernel<V, M>, red_partial_kernel<V_NONE, M_NORMAL>, G1, BL, 0, a1,
-                           "reduction/partial");
+                           "reduction/partial", /*mult_inter=*/1);
     if (rc) return rc;
     return launch_std<V>(L, red_final_kernel<V, M>, red_final_kernel<V_NONE, M_NORMAL>, 1, BL, 0, a2,
                          "reduction/final");

@@ -221,7 +221,8 @@ int sobel_run(Launch& L) {
   SobArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, H, W, nbx};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
-    return launch_std<V>(L, sobel_kernel<V, M>, sobel_kernel<V_NONE, M_NORMAL>, nbx * nby, BL, 0, a, "sobel");
+    return launch_std<V>(L, sobel_kernel<V, M>, sobel_kernel<V_NONE, M_NORMAL>, nbx * nby, BL, 0, a, "sobel", /*mult_inter=*/0,
+                         /*mult_cluster=*/0);
   });
 }
 

@@ -108,7 +108,8 @@ int transpose_run(Launch& L) {
   TrArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, H, W, nsx};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
-    return launch_std<V>(L, tr_kernel<V, M>, tr_kernel<V_NONE, M_NORMAL>, nsx * nty, BL, 0, a, "transpose");
+    return launch_std<V>(L, tr_kernel<V, M>, tr_kernel<V_NONE, M_NORMAL>, nsx * nty, BL, 0, a, "transpose",
+                         /*mult_inter=*/2);
   });
 }
 

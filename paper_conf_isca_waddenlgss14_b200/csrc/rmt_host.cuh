@@ -143,28 +143,27 @@ size_t pad_for_occupancy(K kn, int bn, size_t sn, int target) {
 // Standard launch of one RMT kernel instance: logical grid G of BL-thread
 // logical CTAs, `smem` dynamic shared bytes.  kr = the variant's kernel,
 // kn = the V_NONE kernel (used for the INFLATE ablation).
-// inter_group / inter_cluster launch a resident set of P replica pairs (P <=
-// the pairs that fit on the GPU at once, <= INTER_R queue regions, <= G) and
-// each pair walks the logical CTAs pair, pair + P, ... (Rep::active/advance);
-// `persistent = false` keeps one logical CTA per pair (kernels whose body is not
-// written as the logical-CTA loop).
-// Resident pairs per pair slot.  Measured on the suite (DESIGN.md section 7,
-// "Persistent pairs"): persistent DSMEM pairs help inter_cluster (transpose
-// 3.03 -> 2.68x, FWT 4.12 -> 3.94x), but persistent L2-queue pairs run in
-// lockstep with two L2 round trips per record on the consumer side and lose
-// (transpose 3.1 -> 4.4x), so inter_group keeps one logical CTA per pair.
-// Experiment knob RMT_INTER_PAIRS_MULT (k > 0: k x resident pairs for both; 0: none).
-inline int inter_pairs_mult(bool cluster) {
+// inter_group / inter_cluster launch P = mult x (the pairs that fit on the GPU
+// at once) replica pairs (<= G) and each pair walks the logical CTAs pair,
+// pair + P, ... (Rep::active/advance); mult = 0 keeps one logical CTA per pair
+// (and is required for kernels whose body is not the logical-CTA loop).
+// Persistent replica pairs ("Persistent pairs"): the
+// inter variants launch k x the pairs that fit on the GPU at once, and each pair
+// walks its share of the logical CTAs.  k is chosen per kernel from the suite
+// measurements (0 = one logical CTA per pair); experiment knob
+// RMT_INTER_PAIRS_MULT overrides it for every kernel.
+inline int inter_pairs_mult(int kernel_choice) {
   static int m = [] {
     const char* e = getenv("RMT_INTER_PAIRS_MULT");
     return e ? atoi(e) : -1;
   }();
-  return m >= 0 ? m : (cluster ? 1 : 0);
+  return m >= 0 ? m : kernel_choice;
 }
 
 template <int V, class Args>
-unsigned inter_pairs(void (*kr)(Args, Ctx), int block, size_t dyn_smem, unsigned G, bool cluster) {
-  if (inter_pairs_mult(cluster) <= 0) return G;
+unsigned inter_pairs(void (*kr)(Args, Ctx), int block, size_t dyn_smem, unsigned G, bool cluster, int mult) {
+  mult = inter_pairs_mult(mult);
+  if (mult <= 0) return G;
   int occ = 0;
   if (cluster) {
     cudaLaunchConfig_t cfg = {};
@@ -195,13 +194,13 @@ unsigned inter_pairs(void (*kr)(Args, Ctx), int block, size_t dyn_smem, unsigned
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     occ = per_sm * nsm / 2;
   }
-  unsigned P = (unsigned)(occ < 1 ? 1 : occ) * (unsigned)inter_pairs_mult(cluster);
+  unsigned P = (unsigned)(occ < 1 ? 1 : occ) * (unsigned)mult;
   return P < G ? P : G;
 }
 
 template <int V, class Args>
 int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned G, int BL, size_t smem,
-               const Args& a, const char* what, bool persistent = true, int bl_none = 0) {
+               const Args& a, const char* what, int mult_inter = 0, int mult_cluster = 1, int bl_none = 0) {
   if (G == 0) return RMT_OK;
   Ctx c = L.ctx;
   c.nblocks = (int)G;
@@ -229,10 +228,8 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
       dyn = (size_t)c.R + (size_t)(BL / 32) * c.S * (RING_WORDS * 32 + 1) * 4;
     }
     cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
-    if (persistent) {
-      c.pairs = (int)inter_pairs<V>(kr, Geom<V>::block(BL), dyn, G, true);
-      c.lstride = c.pairs;
-    }
+    c.pairs = (int)inter_pairs<V>(kr, Geom<V>::block(BL), dyn, G, true, mult_cluster);
+    c.lstride = c.pairs < (int)G ? c.pairs : 0;
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(Geom<V>::grid((unsigned)c.pairs));
     cfg.blockDim = dim3(Geom<V>::block(BL));
@@ -251,9 +248,9 @@ int launch_std(Launch& L, void (*kr)(Args, Ctx), void (*kn)(Args, Ctx), unsigned
     if (e != cudaSuccess) return cuda_check(e, what);
   } else {
     if (smem > 48 * 1024) cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (V == V_INTER && persistent) {
-      c.pairs = (int)inter_pairs<V>(kr, Geom<V>::block(BL), smem, G, false);
-      c.lstride = c.pairs;
+    if (V == V_INTER) {
+      c.pairs = (int)inter_pairs<V>(kr, Geom<V>::block(BL), smem, G, false, mult_inter);
+      c.lstride = c.pairs < (int)G ? c.pairs : 0;
     }
     // programmatic dependent launch: the grid is scheduled while the previous
     // kernel drains; Rep::init waits (griddepcontrol.wait) before any access
