@@ -59,9 +59,11 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_init_kernel(FwArgs a, Ct
 // width (coalesced), all loads in flight before the first use.  VPT per
 // variant, measured at n = 4096 (B200): none 4 (52 -> 40 ms), intra 2 (an
 // intra warp carries half the distinct bytes, so more vectors per thread),
-// inter 1 (larger inter CTAs were slower: 2 -> +5%, 8 -> 3.6x).
+// inter 2 with group flags (one published group of 4 records per warp and
+// logical CTA: 703 -> 497 ms at n = 4096 as n launches; 4 was slower, 799 ms;
+// the cooperative single launch below then gives 456 ms).
 #ifndef FW_VPT_INTER
-#define FW_VPT_INTER 1
+#define FW_VPT_INTER 2
 #endif
 #ifndef FW_VPT_INTRA
 #define FW_VPT_INTRA 2
@@ -73,62 +75,116 @@ template <int V>
 constexpr int fw_vpt() {
   return (V == V_INTER || V == V_CLUSTER) ? FW_VPT_INTER : V == V_NONE ? FW_VPT_NONE : FW_VPT_INTRA;
 }
+
+// Logical CTA lb of pass k: (row i, column chunk of BL*4*VPT words), so the row
+// and chunk are CTA-uniform (no per-thread division).  `kf` is the pass index
+// the fault hooks see (the global fault element is k * n^2 + e).
+template <int VPT, class R>
+__device__ __forceinline__ void fw_block(R& rep, const FwArgs& a, unsigned k, unsigned lb) {
+  constexpr int M = R::FAULT ? M_FAULT : M_NORMAL;
+  const unsigned nn = a.n * a.n;
+  const unsigned cpr = (a.n + BL * 4 * VPT - 1) / (BL * 4 * VPT);
+  const unsigned i = lb / cpr;
+  const unsigned jc = (lb - i * cpr) * (BL * 4 * VPT);
+  const unsigned dik0 = a.D[(size_t)i * a.n + k];  // one broadcast word per CTA row
+  // all VPT vector pairs in flight before the first use (L2 latency-bound:
+  // an intra warp carries half the distinct bytes of an unprotected warp)
+  uint4 dkj[VPT], dij[VPT];
+#pragma unroll
+  for (int it = 0; it < VPT; ++it) {
+    const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
+    dkj[it] = make_uint4(0, 0, 0, 0);
+    dij[it] = make_uint4(0, 0, 0, 0);
+    if (j < a.n) {
+      dkj[it] = *reinterpret_cast<const uint4*>(a.D + (size_t)k * a.n + j);
+      dij[it] = *reinterpret_cast<const uint4*>(a.D + i * a.n + j);
+    }
+  }
+#pragma unroll
+  for (int it = 0; it < VPT; ++it) {
+    const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
+    const bool active = j < a.n;
+    const unsigned e0 = i * a.n + j;
+    unsigned dik = dik0;
+    unsigned kj[4] = {dkj[it].x, dkj[it].y, dkj[it].z, dkj[it].w};
+    unsigned ij[4] = {dij[it].x, dij[it].y, dij[it].z, dij[it].w};
+    if constexpr (M == M_FAULT) {
+      dik = rep.fault(SITE_LOAD, (long long)i * a.n + k, dik);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) ij[q] = rep.fault(SITE_LOAD, (long long)e0 + q, ij[q]);
+    }
+    unsigned nd[4], np[4], mask = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      unsigned cand = dik + kj[q];
+      if constexpr (M == M_FAULT) cand = rep.fault(SITE_COMPUTE, (long long)e0 + q, cand);
+      const bool better = active && cand < ij[q];
+      mask |= (better ? 1u : 0u) << q;
+      nd[q] = cand;
+      np[q] = k;
+    }
+    rep.template commit<4, 0, false, true>(mask, active ? e0 : 0u, nd, nn,
+                                           [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); },
+                                           /*defer=*/true);
+    // one published group per logical CTA: every commit but the last is
+    // deferred (2 VPT <= the ring depth)
+    rep.template commit<4, 1, false, true>(mask, active ? e0 : 0u, np, nn,
+                                           [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); },
+                                           /*defer=*/it < VPT - 1);
+  }
+}
+
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ctx c) {
-  constexpr int VPT = fw_vpt<V>();
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
-  Rep<V, M> rep(c);
+  Rep<V, M, V == V_INTER> rep(c);
   rep.init(mb);
-  for (; rep.active(); rep.advance()) {
-    const unsigned nn = a.n * a.n;
-    // logical CTA = (row i, column chunk of BL*4*VPT words): the row and chunk
-    // are CTA-uniform (no per-thread division)
-    const unsigned cpr = (a.n + BL * 4 * VPT - 1) / (BL * 4 * VPT);
-    const unsigned i = (unsigned)rep.lblock / cpr;
-    const unsigned jc = ((unsigned)rep.lblock - i * cpr) * (BL * 4 * VPT);
-    const unsigned dik0 = a.D[(size_t)i * a.n + a.k];  // one broadcast word per CTA row
-    // all VPT vector pairs in flight before the first use (L2 latency-bound:
-    // an intra warp carries half the distinct bytes of an unprotected warp)
-    uint4 dkj[VPT], dij[VPT];
-#pragma unroll
-    for (int it = 0; it < VPT; ++it) {
-      const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
-      dkj[it] = make_uint4(0, 0, 0, 0);
-      dij[it] = make_uint4(0, 0, 0, 0);
-      if (j < a.n) {
-        dkj[it] = *reinterpret_cast<const uint4*>(a.D + (size_t)a.k * a.n + j);
-        dij[it] = *reinterpret_cast<const uint4*>(a.D + i * a.n + j);
-      }
+  for (; rep.active(); rep.advance()) fw_block<fw_vpt<V>()>(rep, a, a.k, (unsigned)rep.lblock);
+  rep.finish();
+}
+
+// Inter-Group FloydWarshall as ONE cooperative launch: 2P resident CTAs (P
+// replica pairs, one ticket and one queue region per pair for the whole run)
+// walk the logical CTAs of pass k, meet at a grid barrier, and go on to pass
+// k + 1 -- instead of n launches that each take tickets, regions and an exit
+// count for thousands of short-lived CTA pairs.  The
+// barrier orders every consumer's committed D stores of pass k before any
+// replica's loads of pass k + 1.  Fault builds see per-pass fault descriptors
+// (the host encodes the pass: elem = k0 n^2 + e).
+__device__ __forceinline__ void grid_barrier(unsigned* bar, unsigned nctas) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned gen = ld_acquire(bar + 1);
+    __threadfence();
+    if (atomicAdd(bar, 1u) == nctas - 1u) {
+      bar[0] = 0u;
+      st_release(bar + 1, gen + 1u);
+    } else {
+      while (ld_acquire(bar + 1) == gen) __nanosleep(32);
     }
-#pragma unroll
-    for (int it = 0; it < VPT; ++it) {
-      const unsigned j = jc + ((unsigned)it * BL + (unsigned)rep.ltid) * 4;
-      const bool active = j < a.n;
-      const unsigned e0 = i * a.n + j;
-      unsigned dik = dik0;
-      unsigned kj[4] = {dkj[it].x, dkj[it].y, dkj[it].z, dkj[it].w};
-      unsigned ij[4] = {dij[it].x, dij[it].y, dij[it].z, dij[it].w};
-      if constexpr (M == M_FAULT) {
-        dik = rep.fault(SITE_LOAD, (long long)i * a.n + a.k, dik);
-#pragma unroll
-        for (int q = 0; q < 4; ++q) ij[q] = rep.fault(SITE_LOAD, (long long)e0 + q, ij[q]);
-      }
-      unsigned nd[4], np[4], mask = 0;
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        unsigned cand = dik + kj[q];
-        if constexpr (M == M_FAULT) cand = rep.fault(SITE_COMPUTE, (long long)e0 + q, cand);
-        const bool better = active && cand < ij[q];
-        mask |= (better ? 1u : 0u) << q;
-        nd[q] = cand;
-        np[q] = a.k;
-      }
-      rep.template commit<4, 0, false, true>(mask, active ? e0 : 0u, nd, nn,
-                                [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.D, idx, m, v); },
-                                /*defer=*/true);
-      rep.template commit<4, 1, false, true>(mask, active ? e0 : 0u, np, nn,
-                                [&](unsigned idx, unsigned m, const unsigned* v) { store4(a.P, idx, m, v); });
+  }
+  __syncthreads();
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_coop_kernel(FwArgs a, Ctx c, unsigned* bar) {
+  __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  Ctx cf = c;  // fault builds: the descriptor is re-aimed at each pass
+  Rep<V, M, true> rep(cf);
+  rep.init(mb);
+  const int first = rep.lblock;
+  const long long nn = (long long)a.n * a.n;
+  for (unsigned k = 0; k < a.n; ++k) {
+    if constexpr (M == M_FAULT) {
+      cf.f = c.f;
+      if ((long long)k == c.f.elem / nn) cf.f.elem = c.f.elem - (long long)k * nn;
+      else cf.f.site = -1;
     }
+    for (int lb = first; lb < c.nblocks; lb += rep.lstride) {
+      rep.lblock = lb;
+      fw_block<fw_vpt<V>()>(rep, a, k, (unsigned)lb);
+    }
+    grid_barrier(bar, 2u * (unsigned)c.pairs);
   }
   rep.finish();
 }
@@ -143,10 +199,43 @@ int floydwarshall_validate(const rmt_bufs_t* b, int64_t n) {
   }
   return RMT_OK;
 }
-size_t floydwarshall_scratch(int64_t, const int64_t*) { return 0; }
+size_t floydwarshall_scratch(int64_t, const int64_t*) { return 64; }  // inter_group grid barrier
 int floydwarshall_inter_warps(int64_t, const int64_t*) { return BL / 32; }
 
 namespace {
+
+// inter_group: the whole pass sequence as one cooperative launch (fw_coop_kernel).
+template <int V, int M>
+int fw_coop_launch(Launch& L, const FwArgs& a, unsigned Gp) {
+  int per_sm = 0, dev = 0, nsm = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fw_coop_kernel<V, M>, Geom<V>::block(BL), 0) !=
+          cudaSuccess ||
+      per_sm < 2)
+    return cuda_check(cudaErrorInvalidConfiguration, "fw/coop occupancy");
+  Ctx c = L.ctx;
+  unsigned P = (unsigned)(per_sm * nsm / 2);
+  if (P > (unsigned)c.R) P = (unsigned)c.R;  // one queue region per pair, no hand-over
+  if (P > Gp) P = Gp;
+  c.nblocks = (int)Gp;
+  c.pairs = (int)P;
+  c.lstride = (int)P;
+  unsigned* bar = (unsigned*)L.scratch;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(2 * P);
+  cfg.blockDim = dim3(Geom<V>::block(BL));
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = L.stream;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;  // every CTA co-resident: the grid barrier cannot deadlock
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  int rc = cuda_check(cudaLaunchKernelEx(&cfg, fw_coop_kernel<V, M>, a, c, bar), "fw/coop");
+  if (!rc) L.launches += 1;
+  return rc;
+}
 
 // The n + 1 launches of one FloydWarshall call, issued on L.stream.
 int fw_issue(Launch& L) {
@@ -164,6 +253,10 @@ int fw_issue(Launch& L) {
     const unsigned Gp = n * ((n + BL * 4 * vpt - 1) / (BL * 4 * vpt));  // rows x column chunks
     L.ctx.f.site = -1;  // the init pass carries no fault
     int rc = launch_std<V>(L, fw_init_kernel<V, M>, fw_init_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "fw/init");
+    L.ctx.f = f;
+    if constexpr (V == V_INTER) {
+      if (!L.inflate && M != M_NOCOMM) return rc ? rc : fw_coop_launch<V, M>(L, a, Gp);
+    }
     for (unsigned k = 0; k < n && rc == RMT_OK; ++k) {
       a.k = k;
       L.ctx.f = f;
@@ -227,7 +320,9 @@ int floydwarshall_run(Launch& L) {
     cudaGetLastError();
     cs = cudaStreamCaptureStatusNone;
   }
-  if (cs != cudaStreamCaptureStatusNone || n < 64) return fw_issue(L);
+  if (cs != cudaStreamCaptureStatusNone || n < 64 ||
+      (L.variant == RMT_INTER_GROUP && !L.inflate && L.mode != M_NOCOMM))  // inter: 2 launches, no graph
+    return fw_issue(L);
   const std::string key = fw_key(L);
   std::lock_guard<std::mutex> lock(g_fw_mu);
   auto it = g_fw_graphs.begin();
