@@ -97,6 +97,9 @@ def parse():
                    help="per (kernel, variant) NVML energy window; 0 disables the energy table")
     p.add_argument("--ablations", action="store_true",
                    help="also time the INFLATE and NOCOMM ablations per kernel x RMT variant (cost attribution)")
+    p.add_argument("--fwt-exchange", default="p2p", choices=["p2p", "sendrecv"],
+                   help="multi-GPU FWT cross-shard stage: the fused combine kernel reading the partner's shard over "
+                        "NVLink peer memory (p2p), or NCCL send/recv then the combine kernel")
     p.add_argument("--dist-backend", default="nccl",
                    help="nccl (one GPU per rank); gloo only to exercise the multi-rank path on one GPU")
     return p.parse_args()
@@ -346,8 +349,10 @@ def main():
     s_tmp = torch.zeros(2, dtype=torch.int32, device="cuda")
     totals = torch.zeros(world, dtype=torch.int64, device="cuda")
     fwt_n = max([j.n for j in jobs if j.kernel == "fwt"] or [0])
-    fwt_recv = torch.empty(fwt_n if world > 1 else 0, dtype=torch.float32, device="cuda")
+    fwt_recv = torch.empty(fwt_n if world > 1 and args.fwt_exchange == "sendrecv" else 0, dtype=torch.float32,
+                           device="cuda")
     fwt_tmp = torch.empty_like(fwt_recv)
+    peer_fwt = parallel.PeerFWT(fwt_n, rmt) if world > 1 and fwt_n and args.fwt_exchange == "p2p" else None
 
     def one(j, v):
         """One launch of job j under variant v; for N > 1 the kernels that need a
@@ -357,7 +362,10 @@ def main():
             return parallel.global_prefixsum(j.dev[0], j.dev[1], s_tmp, totals, err, rmt, variant=v,
                                              ws_red=ws_aux[(j.kernel, v)], ws_ps=ws[(j.kernel, v)]) + 1
         if world > 1 and j.kernel == "fwt":
-            # local transform + log2 G cross-shard butterfly stages (send/recv + combine kernel)
+            # local transform + log2 G cross-shard butterfly stages: the combine kernel reads the
+            # partner's shard over peer memory (fused), or after an NCCL send/recv
+            if peer_fwt is not None:
+                return peer_fwt.run(j.dev[0], err, v, workspace=ws[(j.kernel, v)], ws_comb=ws_aux[(j.kernel, v)])[1]
             return parallel.global_fwt(j.dev[0], j.dev[1].view(torch.float32), fwt_recv, fwt_tmp, err, rmt,
                                        variant=v, workspace=ws[(j.kernel, v)], ws_comb=ws_aux[(j.kernel, v)])
         if world > 1 and j.kernel == "reduction":
@@ -428,6 +436,42 @@ def main():
             if v != "none" and "none" in variants:
                 d[v]["slowdown"] = round(ms / per[(j.kernel, "none")], 3)
         kernels[j.kernel] = d
+
+    # ---- configs[0] (BlackScholes 2^16, launch-latency bound): microseconds per
+    # launch from a CUDA graph of 100 launches per variant (SURVEY.md:559)
+    graph_us = None
+    if args.config == "bs16":
+        graph_us = {}
+        err_g = torch.zeros(1, dtype=torch.int64, device="cuda")
+        gs = torch.cuda.Stream()
+        for j in jobs:
+            for v in variants:
+                w = ws[(j.kernel, v)]
+                gs.wait_stream(stream)
+                with torch.cuda.stream(gs):
+                    for _ in range(3):  # warm outside the capture (lazy module loading)
+                        rmt.launch(j.kernel, v, j.dev, j.n, err_g, dims=j.dims, workspace=w, stream=gs.cuda_stream)
+                    g = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(g, stream=gs):
+                        for _ in range(100):
+                            rmt.launch(j.kernel, v, j.dev, j.n, err_g, dims=j.dims, workspace=w,
+                                       stream=gs.cuda_stream)
+                stream.wait_stream(gs)
+                ts = []
+                for r in range(6):
+                    a = torch.cuda.Event(enable_timing=True)
+                    b = torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
+                    g.replay()
+                    b.record(stream)
+                    torch.cuda.synchronize()
+                    if r:
+                        ts.append(a.elapsed_time(b) * 1e3 / 100)
+                graph_us[v] = round(statistics.median(ts), 3)
+                del g
+        graph_us = {"us_per_launch": graph_us, "note": "median of 5 replays of a CUDA graph of 100 launches",
+                    "slowdown": {v: round(graph_us[v] / graph_us["none"], 3) for v in graph_us if "none" in graph_us},
+                    "err_count": int(err_g.item())}
 
     # ---- the four other BASELINE.json kernels (per-launch medians after the step)
     rest = {}
@@ -667,12 +711,15 @@ def main():
                        "value": "baseline (none) HBM GB/s: sum of algorithmic bytes / sum of none launch times"},
             "step_gbs_all_variants": round(step_bytes * args.steps * world / (ms_total * 1e-3) / 1e9, 1),
             "slowdown_geomean": slowdown_geomean, "baseline_frac": baseline_frac,
-            "kernels": kernels, "rest10": rest or None, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "kernels": kernels, "rest10": rest or None, "graph_launch": graph_us, "roofline": roofline,
+            "cpu_baseline": cpu, "e2e": e2e,
             "attribution": attribution, "extra_variants": extra, "energy": energy,
             "gpu_launches": counts["gpu_launches"], "err_count": errs,
             "clocks": clk.summary(),
         }
         print(json.dumps(line), flush=True)
+    if peer_fwt is not None:
+        peer_fwt.close()
     if world > 1:
         dist.destroy_process_group()
 

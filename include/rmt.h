@@ -286,6 +286,23 @@ int rmt_last_launch_count(void);
  * replication.  Synchronous; allocates and frees its own device buffer. */
 int rmt_probe_cluster_placement(int64_t pairs, int64_t* same_sm_pairs);
 
+/*
+ * Peer device memory for the fused multi-GPU exchange (DESIGN.md
+ * section 9): rmt_ipc_export writes the CUDA IPC handle (RMT_IPC_HANDLE_BYTES
+ * bytes, caller-owned) of the allocation holding dev_ptr and dev_ptr's offset
+ * in it; the partner rank passes both to rmt_ipc_open, which returns a device
+ * pointer valid in the calling process (NVLink peer-to-peer access is enabled
+ * lazily when the memory lives on another GPU; two processes on one GPU share
+ * the memory).  That pointer may be passed as any rmt_launch input buffer: the
+ * FWT cross-shard stage (dims {1, upper}) then reads the partner's shard
+ * directly, with no staged copy.  rmt_ipc_close(ptr, offset) unmaps it.
+ * Synchronous; not graph-capturable; RMT_ECUDA on failure.
+ */
+#define RMT_IPC_HANDLE_BYTES 64
+int rmt_ipc_export(const void* dev_ptr, void* handle, int64_t* offset);
+int rmt_ipc_open(const void* handle, int64_t offset, void** dev_ptr);
+int rmt_ipc_close(void* dev_ptr, int64_t offset);
+
 const char* rmt_strerror(int code);
 const char* rmt_last_error(void); /* thread-local detail of the last failure */
 const char* rmt_kernel_name(int kernel);

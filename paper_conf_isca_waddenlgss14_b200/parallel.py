@@ -167,6 +167,72 @@ def global_fwt(x_local, y_local, recv, tmp, err, rmt_mod, variant="none", worksp
     return k
 
 
+def device_barrier(group=None, device=None):
+    """Every rank's previously launched kernels complete before any rank's next
+    ones start: a one-element NCCL all-reduce is stream-ordered on every rank (no
+    host wait); gloo (tests) synchronises the device and meets on the host."""
+    if not _active(group):
+        return
+    if _host_staged(group):
+        torch.cuda.synchronize()
+        dist.barrier(group=group)
+    else:
+        t = torch.zeros(1, dtype=torch.int32, device=device or "cuda")
+        dist.all_reduce(t, group=group)
+
+
+class PeerFWT:
+    """The fused multi-GPU FWT: each rank
+    keeps two shard buffers and exports both as CUDA IPC handles once; every
+    cross-shard stage runs the RMT combine kernel with the PARTNER's current
+    buffer as its input p -- peer-to-peer loads over NVLink, so the exchange
+    and the butterfly are one kernel and no staged copy is made.  Stage s reads
+    buffer cur of both ranks and writes buffer 1 - cur; a device barrier before
+    each stage makes the partner's writes of cur visible, and one after the last
+    stage keeps a rank from reusing a buffer its partner may still be reading."""
+
+    def __init__(self, n: int, rmt_mod, group=None, device="cuda"):
+        self.n, self.rmt, self.group = n, rmt_mod, group
+        self.ws, self.rk = world() if group is None else (dist.get_world_size(group), dist.get_rank(group))
+        if self.ws & (self.ws - 1):
+            raise ValueError("global FWT needs a power-of-two number of ranks")
+        self.buf = [torch.empty(n, dtype=torch.float32, device=device) for _ in range(2)]
+        mine = [rmt_mod.ipc_export(b) for b in self.buf]
+        allh = [None] * self.ws
+        if _active(group):
+            dist.all_gather_object(allh, mine, group=group)
+        else:
+            allh = [mine]
+        self.peer, self._opened = {}, {}
+        for s in fwt_partner_stages(self.ws):
+            q = self.rk ^ s
+            views = []
+            for h, off in allh[q]:
+                # both buffers may live in one allocation: a handle is opened once
+                if h not in self._opened:
+                    self._opened[h] = rmt_mod.ipc_open(h, 0, 0)
+                views.append(rmt_mod.DevPtr(self._opened[h].ptr + off, 4 * n))
+            self.peer[q] = views
+
+    def close(self):
+        for d in self._opened.values():
+            self.rmt.ipc_close(d)
+        self.peer, self._opened = {}, {}
+
+    def run(self, x_local, err, variant="none", workspace=None, ws_comb=None):
+        """Returns (this rank's slice of the global transform, kernels launched)."""
+        k = self.rmt.launch("fwt", variant, [x_local, self.buf[0]], self.n, err, dims=(0,), workspace=workspace)
+        cur = 0
+        for s in fwt_partner_stages(self.ws):
+            q = self.rk ^ s
+            device_barrier(self.group)
+            k += self.rmt.launch("fwt", variant, [self.buf[cur], self.buf[1 - cur], self.peer[q][cur]], self.n, err,
+                                 dims=(1, 1 if self.rk > q else 0), workspace=ws_comb)
+            cur = 1 - cur
+        device_barrier(self.group)
+        return self.buf[cur], k
+
+
 def sobel_halo_rows(H_total: int, r0: int, r1: int) -> tuple[int, int]:
     """Input rows [lo, hi) a rank owning output rows [r0, r1) of an H_total-row
     image needs: one halo row above and below, clipped at the image border (the

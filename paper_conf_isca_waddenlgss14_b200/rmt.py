@@ -103,6 +103,12 @@ def lib() -> ctypes.CDLL:
         L.rmt_workspace_status.restype = I32
         L.rmt_set_stress.argtypes = [I32, I32, I32, ctypes.c_longlong]
         L.rmt_set_stress.restype = I32
+        L.rmt_ipc_export.argtypes = [P, P, ctypes.POINTER(ctypes.c_int64)]
+        L.rmt_ipc_export.restype = I32
+        L.rmt_ipc_open.argtypes = [P, I64, ctypes.POINTER(P)]
+        L.rmt_ipc_open.restype = I32
+        L.rmt_ipc_close.argtypes = [P, I64]
+        L.rmt_ipc_close.restype = I32
         _lib = L
     return _lib
 
@@ -121,7 +127,36 @@ def _tensor_dtype(t) -> int:
     raise RmtError(f"cannot infer rmt dtype for {t.dtype}")
 
 
+class DevPtr:
+    """A raw device pointer of `nbytes` bytes usable as an rmt_launch buffer
+    (e.g. a peer rank's buffer opened with ipc_open)."""
+
+    def __init__(self, ptr: int, nbytes: int, offset: int = 0):
+        self.ptr, self.nbytes, self.offset = int(ptr), int(nbytes), int(offset)
+
+
+def ipc_export(t: torch.Tensor):
+    """(handle bytes, offset) of the device allocation holding tensor t."""
+    h = (ctypes.c_char * 64)()
+    off = ctypes.c_int64(0)
+    _check(lib().rmt_ipc_export(t.data_ptr(), h, ctypes.byref(off)), "rmt_ipc_export")
+    return bytes(h), off.value
+
+
+def ipc_open(handle: bytes, offset: int, nbytes: int) -> DevPtr:
+    p = ctypes.c_void_p(0)
+    _check(lib().rmt_ipc_open(ctypes.create_string_buffer(handle, 64), int(offset), ctypes.byref(p)),
+           "rmt_ipc_open")
+    return DevPtr(p.value, nbytes, offset)
+
+
+def ipc_close(d: DevPtr):
+    _check(lib().rmt_ipc_close(d.ptr, d.offset), "rmt_ipc_close")
+
+
 def _ptr(t):
+    if isinstance(t, DevPtr):
+        return t.ptr, t.nbytes
     if isinstance(t, torch.Tensor):
         return t.data_ptr(), t.numel() * t.element_size()
     import numpy as np  # host numpy buffers (rmt_run_host)

@@ -112,6 +112,19 @@ def _shards(rank):
         return e, [yy[q * nl:(q + 1) * nl] for q in range(WS)]
     cases["fwt"] = (fwt_shard, fwt_full)
 
+    # the fused FWT: the combine kernel reads the partner's shard through CUDA IPC
+    # (peer-to-peer over NVLink on a multi-GPU box; shared memory of one GPU here)
+    peer = parallel.PeerFWT(nl, rmt)
+
+    def fwt_p2p_shard(v):
+        x = _dev(inputs.fwt_x(5, nl, rank * nl))
+        err = torch.zeros(1, dtype=torch.int64, device="cuda")
+        y, _ = peer.run(x, err, v, workspace=rmt.make_workspace("fwt", v, nl),
+                        ws_comb=rmt.make_workspace("fwt", v, nl, (1, 0)))
+        torch.cuda.synchronize()
+        return int(err.item()), y.cpu().numpy().view(np.uint32)
+    cases["fwt_p2p"] = (fwt_p2p_shard, fwt_full)
+
     # PrefixSum: device all-gather of the shard totals -> device carry
     npl = (1 << 19) + 1028
 
