@@ -461,14 +461,25 @@ struct Rep {
       if (pend == 0u) return;
       const unsigned first = j - pend;
       if (!consumer) {
+        // group flags: record first + l gets pend - l (its distance to the
+        // group's end).  The non-first flags are stored BEFORE the fence and
+        // the first record's flag (the group's "ready" signal) after it: a
+        // consumer that acquired flag[first] then frees the other slots only
+        // after their flag stores, never before one lands late and leaves a
+        // stale "full" flag (found by tests/model/ring_model.cpp)
+        if constexpr (GROUP)
+          if ((unsigned)lane - 1u < pend - 1u) st_relaxed(c.flags + slot_index(first + lane), pend - lane);
 #if RMT_PUB_FENCE_SC
         asm volatile("fence.sc.gpu;" ::: "memory");
 #else
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
 #endif
         __syncwarp();
-        // group flags: record first + l gets pend - l (its distance to the group's end)
-        if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), GROUP ? pend - lane : 1u);
+        if constexpr (GROUP) {
+          if (lane == 0) st_relaxed(c.flags + slot_index(first), pend);
+        } else {
+          if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), 1u);
+        }
       } else {
         __syncwarp();
 #if RMT_FREE_RELAXED

@@ -11,7 +11,8 @@
 //     consumer advances it at exit;
 //   * per (region) a ring of S slots with 0/1 flags; record j lives in slot j % S;
 //   * producer: records are published in groups at every non-deferred commit:
-//     one fence, then record first + l gets flag value g - l (g = group size);
+//     record first + l (l >= 1) gets flag value g - l (g = group size), then
+//     one fence, then record first gets g (the group's "ready" signal);
 //     before writing record j >= S it publishes its pending group and waits
 //     for slot j % S, but only if it must block: S records of its own pending,
 //     or the slot's flag still set (record j - S published, not yet freed);
@@ -71,8 +72,18 @@ static void run_role(Queue& q, unsigned t, unsigned nblocks, const std::vector<b
     if (pend == 0) return;
     const unsigned first = j - pend;
     if (!consumer) {
+      // the group's non-first flags go out BEFORE the fence and the first
+      // record's flag after it: a consumer that acquires flag[first] then sees
+      // every other flag of the group already stored, so its later frees of
+      // those slots cannot be overtaken by a late producer flag store (which
+      // would leave a stale "full" flag: a stale read or a deadlock)
+      // (jitter between the stores: lanes' stores land in any order)
+      for (unsigned l = 1; l < pend; ++l) {
+        q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
+        jitter(rng);
+      }
       std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
-      for (unsigned l = 0; l < pend; ++l) q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
+      q.flag[slot(first)].store(pend, std::memory_order_relaxed);
     } else {
       for (unsigned l = 0; l < pend; ++l) q.flag[slot(first + l)].store(0, std::memory_order_release);
     }

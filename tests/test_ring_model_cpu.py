@@ -9,7 +9,10 @@ threads standing in for the resident CTA slots.  Every configuration must finish
 4 and 8, one region (every pair hands the ring to the next) or several, and
 down to 2 workers (the minimum residency the deadlock-freedom argument needs).
 A mutant without the consumer's "free before waiting when S records are held"
-rule must fail, so the model can tell the difference.
+rule must fail, and so must a mutant that publishes a group's flags in record
+order behind one fence (a consumer that acquired the first flag may free a
+later slot before that slot's flag store lands, leaving a stale "full" flag),
+so the model can tell the difference.
 """
 import os
 import subprocess
@@ -41,7 +44,7 @@ def model(tmp_path_factory):
 def test_ring_protocol_model(model, S, R, workers):
     for seed in range(3):
         r = subprocess.run([model, str(S), str(R), str(workers), "48", "60", str(seed + 17 * S + R), "3"],
-                           capture_output=True, text=True, timeout=300)
+                           capture_output=True, text=True, timeout=60)
         assert r.returncode == 0, r.stderr[-2000:]
         assert r.stdout.startswith("ok")
 
@@ -57,3 +60,28 @@ def test_ring_model_detects_missing_consumer_free(tmp_path):
     except subprocess.TimeoutExpired:
         failed = True  # deadlock
     assert failed, "the model accepted a protocol without the consumer-side free rule"
+
+
+def test_ring_model_detects_group_flags_published_in_order(tmp_path):
+    text = open(SRC).read()
+    fixed = """      for (unsigned l = 1; l < pend; ++l) {
+        q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
+        jitter(rng);
+      }
+      std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
+      q.flag[slot(first)].store(pend, std::memory_order_relaxed);"""
+    in_order = """      std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
+      for (unsigned l = 0; l < pend; ++l) {
+        q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
+        jitter(rng);
+      }"""
+    assert fixed in text
+    exe = _build(tmp_path, text.replace(fixed, in_order), "ring_in_order")
+    failures = 0
+    for seed in range(1, 4):
+        try:
+            r = subprocess.run([exe, "2", "1", "2", "48", "60", str(seed), "3"], capture_output=True, text=True, timeout=10)
+            failures += r.returncode != 0
+        except subprocess.TimeoutExpired:
+            failures += 1  # a stale full flag: the producer waits forever
+    assert failures > 0, "the model accepted group flags published first-record-first"
