@@ -3,15 +3,25 @@
 // Batched lower_bound (reading R-BIN1): idx[j] = #{i : A[i] < q[j]}.
 //
 // B200 design.  A plain binary search over a 256 MiB array misses L2 on ~11 of
-// its 26 levels (every probe is a different 32-B sector).  Instead, each launch
-// first builds a 16-ary sample hierarchy L_k[j] = A[16^k j] (k = 1..T, padded
-// with 0xFFFFFFFF to a multiple of 16; ~N/15 words, dense and L2-resident) --
-// itself an RMT-protected kernel whose stores are committed -- then each query
-// binary-searches the small top level L_T and descends with ONE 64-B block scan
-// per level: if jj = lower_bound in L_{k+1}, then lower_bound in L_k =
-// 16(jj-1) + #{block jj-1 of L_k < key} (jj > 0), which is exact because
-// L_k[16(jj-1)] < key <= L_k[16 jj].  Logical thread = 4 interleaved queries,
-// one 16-B vector commit of idx.
+// its 26 levels.  Instead each launch first builds a 32-ary sample hierarchy
+// L_k[j] = A[32^k j] (k = 1..T, each padded with 0xFFFFFFFF to a multiple of
+// 32 entries; ~N/31 words, L2-resident) -- itself an RMT-protected kernel whose
+// stores are committed -- where T is the first level of at most TMAX entries.
+// The query kernel copies L_T into shared memory once per CTA and finds
+// lower_bound(L_T, key) by a branch-free binary search there; it then descends
+// with ONE 128-B block scan per level: if jj = lower_bound in L_{k+1}, then
+// lower_bound in L_k = 32(jj-1) + #{block jj-1 of L_k < key} (jj > 0), exact
+// because L_k[32(jj-1)] < key <= L_k[32 jj].  For N = 2^26 that is L3 (2048
+// entries) in shared memory and three 128-B global blocks per query (L2, L1
+// in L2; A from DRAM).
+//
+// Why 128-B blocks: a random miss moves a whole 128-B line from DRAM whatever
+// the request size (tools/gather_probe.cu: 117.5 B of DRAM per random 16-, 32-
+// or 64-B read, ~53 G misses/s), so the A block costs the same DRAM time at
+// 128 B as at 64 B, and one 128-B line per query and level is also the L1 data
+// pipe's unit (the 64-B design spent a wavefront per 64 B and 7 levels).
+// Group of 4 logical lanes per query, one 32-B load each (LDG.256); logical
+// thread = 2 interleaved queries, one 8-B vector commit of idx.
 #include <string.h>
 
 #include "rmt_host.cuh"
@@ -20,19 +30,21 @@ namespace rmt {
 namespace {
 
 constexpr int BL = 256;
-constexpr int VEC = 4;
-constexpr int FAN = 16;       // samples per block
+constexpr int VEC = 2;
+constexpr int FAN = 32;       // entries per block (128 B)
 constexpr int MAXLEV = 8;
-constexpr unsigned TOP_MAX = FAN;   // sample until the top level fits in one block
+constexpr unsigned TMAX = 8192;   // shared-memory table: at most 8192 entries (32 KiB per replica)
+constexpr unsigned CHUNK = BL * VEC;  // queries per logical CTA iteration
 
 struct Levels {
-  int T;                         // number of sample levels (0: search A directly)
+  int T;                         // table level (>= 1): L_T lives in shared memory
   unsigned n[MAXLEV + 1];        // entries per level (n[0] = N)
   unsigned off[MAXLEV + 1];      // word offset of level k (k >= 1) in the scratch
-  unsigned padded[MAXLEV + 1];   // entries rounded up to a multiple of 16
+  unsigned padded[MAXLEV + 1];   // entries rounded up to a multiple of 32
   unsigned vecs_before[MAXLEV + 2];  // index-build vector ranges
-  unsigned N16;                  // N rounded down to a multiple of 16
-  unsigned tail_off;             // word offset of the padded copy of A[N16, N) (16 words)
+  unsigned N32;                  // N rounded down to a multiple of 32
+  unsigned tail_off;             // word offset of the padded copy of A[N32, N) (32 words)
+  unsigned P;                    // table entries in shared memory: a power of two >= n[T]
 };
 
 struct BsArgs {
@@ -41,7 +53,10 @@ struct BsArgs {
   unsigned* idx;
   unsigned* lev;  // scratch: sample levels
   unsigned N, Q;
-  int top_iters;
+  unsigned iters;   // chunks of CHUNK queries per logical CTA
+  unsigned plane;   // +LDS: replica r's table copy starts at word r * plane (P + 1: the
+                    // pair's two copies of an entry sit in different banks)
+  unsigned a32;     // A is 32-B aligned (256-bit block loads)
   Levels L;
 };
 
@@ -51,38 +66,50 @@ Levels make_levels(unsigned N) {
   L.n[0] = N;
   unsigned off = 0;
   int k = 0;
-  while (L.n[k] > TOP_MAX && k < MAXLEV) {
+  do {
     ++k;
     L.n[k] = (L.n[k - 1] + FAN - 1) / FAN;
     L.padded[k] = (L.n[k] + FAN - 1) / FAN * FAN;
+    if (L.padded[k] == 0) L.padded[k] = FAN;  // N = 0: one all-padding block
     L.off[k] = off;
     off += L.padded[k];
-  }
+  } while (L.n[k] > TMAX && k < MAXLEV);
   L.T = k;
   L.vecs_before[1] = 0;
   for (int i = 1; i <= L.T; ++i) L.vecs_before[i + 1] = L.vecs_before[i] + L.padded[i] / 4;
-  L.N16 = N & ~15u;
+  L.N32 = N & ~(unsigned)(FAN - 1);
   L.tail_off = off;
+  unsigned P = 32;
+  while (P < L.n[L.T]) P <<= 1;
+  L.P = P;
   return L;
 }
 
-// #{w_i >= k} over the 4 words: each unsigned compare is the carry of w - k
+// #{w_i >= k} over 8 words: each unsigned compare is the carry of w - k
 // (sub.cc: carry = no borrow = w >= k), summed with addc -- two integer-pipe
-// instructions per key instead of a compare, a select and a bit-combine.
-__device__ __forceinline__ unsigned count_ge(uint4 w, unsigned k) {
+// instructions per word instead of a compare, a select and a bit-combine.
+__device__ __forceinline__ unsigned count_ge8(const unsigned (&w)[8], unsigned k) {
   unsigned c, t;
   asm("{\n\t"
-      "sub.cc.u32 %1, %2, %6;\n\t"
+      "sub.cc.u32 %1, %2, %10;\n\t"
       "addc.u32 %0, 0, 0;\n\t"
-      "sub.cc.u32 %1, %3, %6;\n\t"
+      "sub.cc.u32 %1, %3, %10;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %4, %6;\n\t"
+      "sub.cc.u32 %1, %4, %10;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %5, %6;\n\t"
+      "sub.cc.u32 %1, %5, %10;\n\t"
+      "addc.u32 %0, %0, 0;\n\t"
+      "sub.cc.u32 %1, %6, %10;\n\t"
+      "addc.u32 %0, %0, 0;\n\t"
+      "sub.cc.u32 %1, %7, %10;\n\t"
+      "addc.u32 %0, %0, 0;\n\t"
+      "sub.cc.u32 %1, %8, %10;\n\t"
+      "addc.u32 %0, %0, 0;\n\t"
+      "sub.cc.u32 %1, %9, %10;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
       "}"
       : "=r"(c), "=&r"(t)
-      : "r"(w.x), "r"(w.y), "r"(w.z), "r"(w.w), "r"(k));
+      : "r"(w[0]), "r"(w[1]), "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7]), "r"(k));
   (void)t;  // scratch register of the asm (the differences are not needed)
   return c;
 }
@@ -95,9 +122,16 @@ __device__ __forceinline__ const unsigned* wide_addr(const unsigned* p, unsigned
   return r;
 }
 
+// 32 B of a sample level (L2-resident: default caching, 256-bit load)
+__device__ __forceinline__ void ld8(const unsigned* p, unsigned (&w)[8]) {
+  asm volatile("ld.global.nc.v8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+               : "l"(p));
+}
+
 // ---- index build: logical thread v writes 4 consecutive entries of one level,
-// or (the last 4 vectors) 4 words of the padded tail block T[i] = A[N16 + i]
-// (0xFFFFFFFF past N), so the final level's 64-B block loads need no bounds
+// or (the last 8 vectors) 4 words of the padded tail block T[i] = A[N32 + i]
+// (0xFFFFFFFF past N), so the final level's 128-B block loads need no bounds
 // checks (branch-free: all of a thread's block loads are in flight together).
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a, Ctx c) {
@@ -110,10 +144,10 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
     int k = 1;
 #pragma unroll 1
     while (k < a.L.T && v >= a.L.vecs_before[k + 1]) ++k;
-    const bool tail = v >= total && v < total + 4u;
+    const bool tail = v >= total && v < total + FAN / 4;
     const bool active = v < total || tail;
     const unsigned j0 = tail ? (v - total) * 4 : active ? (v - a.L.vecs_before[k]) * 4 : 0u;
-    unsigned stride = 1;
+    unsigned long long stride = 1;
 #pragma unroll 1
     for (int i = 0; i < k; ++i) stride *= FAN;
     unsigned w[4];
@@ -121,10 +155,10 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
     for (int q = 0; q < 4; ++q) {
       const unsigned j = j0 + q;
       if (tail) {
-        w[q] = a.L.N16 + j < a.N ? __ldg(a.A + a.L.N16 + j) : 0xFFFFFFFFu;
+        w[q] = a.L.N32 + j < a.N ? __ldg(a.A + a.L.N32 + j) : 0xFFFFFFFFu;
       } else {
         const unsigned long long src = (unsigned long long)j * stride;
-        w[q] = (active && j < a.L.n[k]) ? __ldcs(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[16^k j] (A: evict-first)
+        w[q] = (active && j < a.L.n[k]) ? __ldcs(a.A + src) : 0xFFFFFFFFu;  // L_k[j] = A[32^k j] (A: evict-first)
       }
     }
     const unsigned dst = tail ? a.L.tail_off + j0 : active ? a.L.off[k] + j0 : 0u;
@@ -137,102 +171,130 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
 }
 
 template <int V, int M>
-// Intra variants: 512-thread CTAs would hold 72 registers (1 CTA/SM); cap at 40.
-__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 3 : 4) bins_kernel(BsArgs a, Ctx c) {
+// Intra variants: 512-thread CTAs; cap registers so that three fit per SM.
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) bins_kernel(BsArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  extern __shared__ __align__(16) unsigned char bins_dyn[];
   Rep<V, M> rep(c);
   rep.init(mb);
+  using R = Rep<V, M>;
+  // ---- the table L_T in shared memory, once per physical CTA (every logical
+  // CTA of a persistent pair reuses it).  +LDS: each replica writes and reads
+  // its own copy; -LDS: one copy, every store compared.
+  unsigned* S = reinterpret_cast<unsigned*>(bins_dyn) + (R::SMDUP ? (unsigned)rep.r * a.plane : 0u);
+  {
+    const unsigned* LT = a.lev + a.L.off[a.L.T];
+    const unsigned nT = a.L.n[a.L.T];
+    const int nthr = BL;
+#pragma unroll 1
+    for (unsigned i = (unsigned)rep.ltid; i < a.L.P; i += nthr) {
+      const unsigned w = i < nT ? __ldg(LT + i) : 0xFFFFFFFFu;
+      if (rep.sts_ok1(w, i)) S[i] = w;
+    }
+  }
+  __syncthreads();
+  const unsigned P = a.L.P;
+  const int T = a.L.T;
   for (; rep.active(); rep.advance()) {
-    const unsigned j0 = ((unsigned)rep.lblock * BL + (unsigned)rep.ltid) * VEC;
-    unsigned key[VEC];
-    unsigned mask = 0;
-    if (j0 + VEC <= a.Q) {
-      uint4 w = __ldcs(reinterpret_cast<const uint4*>(a.q + j0));
-      key[0] = w.x; key[1] = w.y; key[2] = w.z; key[3] = w.w;
-      mask = 0xFu;
-    } else {
+#pragma unroll 1
+    for (unsigned it = 0; it < a.iters; ++it) {
+      const unsigned chunk = (unsigned)rep.lblock * a.iters + it;
+      if ((unsigned long long)chunk * CHUNK >= a.Q) break;  // CTA-uniform
+      const unsigned j0 = (chunk * BL + (unsigned)rep.ltid) * VEC;
+      unsigned key[VEC];
+      unsigned mask = 0;
+      if (j0 + VEC <= a.Q) {
+        uint2 w = __ldcs(reinterpret_cast<const uint2*>(a.q + j0));
+        key[0] = w.x; key[1] = w.y;
+        mask = 0x3u;
+      } else {
 #pragma unroll
-      for (int k = 0; k < VEC; ++k) {
-        const bool in = j0 + k < a.Q;
-        key[k] = in ? a.q[j0 + k] : 0u;
-        mask |= (in ? 1u : 0u) << k;
-      }
-    }
-    if constexpr (M == M_FAULT) {
-#pragma unroll
-      for (int k = 0; k < VEC; ++k) key[k] = rep.fault(SITE_LOAD, (long long)j0 + k, key[k]);
-    }
-    // Groups of 4 logical lanes descend together: for each of the group's 16
-    // queries the 4 members load one 16-B quarter of the same 64-B block, so a
-    // warp-wide load touches one cache line per query (1 L1 wavefront instead
-    // of 4).  Each lane tracks the block base of its OWN 4 queries and fetches the
-    // other members' bases by shuffle.
-    const int gm = rep.llane & 3;
-    const int g0 = rep.llane & ~3;
-    unsigned K[4][VEC];
-#pragma unroll
-    for (int i = 0; i < 4; ++i)
-#pragma unroll
-      for (int s = 0; s < VEC; ++s) K[i][s] = rep.lshfl_idx(key[s], g0 + i);
-    unsigned jj[VEC];
-#pragma unroll
-    for (int s = 0; s < VEC; ++s) jj[s] = a.N ? 1u : 0u;  // "block 0" of the top level
-    // one level: J <- 16 (max(J,1) - 1) + #{block < key}.  When J = 0 (key <= every
-    // entry) block 0 counts 0, so J stays 0 with no special case.
-    const unsigned* tailp = a.lev + a.L.tail_off - a.L.N16;  // tailp[N16 + i] = T[i]
-    // per-lane quarter pointers: element (base + 4 gm) of level P is Pq + 16 base bytes
-    auto level = [&](const unsigned* P, bool last) {
-      const unsigned* Pq = P + 4 * gm;
-      const unsigned* Tq = tailp + 4 * gm;
-#pragma unroll
-      for (int s = 0; s < VEC; ++s) {
-        const unsigned mybase = (max(jj[s], 1u) - 1u) * FAN;
-        unsigned packed = 0;
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const unsigned base = rep.lshfl_idx(mybase, g0 + i);
-          uint4 w;
-          if (!last) {  // sample levels: keep them L2-resident (default policy)
-            w = __ldg(reinterpret_cast<const uint4*>(wide_addr(Pq, base)));
-          } else {  // the caller's A: random 64-B blocks, evict-first; the ragged
-                    // last block comes from the padded copy (a block never straddles N16)
-            w = __ldcs(reinterpret_cast<const uint4*>(wide_addr(base >= a.L.N16 ? Tq : Pq, base)));
-          }
-          packed += count_ge(w, K[i][s]) << (8 * i);
+        for (int k = 0; k < VEC; ++k) {
+          const bool in = j0 + k < a.Q;
+          key[k] = in ? a.q[j0 + k] : 0u;
+          mask |= (in ? 1u : 0u) << k;
         }
-        packed += rep.lshfl_xor(packed, 1);  // sum the 4 quarters (bytes <= 16: no carries)
-        packed += rep.lshfl_xor(packed, 2);
-        jj[s] = mybase + FAN - ((packed >> (8 * gm)) & 0xFFu);  // #{block < key} = 16 - #{block >= key}
       }
-    };
-    for (int lv = a.L.T; lv >= 1; --lv) {  // padded sample levels: no bounds checks
       if constexpr (M == M_FAULT) {
-        if (lv == a.L.T - 1) {  // control-flow fault: a flipped block index, kept in range
 #pragma unroll
-          for (int s = 0; s < VEC; ++s) {
-            const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, jj[s]);
-            jj[s] = f > a.L.n[lv + 1] ? a.L.n[lv + 1] : f;
-          }
+        for (int k = 0; k < VEC; ++k) key[k] = rep.fault(SITE_LOAD, (long long)j0 + k, key[k]);
+      }
+      // ---- lower_bound in L_T: pos = #{S[i] < key} over the P (padded, sorted)
+      // entries, branch-free; the padding (0xFFFFFFFF) is never < key
+      unsigned jj[VEC];
+#pragma unroll
+      for (int s = 0; s < VEC; ++s) jj[s] = 0u;
+#pragma unroll 1
+      for (unsigned step = P >> 1; step >= 1u; step >>= 1) {
+#pragma unroll
+        for (int s = 0; s < VEC; ++s) {
+          unsigned w = S[jj[s] + step - 1u];
+          if constexpr (M == M_FAULT) w = rep.fault(SITE_SMEM, (long long)(jj[s] + step - 1u), w);
+          jj[s] += w < key[s] ? step : 0u;
         }
       }
-      level(a.lev + a.L.off[lv], false);
-    }
-    if constexpr (M == M_FAULT) {
-      if (a.L.T == 1) {
+      if constexpr (M == M_FAULT) {  // control-flow fault: a flipped block index, kept in range
 #pragma unroll
         for (int s = 0; s < VEC; ++s) {
           const unsigned f = rep.fault(SITE_COMPUTE, (long long)j0 + s, jj[s]);
-          jj[s] = f > a.L.n[1] ? a.L.n[1] : f;
+          jj[s] = f > a.L.n[T] ? a.L.n[T] : f;
         }
       }
+      // ---- descent: groups of 4 logical lanes, for each of the group's 8
+      // queries the 4 members load one 32-B quarter of the same 128-B block (one
+      // L1 wavefront per query and level).  Each lane tracks the block base of
+      // its OWN 2 queries and fetches the other members' bases by shuffle.
+      const int gm = rep.llane & 3;
+      const int g0 = rep.llane & ~3;
+      unsigned K[4][VEC];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int s = 0; s < VEC; ++s) K[i][s] = rep.lshfl_idx(key[s], g0 + i);
+      const unsigned* tailp = a.lev + a.L.tail_off - a.L.N32;  // tailp[N32 + i] = T[i]
+      // one level: J <- 32 (max(J,1) - 1) + #{block < key}.  When J = 0 (key <=
+      // every entry) block 0 counts 0, so J stays 0 with no special case.
+      auto level = [&](const unsigned* Pl, bool last) {
+        const unsigned* Pq = Pl + 8 * gm;
+        const unsigned* Tq = tailp + 8 * gm;
+#pragma unroll
+        for (int s = 0; s < VEC; ++s) {
+          const unsigned mybase = (max(jj[s], 1u) - 1u) * FAN;
+          unsigned packed = 0;
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const unsigned base = rep.lshfl_idx(mybase, g0 + i);
+            unsigned w[8];
+            if (!last) {  // sample levels: keep them L2-resident (default policy)
+              ld8(wide_addr(Pq, base), w);
+            } else {      // the caller's A: random 128-B blocks, evict-first; the ragged
+                          // last block comes from the padded copy (a block never straddles N32)
+              const unsigned* p = wide_addr(base >= a.L.N32 ? Tq : Pq, base);
+              if (a.a32 || base >= a.L.N32) {
+                ldcs8(p, w);
+              } else {
+                const uint4 u0 = ldcs4(p), u1 = ldcs4(p + 4);
+                w[0] = u0.x; w[1] = u0.y; w[2] = u0.z; w[3] = u0.w;
+                w[4] = u1.x; w[5] = u1.y; w[6] = u1.z; w[7] = u1.w;
+              }
+            }
+            packed += count_ge8(w, K[i][s]) << (8 * i);
+          }
+          packed += rep.lshfl_xor(packed, 1);  // sum the 4 quarters (bytes <= 32: no carries)
+          packed += rep.lshfl_xor(packed, 2);
+          jj[s] = mybase + FAN - ((packed >> (8 * gm)) & 0xFFu);  // #{block < key} = 32 - #{block >= key}
+        }
+      };
+#pragma unroll 1
+      for (int lv = T - 1; lv >= 1; --lv) level(a.lev + a.L.off[lv], false);  // padded: no bounds checks
+      level(a.A, true);  // the caller's A
+      rep.template commit<VEC, 0>(mask, j0, jj, a.Q, [&](unsigned i, unsigned m, const unsigned* w) {
+        if (m == 0x3u) __stcs(reinterpret_cast<uint2*>(a.idx + i), make_uint2(w[0], w[1]));
+        else
+          for (int k = 0; k < VEC; ++k)
+            if ((m >> k) & 1u) a.idx[i + k] = w[k];
+      });
     }
-    level(a.A, true);  // the caller's A
-    rep.template commit<VEC, 0>(mask, j0, jj, a.Q, [&](unsigned i, unsigned m, const unsigned* w) {
-      if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.idx + i), make_uint4(w[0], w[1], w[2], w[3]));
-      else
-        for (int k = 0; k < VEC; ++k)
-          if ((m >> k) & 1u) a.idx[i + k] = w[k];
-    });
   }
   rep.finish();
 }
@@ -252,7 +314,7 @@ size_t binarysearch_scratch(int64_t, const int64_t* dims) {
   Levels L = make_levels((unsigned)dims[0]);
   size_t words = 0;
   for (int k = 1; k <= L.T; ++k) words += L.padded[k];
-  return (words + 16) * 4 + 64;  // + the padded tail block
+  return (words + FAN) * 4 + 128;  // + the padded tail block
 }
 int binarysearch_inter_warps(int64_t, const int64_t*) { return BL / 32; }
 
@@ -266,9 +328,14 @@ int binarysearch_run(Launch& L) {
   a.N = N;
   a.Q = Q;
   a.L = make_levels(N);
-  a.top_iters = 0;
-  const unsigned Gi = (a.L.vecs_before[a.L.T + 1] + 4 + BL - 1) / BL;
-  const unsigned G = (Q + BL * VEC - 1) / (BL * VEC);
+  a.plane = a.L.P + 1u;
+  a.a32 = ((uintptr_t)a.A % 32) == 0 ? 1u : 0u;
+  const unsigned Gi = (a.L.vecs_before[a.L.T + 1] + FAN / 4 + BL - 1) / BL;
+  const unsigned chunks = (Q + CHUNK - 1) / CHUNK;
+  // about 8 waves of logical CTAs: the table copy is amortised over a.iters chunks
+  a.iters = (chunks + 148u * 8u - 1u) / (148u * 8u);
+  if (a.iters == 0) a.iters = 1;
+  const unsigned G = (chunks + a.iters - 1) / a.iters;
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     int rc = RMT_OK;
@@ -276,7 +343,8 @@ int binarysearch_run(Launch& L) {
       rc = launch_std<V>(L, bins_index_kernel<V, M>, bins_index_kernel<V_NONE, M_NORMAL>, Gi, BL, 0, a,
                          "binarysearch/index");
     if (rc) return rc;
-    return launch_std<V>(L, bins_kernel<V, M>, bins_kernel<V_NONE, M_NORMAL>, G, BL, 0, a, "binarysearch",
+    const size_t smem = (size_t)(Rep<V, M>::SMDUP ? 2u * a.plane : a.L.P) * 4u;
+    return launch_std<V>(L, bins_kernel<V, M>, bins_kernel<V_NONE, M_NORMAL>, G, BL, smem, a, "binarysearch",
                          /*mult_inter=*/2);
   });
 }

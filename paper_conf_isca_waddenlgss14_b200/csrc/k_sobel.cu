@@ -6,7 +6,9 @@
 //
 // Logical thread = 4 horizontally adjacent pixels (16 B) x a vertical strip of
 // RY rows with a rolling 3-row register window (each input row is read once
-// per thread; the two halo pixels come from L1).  Arithmetic is SIMD within a
+// per thread; the two halo pixels come from L1).  Interior threads (all but the
+// image's outer frame) run a copy of the body without bounds checks or border
+// selects.  Arithmetic is SIMD within a
 // register: two channels per 32-bit word in biased 16-bit lanes (no borrows),
 // separable Sobel (vertical smooth / difference per column, then horizontal).
 // isqrt: floor(sqrt(s)/2) = isqrt(s/4); computed as floor(sqrt_approx(s/4 + 1/8))
@@ -20,7 +22,7 @@ namespace rmt {
 namespace {
 
 constexpr int BL = 256;
-constexpr int RY = 32;  // output rows per thread
+constexpr int RY = 30;  // output rows per thread (a multiple of 3: the window rotates by renaming)
 
 struct SobArgs {
   const unsigned* I;
@@ -64,17 +66,17 @@ __device__ __forceinline__ f2_t fma2(f2_t a, f2_t b, f2_t c) {
 // Two channels at once: gw, yw hold two biased 16-bit lanes (value + 1024) of
 // Gx and Gy.  Returns two words 2^23 + floor(sqrt_approx(s/4 + 1/8)) (as fp32
 // bits; the low 10 bits hold the unsaturated output of the low / high lane
-// channel).  s = Gx^2 + Gy^2 < 2^21 is exact in fp32 (exact: see the header).  The 16-bit lanes
-// become floats through the 2^23 magic (PRMT + FADD2), no conversion pipe.
+// channel).  The 16-bit lanes become floats F = 2^23 + v through the magic
+// exponent (one PRMT each, no conversion pipe); d = F/2 - (2^22 + 512) = Gx/2
+// is one exact FFMA2, and s/4 + 1/8 = d^2 + (e^2 + 1/8) two more (every
+// intermediate is a multiple of 1/8 below 2^19: exact in fp32).
 __device__ __forceinline__ void sobel_mag2(unsigned gw, unsigned yw, unsigned& out_lo, unsigned& out_hi) {
   const unsigned MAG = 0x4B000000u;
-  const f2_t gx = add2(f2(__byte_perm(gw, MAG, 0x7610), __byte_perm(gw, MAG, 0x7632)),
-                       f2(__float_as_uint(-8389632.0f), __float_as_uint(-8389632.0f)));  // -(2^23 + 1024)
-  const f2_t gy = add2(f2(__byte_perm(yw, MAG, 0x7610), __byte_perm(yw, MAG, 0x7632)),
-                       f2(__float_as_uint(-8389632.0f), __float_as_uint(-8389632.0f)));
-  const f2_t ss = fma2(gx, gx, mul2(gy, gy));
-  const f2_t f = fma2(ss, f2(__float_as_uint(0.25f), __float_as_uint(0.25f)),
-                      f2(__float_as_uint(0.125f), __float_as_uint(0.125f)));  // s/4 + 1/8, exact
+  const f2_t half = f2(__float_as_uint(0.5f), __float_as_uint(0.5f));
+  const f2_t nb = f2(__float_as_uint(-4194816.0f), __float_as_uint(-4194816.0f));  // -(2^23 + 1024) / 2
+  const f2_t d = fma2(f2(__byte_perm(gw, MAG, 0x7610), __byte_perm(gw, MAG, 0x7632)), half, nb);  // Gx / 2
+  const f2_t e = fma2(f2(__byte_perm(yw, MAG, 0x7610), __byte_perm(yw, MAG, 0x7632)), half, nb);  // Gy / 2
+  const f2_t f = fma2(d, d, fma2(e, e, f2(__float_as_uint(0.125f), __float_as_uint(0.125f))));   // s/4 + 1/8
   unsigned f0, f1;
   f2_split(f, f0, f1);
   const float r0 = sqrt_approx(__uint_as_float(f0));
@@ -89,18 +91,27 @@ struct Row {
   unsigned lo[6], hi[6];  // columns x0-1 .. x0+4, channels (0,2) and (1,3)
 };
 
-// Raw words of one input row (columns x0-1 .. x0+4); zeros outside the image.
-template <int V, int M>
-__device__ __forceinline__ void load_raw(const Rep<V, M>& rep, const SobArgs& a, int y, unsigned x0, bool active,
-                                         unsigned (&p)[6]) {
-#pragma unroll
-  for (int k = 0; k < 6; ++k) p[k] = 0u;
-  if (active && y >= 0 && y < (int)a.H) {
-    const unsigned* row = a.I + (size_t)y * a.W;
-    uint4 c = __ldg(reinterpret_cast<const uint4*>(row + x0));
+// Raw words of one input row (columns x0-1 .. x0+4).  IN (interior thread):
+// the row and both halo columns are inside the image, no checks; otherwise
+// zeros outside the image.
+template <bool IN>
+__device__ __forceinline__ void load_raw(const SobArgs& a, int y, unsigned x0, bool active, unsigned (&p)[6]) {
+  if constexpr (IN) {
+    const unsigned* row = a.I + (size_t)y * a.W + x0;
+    uint4 c = __ldg(reinterpret_cast<const uint4*>(row));
+    p[0] = __ldg(row - 1);
     p[1] = c.x; p[2] = c.y; p[3] = c.z; p[4] = c.w;
-    if (x0 >= 1) p[0] = __ldg(row + x0 - 1);
-    if (x0 + 4 < a.W) p[5] = __ldg(row + x0 + 4);
+    p[5] = __ldg(row + 4);
+  } else {
+#pragma unroll
+    for (int k = 0; k < 6; ++k) p[k] = 0u;
+    if (active && y >= 0 && y < (int)a.H) {
+      const unsigned* row = a.I + (size_t)y * a.W;
+      uint4 c = __ldg(reinterpret_cast<const uint4*>(row + x0));
+      p[1] = c.x; p[2] = c.y; p[3] = c.z; p[4] = c.w;
+      if (x0 >= 1) p[0] = __ldg(row + x0 - 1);
+      if (x0 + 4 < a.W) p[5] = __ldg(row + x0 + 4);
+    }
   }
 }
 
@@ -125,8 +136,13 @@ __device__ __forceinline__ void unpack_row(const Rep<V, M>& rep, const SobArgs& 
   }
 }
 
+template <bool B>
+struct BoolC {
+  static constexpr bool value = B;
+};
+
 template <int V, int M>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP) sobel_kernel(SobArgs a, Ctx c) {
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) sobel_kernel(SobArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);
@@ -135,68 +151,86 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) sobel_kernel(SobArgs a, Ctx
     const unsigned x0 = (bx * BL + (unsigned)rep.ltid) * 4;
     const bool active = x0 < a.W;
     const int y0 = (int)(by * RY);
-    unsigned xin = 0;  // interior columns among this thread's 4 pixels (loop-invariant)
+    // Interior thread: its 4 pixels and both halo columns are interior columns,
+    // and every row it reads (y0-1 .. y0+RY, plus the last prefetch y0+RY+1) is
+    // inside the image: no bounds checks, no border selects.  Most warps.
+    // Warp-uniform (commits are warp-collective: a warp never splits between
+    // the two bodies).
+    const bool interior =
+        __all_sync(0xFFFFFFFFu, x0 >= 4u && x0 + 8u <= a.W && y0 >= 1 && (unsigned)y0 + RY + 2u <= a.H);
+    auto body = [&](auto in_tag) {
+      constexpr bool IN = decltype(in_tag)::value;
+      unsigned xin = 0xFu;  // interior columns among this thread's 4 pixels
+      if constexpr (!IN) {
+        xin = 0u;
 #pragma unroll
-    for (int p = 0; p < 4; ++p) xin |= ((x0 + p >= 1 && x0 + p < a.W - 1) ? 1u : 0u) << p;
-    // one output row from the window (t = y-1, m = y, b = y+1)
-    auto row_out = [&](int y, const Row& t, const Row& m, const Row& b) {
-      unsigned vs_lo[6], vs_hi[6], vd_lo[6], vd_hi[6];
-#pragma unroll
-      for (int k = 0; k < 6; ++k) {
-        vs_lo[k] = t.lo[k] + 2u * m.lo[k] + b.lo[k];   // <= 1020 per lane
-        vs_hi[k] = t.hi[k] + 2u * m.hi[k] + b.hi[k];
-        vd_lo[k] = t.lo[k] + 0x01000100u - b.lo[k];    // 256 + (top - bot)
-        vd_hi[k] = t.hi[k] + 0x01000100u - b.hi[k];
+        for (int p = 0; p < 4; ++p) xin |= ((x0 + p >= 1 && x0 + p < a.W - 1) ? 1u : 0u) << p;
       }
-      const bool yin = y >= 1 && y < (int)a.H - 1;
-      unsigned out[4];
+      // one output row from the window (t = y-1, m = y, b = y+1)
+      auto row_out = [&](int y, const Row& t, const Row& m, const Row& b) {
+        unsigned vs_lo[6], vs_hi[6], vd_lo[6], vd_hi[6];
 #pragma unroll
-      for (int p = 0; p < 4; ++p) {
-        const int w = p + 1;
-        // biased by 1024 per 16-bit lane
-        unsigned gx_lo = vd_lo[w - 1] + 2u * vd_lo[w] + vd_lo[w + 1];
-        const unsigned gx_hi = vd_hi[w - 1] + 2u * vd_hi[w] + vd_hi[w + 1];
-        const unsigned gy_lo = vs_lo[w - 1] + 0x04000400u - vs_lo[w + 1];
-        const unsigned gy_hi = vs_hi[w - 1] + 0x04000400u - vs_hi[w + 1];
-        if constexpr (M == M_FAULT) gx_lo = rep.fault(SITE_COMPUTE, (long long)y * a.W + x0 + p, gx_lo);
-        unsigned m0, m2, m1, m3;
-        sobel_mag2(gx_lo, gy_lo, m0, m2);  // channels 0, 2
-        sobel_mag2(gx_hi, gy_hi, m1, m3);  // channels 1, 3
-        // two channels per 16-bit lane pair, saturated with one VIMNMX.U16x2 each
-        const unsigned h01 = __vminu2(__byte_perm(m0, m1, 0x5410), 0x00FF00FFu);
-        const unsigned h23 = __vminu2(__byte_perm(m2, m3, 0x5410), 0x00FF00FFu);
-        const unsigned px = __byte_perm(h01, h23, 0x6420);
-        out[p] = (yin && ((xin >> p) & 1u)) ? px : 0u;
-      }
-      const unsigned mask = (active && y < (int)a.H) ? 0xFu : 0u;
-      rep.template commit<4, 0>(mask, (unsigned)y * a.W + x0, out, a.H * a.W,
-                                [&](unsigned idx, unsigned mm, const unsigned* w) {
-                                  if (mm == 0xFu)
-                                    __stcs(reinterpret_cast<uint4*>(a.O + idx), make_uint4(w[0], w[1], w[2], w[3]));
-                                  else
-                                    for (int k = 0; k < 4; ++k)
-                                      if ((mm >> k) & 1u) a.O[idx + k] = w[k];
-                                });
-    };
-    // rolling 3-row window; the raw words of the row after next are in flight
-    // while the current row is filtered (one row of prefetch distance)
-    Row top, mid, bot;
-    unsigned raw[6], nxt[6];
-    load_raw(rep, a, y0 - 1, x0, active, raw);
-    unpack_row(rep, a, y0 - 1, x0, raw, top);
-    load_raw(rep, a, y0, x0, active, raw);
-    load_raw(rep, a, y0 + 1, x0, active, nxt);
-    unpack_row(rep, a, y0, x0, raw, mid);
+        for (int k = 0; k < 6; ++k) {
+          vs_lo[k] = t.lo[k] + 2u * m.lo[k] + b.lo[k];   // <= 1020 per lane
+          vs_hi[k] = t.hi[k] + 2u * m.hi[k] + b.hi[k];
+          vd_lo[k] = t.lo[k] + 0x01000100u - b.lo[k];    // 256 + (top - bot)
+          vd_hi[k] = t.hi[k] + 0x01000100u - b.hi[k];
+        }
+        bool yin = true;
+        if constexpr (!IN) yin = y >= 1 && y < (int)a.H - 1;
+        unsigned out[4];
+#pragma unroll
+        for (int p = 0; p < 4; ++p) {
+          const int w = p + 1;
+          // biased by 1024 per 16-bit lane
+          unsigned gx_lo = vd_lo[w - 1] + 2u * vd_lo[w] + vd_lo[w + 1];
+          const unsigned gx_hi = vd_hi[w - 1] + 2u * vd_hi[w] + vd_hi[w + 1];
+          const unsigned gy_lo = vs_lo[w - 1] + 0x04000400u - vs_lo[w + 1];
+          const unsigned gy_hi = vs_hi[w - 1] + 0x04000400u - vs_hi[w + 1];
+          if constexpr (M == M_FAULT) gx_lo = rep.fault(SITE_COMPUTE, (long long)y * a.W + x0 + p, gx_lo);
+          unsigned m0, m2, m1, m3;
+          sobel_mag2(gx_lo, gy_lo, m0, m2);  // channels 0, 2
+          sobel_mag2(gx_hi, gy_hi, m1, m3);  // channels 1, 3
+          // two channels per 16-bit lane pair, saturated with one VIMNMX.U16x2 each
+          const unsigned h01 = __vminu2(__byte_perm(m0, m1, 0x5410), 0x00FF00FFu);
+          const unsigned h23 = __vminu2(__byte_perm(m2, m3, 0x5410), 0x00FF00FFu);
+          const unsigned px = __byte_perm(h01, h23, 0x6420);
+          if constexpr (IN) out[p] = px;
+          else out[p] = (yin && ((xin >> p) & 1u)) ? px : 0u;
+        }
+        unsigned mask = 0xFu;
+        if constexpr (!IN) mask = (active && y < (int)a.H) ? 0xFu : 0u;
+        rep.template commit<4, 0>(mask, (unsigned)y * a.W + x0, out, a.H * a.W,
+                                  [&](unsigned idx, unsigned mm, const unsigned* w) {
+                                    if (mm == 0xFu)
+                                      __stcs(reinterpret_cast<uint4*>(a.O + idx), make_uint4(w[0], w[1], w[2], w[3]));
+                                    else
+                                      for (int k = 0; k < 4; ++k)
+                                        if ((mm >> k) & 1u) a.O[idx + k] = w[k];
+                                  });
+      };
+      // rolling 3-row window; the raw words of the row after next are in flight
+      // while the current row is filtered (one row of prefetch distance)
+      Row top, mid, bot;
+      unsigned raw[6], nxt[6];
+      load_raw<IN>(a, y0 - 1, x0, active, raw);
+      unpack_row(rep, a, y0 - 1, x0, raw, top);
+      load_raw<IN>(a, y0, x0, active, raw);
+      load_raw<IN>(a, y0 + 1, x0, active, nxt);
+      unpack_row(rep, a, y0, x0, raw, mid);
 #pragma unroll 1
-    for (int y = y0; y < y0 + RY; ++y) {
+      for (int y = y0; y < y0 + RY; ++y) {
 #pragma unroll
-      for (int k = 0; k < 6; ++k) raw[k] = nxt[k];
-      load_raw(rep, a, y + 2, x0, active, nxt);
-      unpack_row(rep, a, y + 1, x0, raw, bot);
-      row_out(y, top, mid, bot);
-      top = mid;
-      mid = bot;
-    }
+        for (int k = 0; k < 6; ++k) raw[k] = nxt[k];
+        load_raw<IN>(a, y + 2, x0, active, nxt);
+        unpack_row(rep, a, y + 1, x0, raw, bot);
+        row_out(y, top, mid, bot);
+        top = mid;
+        mid = bot;
+      }
+    };
+    if (interior) body(BoolC<true>{});
+    else body(BoolC<false>{});
   }
   rep.finish();
 }

@@ -24,7 +24,10 @@ pytestmark = pytest.mark.gpu
 CAMPAIGN = [
     (lambda: BlackScholes(5000), {"load": lambda c: c.n, "compute": lambda c: c.n, "store_val": lambda c: c.n,
                                   "store_addr": lambda c: c.n}),
+    # BinarySearch SMEM = an entry of the shared-memory table L_1 = A[32 j] (2048
+    # entries at N = 2^16), flipped where the binary search reads it
     (lambda: BinarySearch(1 << 16, 4000), {"load": lambda c: c.Q, "compute": lambda c: c.Q,
+                                           "smem": lambda c: (c.N + 31) // 32,
                                            "store_val": lambda c: c.Q, "store_addr": lambda c: c.Q}),
     (lambda: FWT(1 << 14), {"load": lambda c: c.n, "compute": lambda c: c.n, "smem": lambda c: c.n,
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),
@@ -41,7 +44,7 @@ CAMPAIGN = [
                                  "smem": lambda c: 1184 * 8, "store_val": lambda c: 1, "store_addr": lambda c: 1}),
     (lambda: Transpose(96, 160), {"load": lambda c: c.n, "smem": lambda c: c.n, "store_val": lambda c: c.n,
                                   "store_addr": lambda c: c.n}),
-    (lambda: Sobel(40, 132), {"load": lambda c: c.n, "compute": lambda c: c.n, "store_val": lambda c: c.n,
+    (lambda: Sobel(72, 132), {"load": lambda c: c.n, "compute": lambda c: c.n, "store_val": lambda c: c.n,
                               "store_addr": lambda c: c.n}),
     (lambda: DCT(32, 264), {"load": lambda c: c.n, "compute": lambda c: c.n, "smem": lambda c: c.n,
                             "store_val": lambda c: c.n, "store_addr": lambda c: c.n}),

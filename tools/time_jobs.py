@@ -1,5 +1,5 @@
 """Median device time per (kernel, variant) for a bench config (quick look).
-usage: time_jobs.py CONFIG [REPS] [VARIANTS]"""
+usage: time_jobs.py CONFIG [REPS] [VARIANTS]   (RMT_KERNELS=a,b: only those kernels)"""
 import sys, os, statistics
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -10,7 +10,10 @@ if os.environ.get("RMT_ABL"):  # full | nocomm | inflate
     rmt.set_ablation(os.environ["RMT_ABL"])
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 variants = sys.argv[3].split(",") if len(sys.argv) > 3 else ["none", "intra_smem", "intra_reg", "inter_group", "inter_cluster", "intra_nolds", "dup_kernel"]
+only = os.environ.get("RMT_KERNELS", "").split(",") if os.environ.get("RMT_KERNELS") else None
 for j in workloads.config_jobs(cfg):
+    if only and j.kernel not in only:
+        continue
     b = j.device_buffers()
     base = None
     for v in variants:
