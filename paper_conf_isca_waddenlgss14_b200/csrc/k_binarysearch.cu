@@ -21,7 +21,8 @@
 // 128 B as at 64 B, and one 128-B line per query and level is also the L1 data
 // pipe's unit (the 64-B design spent a wavefront per 64 B and 7 levels).
 // Group of 4 logical lanes per query, one 32-B load each (LDG.256); logical
-// thread = 2 interleaved queries, one 8-B vector commit of idx.
+// thread = 2 interleaved queries, one 8-B vector commit of idx; every lane of a
+// group loads the group's 8 keys with one 256-bit load.
 #include <string.h>
 
 #include "rmt_host.cuh"
@@ -57,6 +58,7 @@ struct BsArgs {
   unsigned plane;   // +LDS: replica r's table copy starts at word r * plane (P + 1: the
                     // pair's two copies of an entry sit in different banks)
   unsigned a32;     // A is 32-B aligned (256-bit block loads)
+  unsigned q32;     // q is 32-B aligned (256-bit key loads)
   Levels L;
 };
 
@@ -114,6 +116,12 @@ __device__ __forceinline__ unsigned count_ge8(const unsigned (&w)[8], unsigned k
   return c;
 }
 
+// Shared-memory table swizzle: entry i lives at word i ^ ((i >> 6) & 31).  The
+// binary search's probes at step >= 32 are pos + step - 1 with pos a multiple
+// of 2 step -- all in ONE bank unswizzled (a 32-way conflict at step 32); with
+// the row index folded into the bank they spread over distinct banks.
+__device__ __forceinline__ unsigned tsw(unsigned i) { return i ^ ((i >> 6) & 31u); }
+
 // p + i (u32 elements) as one wide multiply-add (keeps nvcc from widening the
 // index sum with carries)
 __device__ __forceinline__ const unsigned* wide_addr(const unsigned* p, unsigned i) {
@@ -170,9 +178,12 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
   rep.finish();
 }
 
+#ifndef BINS_MINB
+#define BINS_MINB 4
+#endif
 template <int V, int M>
-// Intra variants: 512-thread CTAs; cap registers so that three fit per SM.
-__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) bins_kernel(BsArgs a, Ctx c) {
+// Registers capped at 64 (4 CTAs of 256 / 2 of 512 threads per SM).
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? BINS_MINB / 2 : BINS_MINB) bins_kernel(BsArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   extern __shared__ __align__(16) unsigned char bins_dyn[];
   Rep<V, M> rep(c);
@@ -189,7 +200,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) 
 #pragma unroll 1
     for (unsigned i = (unsigned)rep.ltid; i < a.L.P; i += nthr) {
       const unsigned w = i < nT ? __ldg(LT + i) : 0xFFFFFFFFu;
-      if (rep.sts_ok1(w, i)) S[i] = w;
+      if (rep.sts_ok1(w, i)) S[tsw(i)] = w;
     }
   }
   __syncthreads();
@@ -201,26 +212,45 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) 
       const unsigned chunk = (unsigned)rep.lblock * a.iters + it;
       if ((unsigned long long)chunk * CHUNK >= a.Q) break;  // CTA-uniform
       const unsigned j0 = (chunk * BL + (unsigned)rep.ltid) * VEC;
-      unsigned key[VEC];
-      unsigned mask = 0;
-      if (j0 + VEC <= a.Q) {
-        uint2 w = __ldcs(reinterpret_cast<const uint2*>(a.q + j0));
-        key[0] = w.x; key[1] = w.y;
-        mask = 0x3u;
-      } else {
+      // Groups of 4 logical lanes descend together (below); every lane loads the
+      // group's 8 keys (4 members x VEC, contiguous and 32-B aligned: one 256-bit
+      // load, the 4 lanes' identical requests served by the same lines) --
+      // K[i][s] = key s of member i, no shuffles.
+      const int gm = rep.llane & 3;
+      const int g0 = rep.llane & ~3;
+      const unsigned jg = j0 - (unsigned)gm * VEC;  // the group's first query
+      unsigned K[4][VEC];
+      {
+        unsigned w[8];
+        if (jg + 4 * VEC <= a.Q && a.q32) {
+          ldcs8(a.q + jg, w);
+        } else {
 #pragma unroll
-        for (int k = 0; k < VEC; ++k) {
-          const bool in = j0 + k < a.Q;
-          key[k] = in ? a.q[j0 + k] : 0u;
-          mask |= (in ? 1u : 0u) << k;
+          for (int k = 0; k < 8; ++k) w[k] = jg + k < a.Q ? __ldcs(a.q + jg + k) : 0u;
         }
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int s = 0; s < VEC; ++s) K[i][s] = w[i * VEC + s];
       }
       if constexpr (M == M_FAULT) {
 #pragma unroll
-        for (int k = 0; k < VEC; ++k) key[k] = rep.fault(SITE_LOAD, (long long)j0 + k, key[k]);
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int s = 0; s < VEC; ++s) K[i][s] = rep.fault(SITE_LOAD, (long long)jg + i * VEC + s, K[i][s]);
+      }
+      unsigned key[VEC];
+      unsigned mask = 0;
+#pragma unroll
+      for (int s = 0; s < VEC; ++s) {
+        key[s] = gm == 0 ? K[0][s] : gm == 1 ? K[1][s] : gm == 2 ? K[2][s] : K[3][s];
+        mask |= (j0 + s < a.Q ? 1u : 0u) << s;
       }
       // ---- lower_bound in L_T: pos = #{S[i] < key} over the P (padded, sorted)
-      // entries, branch-free; the padding (0xFFFFFFFF) is never < key
+      // entries, branch-free; the padding (0xFFFFFFFF) is never < key.  The
+      // halving steps leave pos in [0, P-1] with S[0, pos) < key <= S[pos + 1]
+      // (when that exists); one last compare of S[pos] decides pos vs pos + 1
+      // (pos = P when every entry is < key: n_T = P, no padding).
       unsigned jj[VEC];
 #pragma unroll
       for (int s = 0; s < VEC; ++s) jj[s] = 0u;
@@ -228,10 +258,16 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) 
       for (unsigned step = P >> 1; step >= 1u; step >>= 1) {
 #pragma unroll
         for (int s = 0; s < VEC; ++s) {
-          unsigned w = S[jj[s] + step - 1u];
+          unsigned w = S[tsw(jj[s] + step - 1u)];
           if constexpr (M == M_FAULT) w = rep.fault(SITE_SMEM, (long long)(jj[s] + step - 1u), w);
           jj[s] += w < key[s] ? step : 0u;
         }
+      }
+#pragma unroll
+      for (int s = 0; s < VEC; ++s) {
+        unsigned w = S[tsw(jj[s])];
+        if constexpr (M == M_FAULT) w = rep.fault(SITE_SMEM, (long long)jj[s], w);
+        jj[s] += w < key[s] ? 1u : 0u;
       }
       if constexpr (M == M_FAULT) {  // control-flow fault: a flipped block index, kept in range
 #pragma unroll
@@ -240,17 +276,12 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) 
           jj[s] = f > a.L.n[T] ? a.L.n[T] : f;
         }
       }
-      // ---- descent: groups of 4 logical lanes, for each of the group's 8
-      // queries the 4 members load one 32-B quarter of the same 128-B block (one
-      // L1 wavefront per query and level).  Each lane tracks the block base of
-      // its OWN 2 queries and fetches the other members' bases by shuffle.
-      const int gm = rep.llane & 3;
-      const int g0 = rep.llane & ~3;
-      unsigned K[4][VEC];
-#pragma unroll
-      for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int s = 0; s < VEC; ++s) K[i][s] = rep.lshfl_idx(key[s], g0 + i);
+      // ---- descent: for each of the group's 8 queries the 4 members load one
+      // 32-B quarter of the same 128-B block (one L1 wavefront per query and
+      // level).  Each lane tracks the block base of its OWN 2 queries and
+      // fetches the other members' bases by shuffle.  (Tracking all 8 positions
+      // in every lane instead saves the base shuffles but costs more
+      // instructions: measured 0.452 -> 0.498 ms at Q = 2^24, latency-bound.)
       const unsigned* tailp = a.lev + a.L.tail_off - a.L.N32;  // tailp[N32 + i] = T[i]
       // one level: J <- 32 (max(J,1) - 1) + #{block < key}.  When J = 0 (key <=
       // every entry) block 0 counts 0, so J stays 0 with no special case.
@@ -330,6 +361,7 @@ int binarysearch_run(Launch& L) {
   a.L = make_levels(N);
   a.plane = a.L.P + 1u;
   a.a32 = ((uintptr_t)a.A % 32) == 0 ? 1u : 0u;
+  a.q32 = ((uintptr_t)a.q % 32) == 0 ? 1u : 0u;
   const unsigned Gi = (a.L.vecs_before[a.L.T + 1] + FAN / 4 + BL - 1) / BL;
   const unsigned chunks = (Q + CHUNK - 1) / CHUNK;
   // about 8 waves of logical CTAs: the table copy is amortised over a.iters chunks

@@ -306,12 +306,15 @@ struct Rep {
   unsigned pend;  // inter: records not yet published (producer) / freed (consumer)
   unsigned region, epoch;
   unsigned rdy_hi;  // inter consumer: records below this are known to be published (group flags)
+  unsigned pempty;  // inter producer: bit l = pending record (j - pend + l) is empty (COND, no lane stores)
+  unsigned cempty, cbase;  // inter consumer: emptiness bits of the group starting at record cbase
   unsigned* mbox;  // intra_smem: this warp's mailbox
   unsigned tr_id;  // RMT_TRACE: trace row (inter ticket)
   unsigned cl_pay, cl_full;  // inter_cluster: this warp's mailbox / flags in the consumer CTA (shared::cluster)
 
   __device__ __forceinline__ explicit Rep(const Ctx& ctx)
-      : c(ctx), j(0), lstride(0), nerr(0), pend(0), region(0), epoch(0), rdy_hi(0), mbox(nullptr), cl_pay(0),
+      : c(ctx), j(0), lstride(0), nerr(0), pend(0), region(0), epoch(0), rdy_hi(0), pempty(0), cempty(0), cbase(0),
+        mbox(nullptr), cl_pay(0),
         cl_full(0) {}
 
   // ---- logical-CTA loop.  Kernel bodies are written
@@ -467,6 +470,10 @@ struct Rep {
         // consumer that acquired flag[first] then frees the other slots only
         // after their flag stores, never before one lands late and leaves a
         // stale "full" flag (found by tests/model/ring_model.cpp)
+        // Flag value = distance to the group's end | emptiness << 8: an EMPTY
+        // record (a COND commit where no lane stores) carries no payload, the
+        // consumer learns it from the flag (group flags: the first record's flag
+        // holds the whole group's emptiness bits).
         if constexpr (GROUP)
           if ((unsigned)lane - 1u < pend - 1u) st_relaxed(c.flags + slot_index(first + lane), pend - lane);
 #if RMT_PUB_FENCE_SC
@@ -476,10 +483,11 @@ struct Rep {
 #endif
         __syncwarp();
         if constexpr (GROUP) {
-          if (lane == 0) st_relaxed(c.flags + slot_index(first), pend);
+          if (lane == 0) st_relaxed(c.flags + slot_index(first), pend | (pempty << 8));
         } else {
-          if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), 1u);
+          if ((unsigned)lane < pend) st_relaxed(c.flags + slot_index(first + lane), 1u | (((pempty >> lane) & 1u) << 8));
         }
+        pempty = 0u;
       } else {
         __syncwarp();
 #if RMT_FREE_RELAXED
@@ -709,12 +717,16 @@ struct Rep {
       unsigned key;
       if constexpr (NW == 1) key = mask ? idx : 0xffffffffu;
       else key = mask ? (idx ^ (mask << 28)) : 0xffffffffu;
+      unsigned key0 = 0xffffffffu;  // the key of a lane that stores nothing
       if constexpr (STRESS) {
         // (pair, warp, sequence) tag folded into the key on both sides: a record
         // consumed out of order, twice, or from another pair's/warp's ring fails
         // the compare (counted in err)
         const unsigned tag = mix32(((unsigned)lblock * 64u + (unsigned)warp) * 0x01000193u) ^ mix32(j + 0x51ED270Bu);
-        if (c.stress & STRESS_TAGS) key ^= tag;
+        if (c.stress & STRESS_TAGS) {
+          key ^= tag;
+          key0 ^= tag;
+        }
         if (c.stress & STRESS_SKEW) {  // one commit in 8 (per warp and role) sleeps a random while
           const unsigned h = mix32(tag ^ (unsigned)r * 0x2545F491u);
           if ((h & 7u) == 0u) __nanosleep((h >> 3) % (c.skew_ns + 1u));
@@ -804,28 +816,46 @@ struct Rep {
               spin_until(fl, 0u, c, lane == 0);
             }
           }
-          pl[lane] = key;
+          // COND: an empty record (no lane of the warp stores) moves no payload,
+          // only its emptiness bit in the flag ("never execute a global write")
+          bool empty = false;
+          if constexpr (COND) empty = __ballot_sync(FULL, mask != 0u) == 0u;
+          if (!empty) {
+            pl[lane] = key;
 #pragma unroll
-          for (int k = 0; k < NW; ++k)
-            if (!COND || ((mask >> k) & 1u)) pl[(1 + k) * 32 + lane] = v[k];  // COND: only stored words move
+            for (int k = 0; k < NW; ++k)
+              if (!COND || ((mask >> k) & 1u)) pl[(1 + k) * 32 + lane] = v[k];  // COND: only stored words move
+          }
+          pempty |= (empty ? 1u : 0u) << pend;
           // The "ready" signal ("signals the work-item in the consumer") is
           // published by flush(): every lane fences its own payload stores (a
           // release by one lane does not order the other lanes' in-flight stores).
         } else {
           if (pend >= (unsigned)c.S) flush();  // as above: never wait on a slot we still hold
-          bool ok = true;
+          bool ok = true, empty = false;
           if constexpr (GROUP) {
             if (j >= rdy_hi) {  // each lane acquires the "ready" signal of the group's first record
               const unsigned g = spin_nonzero(fl, c, lane == 0);
               ok = g != 0u;
-              rdy_hi = j + g;  // records j .. j+g-1 were published behind one fence
+              rdy_hi = j + (g & 0xFFu);  // records j .. j+g-1 were published behind one fence
+              cempty = g >> 8;
+              cbase = j;
             }
+            empty = (cempty >> (j - cbase)) & 1u;
           } else {
-            ok = spin_until(fl, 1u, c, lane == 0);  // each lane acquires the "ready" signal
+            const unsigned fv = spin_nonzero(fl, c, lane == 0);  // each lane acquires the "ready" signal
+            ok = fv != 0u;
+            empty = (fv >> 8) & 1u;
           }
-          pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
+          if (COND && empty) {  // the producer stored nothing: every lane's key is key0
+            pk = key0;
 #pragma unroll
-          for (int k = 0; k < NW; ++k) pv[k] = (!COND || ((mask >> k) & 1u)) ? ld_relaxed(pl + (1 + k) * 32 + lane) : 0u;
+            for (int k = 0; k < NW; ++k) pv[k] = 0u;
+          } else {
+            pk = ld_relaxed(pl + lane);  // L2-coherent (bypasses L1)
+#pragma unroll
+            for (int k = 0; k < NW; ++k) pv[k] = (!COND || ((mask >> k) & 1u)) ? ld_relaxed(pl + (1 + k) * 32 + lane) : 0u;
+          }
           have = ok;
           // the buffer is freed only after every lane has consumed its words
           // (below, after the compare's warp ballot)

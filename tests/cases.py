@@ -350,6 +350,12 @@ class BinarySearch(Case):
     def flipped_oracle(self, elem, bit):  # LOAD = the query word
         return [oracle.binarysearch(self.A, _flip(self.q, elem, bit))]
 
+    def commit_group(self, e):
+        # a logical thread searches 2 interleaved queries and commits them as one
+        # 8-B vector (k_binarysearch.cu)
+        lo = e - e % 2
+        return np.arange(lo, min(lo + 2, self.Q))
+
     def out_elems(self):
         return 2, self.Q
 

@@ -12,7 +12,8 @@
 //   * per (region) a ring of S slots with 0/1 flags; record j lives in slot j % S;
 //   * producer: records are published in groups at every non-deferred commit:
 //     record first + l (l >= 1) gets flag value g - l (g = group size), then
-//     one fence, then record first gets g (the group's "ready" signal);
+//     one fence, then record first gets g | emptiness bits << 8 (the group's
+//     "ready" signal; an empty record -- no lane stores -- has no payload);
 //     before writing record j >= S it publishes its pending group and waits
 //     for slot j % S, but only if it must block: S records of its own pending,
 //     or the slot's flag still set (record j - S published, not yet freed);
@@ -58,6 +59,9 @@ static void jitter(std::mt19937& rng) {
 }
 
 static uint64_t tag(unsigned pair, unsigned seq) { return ((uint64_t)pair << 32) ^ (seq * 0x9E3779B97F4A7C15ull); }
+// an EMPTY record (a COND commit where no lane stores) carries no payload: the
+// producer sets its emptiness bit in the group's first flag (bits 8..15)
+static bool is_empty(unsigned pair, unsigned seq) { return ((pair * 0x9E3779B9u) ^ (seq * 0x85EBCA6Bu)) % 3u == 0u; }
 
 // one CTA role: the commit sequence of a warp (deferral pattern = program order,
 // identical in both roles: `defer[j]`)
@@ -67,7 +71,7 @@ static void run_role(Queue& q, unsigned t, unsigned nblocks, const std::vector<b
   const unsigned region = pair % (unsigned)q.R, epoch = pair / (unsigned)q.R;
   while (q.turn[region].load(std::memory_order_acquire) != epoch) std::this_thread::yield();  // region ownership
   auto slot = [&](unsigned rec) { return (size_t)region * q.S + rec % (unsigned)q.S; };
-  unsigned j = 0, pend = 0, rdy_hi = 0;
+  unsigned j = 0, pend = 0, rdy_hi = 0, pempty = 0, cempty = 0, cbase = 0;
   auto flush = [&]() {
     if (pend == 0) return;
     const unsigned first = j - pend;
@@ -83,7 +87,8 @@ static void run_role(Queue& q, unsigned t, unsigned nblocks, const std::vector<b
         jitter(rng);
       }
       std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
-      q.flag[slot(first)].store(pend, std::memory_order_relaxed);
+      q.flag[slot(first)].store(pend | (pempty << 8), std::memory_order_relaxed);
+      pempty = 0;
     } else {
       for (unsigned l = 0; l < pend; ++l) q.flag[slot(first + l)].store(0, std::memory_order_release);
     }
@@ -97,15 +102,23 @@ static void run_role(Queue& q, unsigned t, unsigned nblocks, const std::vector<b
         flush();
         while (q.flag[s].load(std::memory_order_acquire) != 0) std::this_thread::yield();
       }
-      q.payload[s].store(tag(pair, j), std::memory_order_relaxed);
+      if (is_empty(pair, j)) pempty |= 1u << pend;
+      else q.payload[s].store(tag(pair, j), std::memory_order_relaxed);
     } else {
       if (pend >= (unsigned)q.S) flush();
       if (j >= rdy_hi) {
         unsigned g;
         while ((g = q.flag[s].load(std::memory_order_acquire)) == 0) std::this_thread::yield();
-        rdy_hi = j + g;
+        rdy_hi = j + (g & 0xFFu);
+        cempty = g >> 8;
+        cbase = j;
       }
-      const uint64_t got = q.payload[s].load(std::memory_order_relaxed);
+      const bool empty = (cempty >> (j - cbase)) & 1u;
+      if (empty != is_empty(pair, j)) {
+        g_errors.fetch_add(1);
+        std::fprintf(stderr, "pair %u record %u: emptiness bit %d\n", pair, j, (int)empty);
+      }
+      const uint64_t got = empty ? tag(pair, j) : q.payload[s].load(std::memory_order_relaxed);
       if (got != tag(pair, j)) {
         g_errors.fetch_add(1);
         std::fprintf(stderr, "pair %u record %u: got tag %llx\n", pair, j, (unsigned long long)got);
