@@ -3,7 +3,8 @@
 // P:809).  Forward orthonormal 8x8 DCT-II per block (reading R-DCT1):
 //   Y = C X C^T,  C[u][x] = alpha(u) cos((2x+1) u pi / 16).
 //
-// Logical CTA = a strip of 8 image rows x 256 columns (32 blocks); logical
+// Logical CTA = NS = 4 vertically consecutive strips of 8 image rows x 256
+// columns (32 blocks each), walked with the next strip's loads in flight; logical
 // thread (row r, block b) does the row pass Z[r][.] = X[r][.] C^T (8 FMA-chains
 // of length 8), Z goes through (duplicated, +LDS) shared memory, then logical
 // thread (b, u) does the column pass Y[u][.] = C[u][.] Z and commits its output
@@ -22,12 +23,17 @@ constexpr int BLOCKS = 32;       // 8x8 blocks per logical CTA
 constexpr int BSTRIDE = 68;      // words per block in smem (64 + 4: conflict-free column pass)
 constexpr int ZWORDS = BLOCKS * BSTRIDE;
 constexpr int PLANE = ZWORDS + 16;  // replica plane offset (16 banks apart)
+#ifndef DCT_NS
+#define DCT_NS 4
+#endif
+constexpr unsigned NS = DCT_NS;     // 8-row strips per logical CTA
 
 struct DctArgs {
   const float* X;
   float* Y;
   unsigned H, W;
   unsigned nbx;  // logical CTAs across a row strip
+  unsigned nby;  // 8-row strips
   unsigned v8;   // X is 32-B aligned: 256-bit row loads
   float C[8][8];
 };
@@ -40,31 +46,47 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c
   Rep<V, M> rep(c);
   rep.init(mb);
   for (; rep.active(); rep.advance()) {
-    const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
+    const unsigned bg = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
     // row pass: logical warp w = image row r of the strip, lane = block b, so a
     // warp's loads are one contiguous 1 KiB row segment (coalesced; with the
     // block-major mapping of the column pass below the loads touched 8 rows per
     // instruction and L1 ran at 98%: 0.203 -> 0.154 ms at 8192^2)
-    int b = rep.ltid % BLOCKS, r = rep.ltid / BLOCKS;
-    unsigned col0 = (bx * BLOCKS + b) * 8;
-    bool active = col0 < a.W;
+    const int b0 = rep.ltid % BLOCKS, r = rep.ltid / BLOCKS;
+    const unsigned col00 = (bx * BLOCKS + b0) * 8;
+    const bool active0 = col00 < a.W;
+    auto load_x = [&](unsigned by, float (&x)[8]) {
+      const unsigned row = by * 8 + r;
+      if (active0) {
+        if (a.v8) {  // one 256-bit load: the warp's 1 KiB row segment in whole lines
+          unsigned w[8];
+          ldcs8(a.X + (size_t)row * a.W + col00, w);
+#pragma unroll
+          for (int y = 0; y < 8; ++y) x[y] = __uint_as_float(w[y]);
+        } else {  // X only 16-B aligned (the ABI minimum)
+          const float4* src = reinterpret_cast<const float4*>(a.X + (size_t)row * a.W + col00);
+          float4 p = __ldcs(src), q = __ldcs(src + 1);
+          x[0] = p.x; x[1] = p.y; x[2] = p.z; x[3] = p.w; x[4] = q.x; x[5] = q.y; x[6] = q.z; x[7] = q.w;
+        }
+      } else {
+#pragma unroll
+        for (int y = 0; y < 8; ++y) x[y] = 0.0f;
+      }
+    };
+    // A logical CTA walks NS vertically consecutive strips; the next strip's
+    // row segment is in flight while this one is transformed (register double
+    // buffer: twice the bytes in flight per SM)
+    float xn[8];
+    load_x(bg * NS, xn);
+#pragma unroll 1
+    for (unsigned by = bg * NS; by < bg * NS + NS && by < a.nby; ++by) {  // CTA-uniform
+    int b = b0;
+    unsigned col0 = col00;
+    bool active = active0;
     const unsigned row = by * 8 + r;
     float x[8];
-    if (active) {
-      if (a.v8) {  // one 256-bit load: the warp's 1 KiB row segment in whole lines
-        unsigned w[8];
-        ldcs8(a.X + (size_t)row * a.W + col0, w);
 #pragma unroll
-        for (int y = 0; y < 8; ++y) x[y] = __uint_as_float(w[y]);
-      } else {  // X only 16-B aligned (the ABI minimum)
-        const float4* src = reinterpret_cast<const float4*>(a.X + (size_t)row * a.W + col0);
-        float4 p = __ldcs(src), q = __ldcs(src + 1);
-        x[0] = p.x; x[1] = p.y; x[2] = p.z; x[3] = p.w; x[4] = q.x; x[5] = q.y; x[6] = q.z; x[7] = q.w;
-      }
-    } else {
-#pragma unroll
-      for (int y = 0; y < 8; ++y) x[y] = 0.0f;
-    }
+    for (int y = 0; y < 8; ++y) x[y] = xn[y];
+    if (by + 1 < bg * NS + NS && by + 1 < a.nby) load_x(by + 1, xn);
     if constexpr (M == M_FAULT) {
 #pragma unroll
       for (int y = 0; y < 8; ++y) x[y] = rep.faultf(SITE_LOAD, (long long)row * a.W + col0 + y, x[y]);
@@ -153,6 +175,8 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c
                                 },
                                 /*defer=*/h == 0);
     }
+    __syncthreads();  // the column pass has read Zs before the next strip's row pass writes it
+    }
   }
   rep.finish();
 }
@@ -180,13 +204,15 @@ int dct_run(Launch& L) {
   a.H = H;
   a.W = W;
   a.nbx = nbx;
+  a.nby = nby;
   a.v8 = ((uintptr_t)a.X % 32) == 0 ? 1u : 0u;
   for (int u = 0; u < 8; ++u)  // C[u][x] = alpha(u) cos((2x+1) u pi / 16), in fp64 then rounded
     for (int x = 0; x < 8; ++x)
       a.C[u][x] = (float)((u == 0 ? sqrt(0.125) : 0.5) * cos((2.0 * x + 1.0) * u * 3.14159265358979323846 / 16.0));
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
-    return launch_std<V>(L, dct_kernel<V, M>, dct_kernel<V_NONE, M_NORMAL>, nbx * nby, BL, 0, a, "dct");
+    return launch_std<V>(L, dct_kernel<V, M>, dct_kernel<V_NONE, M_NORMAL>, nbx * ((nby + NS - 1) / NS), BL, 0, a,
+                         "dct");
   });
 }
 
