@@ -409,6 +409,31 @@ def test_dct_vs_scipy_and_closed_forms():
     assert np.all(B >= np.abs(Y) - 1e-9)
 
 
+def test_dct_absbound_tight_and_additive():
+    """The conditioning bound B[u][v] = sum_xy |C[u][x]| |X[x][y]| |C[v][y]| is
+    pinned by what it must satisfy, not by its formula: on a delta block every
+    Y[u][v] is a single product, so B == |Y| exactly; B is additive over
+    blocks of disjoint support and absolutely homogeneous; a sign-matched block
+    X = outer(sign C[u], sign C[v]) attains B[u][v] = |Y[u][v]|."""
+    Cm = np.array([[(math.sqrt(1 / 8) if a == 0 else 0.5) * math.cos((2 * x + 1) * a * math.pi / 16)
+                    for x in range(8)] for a in range(8)])
+    Bsum = np.zeros((8, 8))
+    rng = np.random.default_rng(5)
+    Xr = rng.uniform(-3, 3, (8, 8)).astype(np.float32)
+    for x in range(8):
+        for y in range(8):
+            D = np.zeros((8, 8), np.float32)
+            D[x, y] = 1.0
+            Bd = oracle.dct8x8_absbound(D)
+            assert np.allclose(Bd, np.abs(oracle.dct8x8(D)), rtol=1e-12, atol=1e-15)
+            Bsum += abs(float(Xr[x, y])) * Bd
+    assert np.allclose(oracle.dct8x8_absbound(Xr), Bsum, rtol=1e-12, atol=1e-12)
+    assert np.allclose(oracle.dct8x8_absbound(-2 * Xr), 2 * oracle.dct8x8_absbound(Xr), rtol=1e-12)
+    for u, v in ((0, 0), (3, 5), (7, 1)):
+        Xs = np.outer(np.sign(Cm[u]), np.sign(Cm[v])).astype(np.float32)
+        assert abs(oracle.dct8x8_absbound(Xs)[u, v] - abs(oracle.dct8x8(Xs)[u, v])) < 1e-9
+
+
 # ---------------------------------------------------------------- MatrixMultiplication
 
 
