@@ -181,14 +181,19 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
 #ifndef BINS_MINB
 #define BINS_MINB 4
 #endif
+#ifndef BINS_GROUP
+#define BINS_GROUP 1
+#endif
 template <int V, int M>
 // Registers capped at 64 (4 CTAs of 256 / 2 of 512 threads per SM).
 __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? BINS_MINB / 2 : BINS_MINB) bins_kernel(BsArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   extern __shared__ __align__(16) unsigned char bins_dyn[];
-  Rep<V, M> rep(c);
+  // inter: group flags, the commits of BINS_GROUP consecutive chunks published
+  // behind one fence (deferred commits; the last chunk of a logical CTA closes)
+  Rep<V, M, (BINS_GROUP > 1)> rep(c);
   rep.init(mb);
-  using R = Rep<V, M>;
+  using R = Rep<V, M, (BINS_GROUP > 1)>;
   // ---- the table L_T in shared memory, once per physical CTA (every logical
   // CTA of a persistent pair reuses it).  +LDS: each replica writes and reads
   // its own copy; -LDS: one copy, every store compared.
@@ -319,12 +324,14 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? BINS_MI
 #pragma unroll 1
       for (int lv = T - 1; lv >= 1; --lv) level(a.lev + a.L.off[lv], false);  // padded: no bounds checks
       level(a.A, true);  // the caller's A
+      const bool close = (it + 1u) % BINS_GROUP == 0u || it + 1u == a.iters ||
+                         (unsigned long long)(chunk + 1u) * CHUNK >= a.Q;  // CTA-uniform
       rep.template commit<VEC, 0>(mask, j0, jj, a.Q, [&](unsigned i, unsigned m, const unsigned* w) {
         if (m == 0x3u) __stcs(reinterpret_cast<uint2*>(a.idx + i), make_uint2(w[0], w[1]));
         else
           for (int k = 0; k < VEC; ++k)
             if ((m >> k) & 1u) a.idx[i + k] = w[k];
-      });
+      }, /*defer=*/!close);
     }
   }
   rep.finish();
