@@ -652,6 +652,9 @@ def small_cases():
         BinarySearch((1 << 20) + 13, 70001), BinarySearch(4096 + 9, 5000, odd=True),
         BinarySearch(5, 64, dups=True), BinarySearch(4096 * 3 + 7, 20001, dups=True),
         BinarySearch((1 << 21) + 5, 1 << 16, dups=True),
+        # shared-memory table edges (k_binarysearch.cu): n_T = 8192 = P exactly
+        # (no padding entry: the final compare), and three sample levels (T = 3)
+        BinarySearch(1 << 18, 3001), BinarySearch((8 << 20) + 7, 40000),
         Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
         DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8), DCT(64, 512, specials=True),
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),

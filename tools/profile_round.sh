@@ -35,6 +35,7 @@ ls -la $out $out/full
 # summarise on the box (the .ncu-rep files together exceed gpurun's 64 MiB
 # copy-back limit); keep the dominant kernel's report only
 python tools/ncu_summary.py $out/full/*.ncu-rep --json $out/ncu_full_summary.json > $out/ncu_full_summary.txt 2>&1
+python tools/traffic_from_summary.py $out/ncu_full_summary.json $out/ncu_traffic.json
 mkdir -p $out/keep
 mv $out/full/binarysearch_inter_group.ncu-rep $out/keep/ 2>/dev/null
 rm -f $out/full/*.ncu-rep
