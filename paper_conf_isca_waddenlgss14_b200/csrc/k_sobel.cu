@@ -22,6 +22,16 @@ namespace rmt {
 namespace {
 
 constexpr int BL = 256;
+// inter_group: the records of SOBEL_GROUP consecutive rows are published as one
+// group behind one fence (group flags).  Measured at 8192^2 (x none): 1 row
+// 3.89x, 2 3.62x, 3 3.36x, 5 3.41x, 6 3.57x, 8 4.08x; inter_cluster publishes
+// every row (deferral there: 2.99 -> 3.04-3.49x); persistent pairs lose (4.0-4.2x).
+#ifndef SOBEL_GROUP
+#define SOBEL_GROUP 3
+#endif
+#ifndef SOBEL_MULT_INTER
+#define SOBEL_MULT_INTER 0
+#endif
 constexpr int RY = 30;  // output rows per thread (measured: 32 rows 0.174 ms, 30 rows 0.162 ms at 8192^2)
 
 struct SobArgs {
@@ -116,8 +126,8 @@ __device__ __forceinline__ void load_raw(const SobArgs& a, int y, unsigned x0, b
 }
 
 // Apply the LOAD-site fault hook and split into 16-bit channel lanes.
-template <int V, int M>
-__device__ __forceinline__ void unpack_row(const Rep<V, M>& rep, const SobArgs& a, int y, unsigned x0,
+template <int V, int M, bool G>
+__device__ __forceinline__ void unpack_row(const Rep<V, M, G>& rep, const SobArgs& a, int y, unsigned x0,
                                            unsigned (&p)[6], Row& R) {
   if constexpr (M == M_FAULT) {
     if (y >= 0 && y < (int)a.H) {
@@ -144,7 +154,7 @@ struct BoolC {
 template <int V, int M>
 __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) sobel_kernel(SobArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
-  Rep<V, M> rep(c);
+  Rep<V, M, (SOBEL_GROUP > 1 && V == V_INTER)> rep(c);
   rep.init(mb);
   for (; rep.active(); rep.advance()) {
     const unsigned by = (unsigned)rep.lblock / a.nbx, bx = (unsigned)rep.lblock % a.nbx;
@@ -207,7 +217,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) 
                                     else
                                       for (int k = 0; k < 4; ++k)
                                         if ((mm >> k) & 1u) a.O[idx + k] = w[k];
-                                  });
+                                  }, /*defer=*/V == V_INTER && SOBEL_GROUP > 1 && (y - y0) % SOBEL_GROUP != SOBEL_GROUP - 1 && y + 1 < y0 + RY);
       };
       // rolling 3-row window; the raw words of the row after next are in flight
       // while the current row is filtered (one row of prefetch distance)
@@ -255,7 +265,7 @@ int sobel_run(Launch& L) {
   SobArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, H, W, nbx};
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
-    return launch_std<V>(L, sobel_kernel<V, M>, sobel_kernel<V_NONE, M_NORMAL>, nbx * nby, BL, 0, a, "sobel", /*mult_inter=*/0,
+    return launch_std<V>(L, sobel_kernel<V, M>, sobel_kernel<V_NONE, M_NORMAL>, nbx * nby, BL, 0, a, "sobel", /*mult_inter=*/SOBEL_MULT_INTER,
                          /*mult_cluster=*/0);
   });
 }
