@@ -186,6 +186,55 @@ __device__ __forceinline__ void cluster_sync_all() {
 #ifndef RMT_SPIN_NSMAX
 #define RMT_SPIN_NSMAX 512  // back-off cap
 #endif
+// Inter-Group record format (reading R-C-Q2):
+// 1 = digest records -- one 64-bit word per lane and record, (j + 1) << 32 |
+// digest(key, stored words), published and freed with single-copy-atomic
+// relaxed accesses (no flag, fence or lock); 0 = the round-1/2 flag protocol
+// (full key + value words behind group flags and a fence).
+#ifndef RMT_INTER_DIGEST
+#define RMT_INTER_DIGEST 1
+#endif
+
+// Record digest: a chain of bijections in each word (x -> (h ^ x) * odd, then an
+// xorshift), so a change confined to ANY ONE word of (key, v0..v3) -- every
+// single-bit fault of the fault model -- always changes the digest; changes in
+// several words alias with probability ~2^-32.
+template <int NW>
+__device__ __forceinline__ unsigned rec_digest(unsigned key, unsigned mask, const unsigned (&v)[NW]) {
+  unsigned h = key * 0x9E3779B1u;
+  h ^= h >> 15;
+#pragma unroll
+  for (int k = 0; k < NW; ++k) {
+    const unsigned w = ((mask >> k) & 1u) ? v[k] : 0u;  // unstored words are not compared (COND sites)
+    h = (h ^ w) * 0x85EBCA77u;
+    h ^= h >> 13;
+  }
+  return h;
+}
+
+// Spin (relaxed, L2-coherent: P:693) until the 64-bit word at p satisfies
+// pred(word); returns the last word read.  Watchdog as spin_until below.
+template <class Pred>
+__device__ __forceinline__ unsigned long long spin64(const unsigned long long* p, unsigned long long x, Pred pred,
+                                                     const Ctx& c, bool count) {
+  if (pred(x)) return x;
+  unsigned long long t0 = clock64();
+  unsigned ns = RMT_SPIN_NS0;
+  while (true) {
+    if (ns) __nanosleep(ns);
+    x = ld_relaxed64(p);
+    if (pred(x)) return x;
+    if (ns && ns < RMT_SPIN_NSMAX) ns <<= 1;
+    if (clock64() - t0 > c.wd) {
+      if (count) {
+        atomicAdd(c.err, 1ull);
+        atomicExch(c.ctrl + CTRL_WATCHDOG, 1u);
+      }
+      return x;
+    }
+  }
+}
+
 // Spin until *p == want (acquire), with back-off and a watchdog that converts a
 // hang (a fault that desynchronised a pair) into err+1 and a sticky flag.
 // Every thread that will touch the guarded data must do its own acquire: a lane
@@ -308,12 +357,15 @@ struct Rep {
   unsigned rdy_hi;  // inter consumer: records below this are known to be published (group flags)
   unsigned pempty;  // inter producer: bit l = pending record (j - pend + l) is empty (COND, no lane stores)
   unsigned cempty, cbase;  // inter consumer: emptiness bits of the group starting at record cbase
+  unsigned long long pf;  // inter (digest records): the word of the next record's slot, loaded ahead
+  bool pfv;               // pf holds that word
   unsigned* mbox;  // intra_smem: this warp's mailbox
   unsigned tr_id;  // RMT_TRACE: trace row (inter ticket)
   unsigned cl_pay, cl_full;  // inter_cluster: this warp's mailbox / flags in the consumer CTA (shared::cluster)
 
   __device__ __forceinline__ explicit Rep(const Ctx& ctx)
       : c(ctx), j(0), lstride(0), nerr(0), pend(0), region(0), epoch(0), rdy_hi(0), pempty(0), cempty(0), cbase(0),
+        pf(0ull), pfv(false),
         mbox(nullptr), cl_pay(0),
         cl_full(0) {}
 
@@ -460,7 +512,7 @@ struct Rep {
       }
       pend = 0u;
     }
-    if constexpr (INTER && !NOCOMM) {
+    if constexpr (INTER && !NOCOMM && !RMT_INTER_DIGEST) {
       if (pend == 0u) return;
       const unsigned first = j - pend;
       if (!consumer) {
@@ -537,6 +589,10 @@ struct Rep {
         if (ld_relaxed(c.ctrl + CTRL_WATCHDOG) != 0u) {
           const size_t nslots = (size_t)c.R * (size_t)c.W * (size_t)INTER_SLOTS_MAX;
           for (size_t i = threadIdx.x; i < nslots; i += blockDim.x) c.flags[i] = 0u;
+          if (RMT_INTER_DIGEST) {  // digest records: every slot word a lost consumer left behind
+            unsigned long long* w = reinterpret_cast<unsigned long long*>(c.payload);
+            for (size_t i = threadIdx.x; i < nslots * 32; i += blockDim.x) w[i] = 0ull;
+          }
         }
         if (threadIdx.x == 0) {
           c.ctrl[CTRL_TICKET] = 0;
@@ -789,6 +845,35 @@ struct Rep {
 #pragma unroll
           for (int k = 0; k < NW; ++k) pv[k] = (!COND || ((mask >> k) & 1u)) ? ld_cl(pa + (1 + k) * 32 * 4) : 0u;
         }
+      } else if constexpr (V == V_INTER && RMT_INTER_DIGEST) {
+        // Digest records (R-C-Q2): record j of this (region, warp) is ONE 64-bit
+        // word per lane in slot j % S: (j + 1) << 32 | digest(key, stored words).
+        // A slot word is 0 (free) or a record; the producer writes only a free
+        // slot, the consumer waits for marker j + 1 and frees it -- all relaxed
+        // accesses to the same address, ordered by coherence, so no flag,
+        // fence or lock; the first tier (region turns) is unchanged.  The
+        // word of the next record's slot is loaded ahead at the end of a commit.
+        const unsigned h = rec_digest<NW>(key, mask, v);
+        unsigned long long* const ring = reinterpret_cast<unsigned long long*>(c.payload);
+        unsigned long long* const pw = ring + slot_index(j) * 32 + lane;
+        if (!consumer) {
+          if (j >= (unsigned)c.S) {  // record j - S must have been freed ("waits for a free buffer")
+            const unsigned long long x = pfv ? pf : ld_relaxed64(pw);
+            spin64(pw, x, [](unsigned long long w) { return w == 0ull; }, c, lane == 0);
+          }
+          st_relaxed64(pw, ((unsigned long long)(j + 1u) << 32) | h);
+          pfv = j + 1u >= (unsigned)c.S;
+          if (pfv) pf = ld_relaxed64(ring + slot_index(j + 1u) * 32 + lane);
+        } else {
+          const unsigned mk = j + 1u;
+          unsigned long long x = pfv ? pf : ld_relaxed64(pw);
+          x = spin64(pw, x, [mk](unsigned long long w) { return (unsigned)(w >> 32) == mk; }, c, lane == 0);
+          have = (unsigned)(x >> 32) == mk;
+          st_relaxed64(pw, 0ull);  // free: the same address, after the read
+          pk = (unsigned)x ^ h;    // 0 iff the digests agree
+          pfv = true;
+          pf = ld_relaxed64(ring + slot_index(j + 1u) * 32 + lane);
+        }
       } else {  // V_INTER: per-(region, warp) queue of S records
 #ifdef RMT_TRACE
         if (j == 0) RMT_TR(2, gtimer());
@@ -864,9 +949,15 @@ struct Rep {
       bool mism = false;
       if (consumer) {
         // bitwise difference of key (address + predicate) and of the stored words
-        unsigned d = pk ^ key;
+        // (digest records: pk is already the digest difference)
+        unsigned d;
+        if constexpr (V == V_INTER && RMT_INTER_DIGEST) {
+          d = pk;
+        } else {
+          d = pk ^ key;
 #pragma unroll
-        for (int k = 0; k < NW; ++k) d |= (pv[k] ^ v[k]) & (0u - ((mask >> k) & 1u));
+          for (int k = 0; k < NW; ++k) d |= (pv[k] ^ v[k]) & (0u - ((mask >> k) & 1u));
+        }
         const bool eq = have && d == 0u;
         if (eq) {
           if (mask != 0u) store(idx, mask, v);
@@ -888,7 +979,9 @@ struct Rep {
         const unsigned mb = __ballot_sync(FULL, mism);
         if (mb != 0u && lane == __ffs(mb) - 1) atomicAdd(c.err, (unsigned long long)__popc(mb));
       }
-      if constexpr (INTER || CLUSTER) {
+      if constexpr (V == V_INTER && RMT_INTER_DIGEST) {
+        ++j;  // published and freed above; nothing pending
+      } else if constexpr (INTER || CLUSTER) {
         ++j;
         ++pend;
         if (!defer) flush();  // publish (producer) / free the buffers (consumer)

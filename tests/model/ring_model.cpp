@@ -4,29 +4,28 @@
 //
 // Restates, with std::atomic and C++ memory orders, the protocol that
 // paper_conf_isca_waddenlgss14_b200/csrc/rmt_device.cuh implements for
-// V_INTER (Rep::init / commit / flush / finish), one thread per CTA role:
+// V_INTER (Rep::init / commit / finish), one thread per CTA role (a lane of a
+// warp: lanes are independent, each owns one 64-bit word per slot):
 //   * tickets from a global counter in start order; pair = t >> 1, even ticket =
 //     producer, odd = consumer;
-//   * region = pair % R; both roles wait for turn[region] == pair / R, the
-//     consumer advances it at exit;
-//   * per (region) a ring of S slots with 0/1 flags; record j lives in slot j % S;
-//   * producer: records are published in groups at every non-deferred commit:
-//     record first + l (l >= 1) gets flag value g - l (g = group size), then
-//     one fence, then record first gets g | emptiness bits << 8 (the group's
-//     "ready" signal; an empty record -- no lane stores -- has no payload);
-//     before writing record j >= S it publishes its pending group and waits
-//     for slot j % S, but only if it must block: S records of its own pending,
-//     or the slot's flag still set (record j - S published, not yet freed);
-//   * consumer: before waiting on record j it frees its pending records if it
-//     holds S of them; for the first record of a group it waits for a nonzero
-//     flag (acquire) -- the value g says records j .. j+g-1 are visible, so
-//     those need no flag check of their own; it reads, compares, and frees in
-//     batches at every non-deferred commit (release store of 0);
-//   * the last finisher resets tickets and turns.
+//   * first tier: region = pair % R; both roles wait for turn[region] ==
+//     pair / R, the consumer advances it (release) at exit;
+//   * second tier, per (region) a ring of S one-word slots; record j lives in
+//     slot j % S as ONE 64-bit word (j + 1) << 32 | digest, so a record is
+//     published and read with single-copy-atomic accesses and needs no flag,
+//     fence or lock: a slot holds 0 (free) or a record;
+//   * producer: record j >= S waits until its slot reads 0 (the consumer freed
+//     record j - S), then stores the word (relaxed);
+//   * consumer: waits until its slot holds marker j + 1, reads the digest,
+//     then stores 0 (relaxed; the same address, so coherence orders the free
+//     after the read and the producer's next write after the free);
+//   * every consumed slot is freed, so a pair leaves its region all-zero; the
+//     last finisher resets tickets and turns.
 // Workers (the resident CTA slots) take tickets until 2P are gone.  Checks: every
-// record is consumed exactly once, in order, with the payload its producer wrote
+// record is consumed exactly once, in order, with the digest its producer wrote
 // (tagged (pair, seq)); every launch finishes (no deadlock) for any S >= 1, any
-// R >= 1 and any number of workers >= 2; the control block is zero afterwards.
+// R >= 1 and any number of workers >= 2; the control block and every slot are
+// zero afterwards.
 //
 //   ring_model S R WORKERS PAIRS RECORDS SEED LAUNCHES
 #include <atomic>
@@ -40,13 +39,11 @@
 struct Queue {
   int S, R;
   std::atomic<unsigned> ticket{0}, done{0};
-  std::vector<std::atomic<unsigned>> turn;     // R
-  std::vector<std::atomic<unsigned>> flag;     // R * S
-  std::vector<std::atomic<uint64_t>> payload;  // R * S (relaxed: ordered by the flags)
-  Queue(int S_, int R_) : S(S_), R(R_), turn(R_), flag((size_t)R_ * S_), payload((size_t)R_ * S_) {
+  std::vector<std::atomic<unsigned>> turn;  // R
+  std::vector<std::atomic<uint64_t>> slot;  // R * S
+  Queue(int S_, int R_) : S(S_), R(R_), turn(R_), slot((size_t)R_ * S_) {
     for (auto& t : turn) t.store(0);
-    for (auto& f : flag) f.store(0);
-    for (auto& p : payload) p.store(0);
+    for (auto& w : slot) w.store(0);
   }
 };
 
@@ -58,77 +55,30 @@ static void jitter(std::mt19937& rng) {
   else if (r == 1) for (volatile int i = 0; i < (int)(rng() % 2000); ++i) {}
 }
 
-static uint64_t tag(unsigned pair, unsigned seq) { return ((uint64_t)pair << 32) ^ (seq * 0x9E3779B97F4A7C15ull); }
-// an EMPTY record (a COND commit where no lane stores) carries no payload: the
-// producer sets its emptiness bit in the group's first flag (bits 8..15)
-static bool is_empty(unsigned pair, unsigned seq) { return ((pair * 0x9E3779B9u) ^ (seq * 0x85EBCA6Bu)) % 3u == 0u; }
+static uint32_t tag(unsigned pair, unsigned seq) { return (pair * 0x9E3779B9u) ^ (seq * 0x85EBCA6Bu) ^ 0x5bd1e995u; }
 
-// one CTA role: the commit sequence of a warp (deferral pattern = program order,
-// identical in both roles: `defer[j]`)
-static void run_role(Queue& q, unsigned t, unsigned nblocks, const std::vector<bool>& defer, std::mt19937& rng) {
+static void run_role(Queue& q, unsigned t, unsigned nblocks, unsigned nrec, std::mt19937& rng) {
   const unsigned pair = t >> 1;
   const bool consumer = t & 1u;
   const unsigned region = pair % (unsigned)q.R, epoch = pair / (unsigned)q.R;
   while (q.turn[region].load(std::memory_order_acquire) != epoch) std::this_thread::yield();  // region ownership
-  auto slot = [&](unsigned rec) { return (size_t)region * q.S + rec % (unsigned)q.S; };
-  unsigned j = 0, pend = 0, rdy_hi = 0, pempty = 0, cempty = 0, cbase = 0;
-  auto flush = [&]() {
-    if (pend == 0) return;
-    const unsigned first = j - pend;
-    if (!consumer) {
-      // the group's non-first flags go out BEFORE the fence and the first
-      // record's flag after it: a consumer that acquires flag[first] then sees
-      // every other flag of the group already stored, so its later frees of
-      // those slots cannot be overtaken by a late producer flag store (which
-      // would leave a stale "full" flag: a stale read or a deadlock)
-      // (jitter between the stores: lanes' stores land in any order)
-      for (unsigned l = 1; l < pend; ++l) {
-        q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
-        jitter(rng);
-      }
-      std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
-      q.flag[slot(first)].store(pend | (pempty << 8), std::memory_order_relaxed);
-      pempty = 0;
-    } else {
-      for (unsigned l = 0; l < pend; ++l) q.flag[slot(first + l)].store(0, std::memory_order_release);
-    }
-    pend = 0;
-  };
-  for (size_t k = 0; k < defer.size(); ++k) {
+  for (unsigned j = 0; j < nrec; ++j) {
     jitter(rng);
-    const size_t s = slot(j);
+    std::atomic<uint64_t>& w = q.slot[(size_t)region * q.S + j % (unsigned)q.S];
     if (!consumer) {
-      if (j >= (unsigned)q.S && (pend >= (unsigned)q.S || q.flag[s].load(std::memory_order_acquire) != 0)) {
-        flush();
-        while (q.flag[s].load(std::memory_order_acquire) != 0) std::this_thread::yield();
-      }
-      if (is_empty(pair, j)) pempty |= 1u << pend;
-      else q.payload[s].store(tag(pair, j), std::memory_order_relaxed);
+      if (j >= (unsigned)q.S)
+        while (w.load(std::memory_order_relaxed) != 0) std::this_thread::yield();  // record j - S freed
+      w.store((uint64_t)(j + 1) << 32 | tag(pair, j), std::memory_order_relaxed);
     } else {
-      if (pend >= (unsigned)q.S) flush();
-      if (j >= rdy_hi) {
-        unsigned g;
-        while ((g = q.flag[s].load(std::memory_order_acquire)) == 0) std::this_thread::yield();
-        rdy_hi = j + (g & 0xFFu);
-        cempty = g >> 8;
-        cbase = j;
-      }
-      const bool empty = (cempty >> (j - cbase)) & 1u;
-      if (empty != is_empty(pair, j)) {
+      uint64_t v;
+      while (((v = w.load(std::memory_order_relaxed)) >> 32) != j + 1) std::this_thread::yield();
+      if ((uint32_t)v != tag(pair, j)) {
         g_errors.fetch_add(1);
-        std::fprintf(stderr, "pair %u record %u: emptiness bit %d\n", pair, j, (int)empty);
+        std::fprintf(stderr, "pair %u record %u: got digest %x\n", pair, j, (unsigned)v);
       }
-      const uint64_t got = empty ? tag(pair, j) : q.payload[s].load(std::memory_order_relaxed);
-      if (got != tag(pair, j)) {
-        g_errors.fetch_add(1);
-        std::fprintf(stderr, "pair %u record %u: got tag %llx\n", pair, j, (unsigned long long)got);
-      }
+      w.store(0, std::memory_order_relaxed);  // free (same address: after the read)
     }
-    ++j;
-    ++pend;
-    if (!defer[k]) flush();
   }
-  flush();
   if (consumer) q.turn[region].store(epoch + 1, std::memory_order_release);
   std::atomic_thread_fence(std::memory_order_seq_cst);
   const unsigned d = q.done.fetch_add(1);
@@ -146,19 +96,11 @@ int main(int argc, char** argv) {
   }
   const int S = atoi(argv[1]), R = atoi(argv[2]), W = atoi(argv[3]);
   const unsigned P = (unsigned)atoi(argv[4]);
-  const int NREC = atoi(argv[5]);
+  const unsigned NREC = (unsigned)atoi(argv[5]);
   const unsigned seed = (unsigned)atoi(argv[6]);
   const int launches = atoi(argv[7]);
   Queue q(S, R);
-  std::mt19937 g(seed);
   for (int L = 0; L < launches; ++L) {
-    // the warp's commit sequence: runs of 0..5 deferred commits closed by a non-deferred one
-    std::vector<bool> defer;
-    while ((int)defer.size() < NREC) {
-      int run = (int)(g() % 6);
-      for (int i = 0; i < run && (int)defer.size() < NREC - 1; ++i) defer.push_back(true);
-      defer.push_back(false);
-    }
     std::atomic<unsigned> next{0};
     std::vector<std::thread> th;
     for (int w = 0; w < W; ++w) {
@@ -168,16 +110,16 @@ int main(int argc, char** argv) {
           // a worker (resident CTA slot) starts the next CTA: it takes a ticket first
           if (next.fetch_add(1) >= 2 * P) break;
           const unsigned t = q.ticket.fetch_add(1);
-          run_role(q, t, P, defer, rng);
+          run_role(q, t, P, NREC, rng);
         }
       });
     }
     for (auto& t : th) t.join();
     bool clean = q.ticket.load() == 0 && q.done.load() == 0;
     for (auto& tr : q.turn) clean = clean && tr.load() == 0;
-    for (auto& f : q.flag) clean = clean && f.load() == 0;
+    for (auto& s : q.slot) clean = clean && s.load() == 0;
     if (!clean) {
-      std::fprintf(stderr, "launch %d: control block not reset\n", L);
+      std::fprintf(stderr, "launch %d: control block or a slot not reset\n", L);
       return 1;
     }
   }
@@ -185,6 +127,6 @@ int main(int argc, char** argv) {
     std::fprintf(stderr, "%ld out-of-order / foreign records\n", g_errors.load());
     return 1;
   }
-  std::printf("ok S=%d R=%d workers=%d pairs=%u records=%d launches=%d\n", S, R, W, P, NREC, launches);
+  std::printf("ok S=%d R=%d workers=%d pairs=%u records=%u launches=%d\n", S, R, W, P, NREC, launches);
   return 0;
 }

@@ -2,17 +2,16 @@
 "C-Q inter-group ring": a std::atomic model of the same protocol under stress).
 
 tests/model/ring_model.cpp restates the protocol of rmt_device.cuh (V_INTER)
-with C++ acquire/release atomics, one thread per CTA role and a pool of worker
-threads standing in for the resident CTA slots.  Every configuration must finish
-(no deadlock) with every record consumed once, in order, with its producer's
-(pair, sequence) tag, and leave the control block zeroed -- at ring depth 1, 2,
-4 and 8, one region (every pair hands the ring to the next) or several, and
-down to 2 workers (the minimum residency the deadlock-freedom argument needs).
-A mutant without the consumer's "free before waiting when S records are held"
-rule must fail, and so must a mutant that publishes a group's flags in record
-order behind one fence (a consumer that acquired the first flag may free a
-later slot before that slot's flag store lands, leaving a stale "full" flag),
-so the model can tell the difference.
+with C++ atomics, one thread per CTA role and a pool of worker threads standing
+in for the resident CTA slots: region turns (first tier) and per-slot 64-bit
+records (marker j + 1, digest) freed by the consumer (second tier).  Every
+configuration must finish (no deadlock) with every record consumed once, in
+order, with its producer's (pair, sequence) digest, and leave the control block
+and every slot zeroed -- at ring depth 1, 2, 4 and 8, one region (every pair
+hands the ring to the next) or several, and down to 2 workers (the minimum
+residency the deadlock-freedom argument needs).  Mutants that drop the
+consumer's free or the producer's wait for a free slot must fail, so the model
+can tell the difference.
 """
 import os
 import subprocess
@@ -49,39 +48,26 @@ def test_ring_protocol_model(model, S, R, workers):
         assert r.stdout.startswith("ok")
 
 
-def test_ring_model_detects_missing_consumer_free(tmp_path):
+def _mutant_fails(tmp_path, old, new, name):
     text = open(SRC).read()
-    rule = "      if (pend >= (unsigned)q.S) flush();\n"
-    assert rule in text
-    exe = _build(tmp_path, text.replace(rule, ""), "ring_mutant")
-    try:
-        r = subprocess.run([exe, "1", "2", "2", "16", "40", "1", "3"], capture_output=True, text=True, timeout=10)
-        failed = r.returncode != 0
-    except subprocess.TimeoutExpired:
-        failed = True  # deadlock
-    assert failed, "the model accepted a protocol without the consumer-side free rule"
-
-
-def test_ring_model_detects_group_flags_published_in_order(tmp_path):
-    text = open(SRC).read()
-    fixed = """      for (unsigned l = 1; l < pend; ++l) {
-        q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
-        jitter(rng);
-      }
-      std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
-      q.flag[slot(first)].store(pend, std::memory_order_relaxed);"""
-    in_order = """      std::atomic_thread_fence(std::memory_order_seq_cst);  // fence.sc.gpu
-      for (unsigned l = 0; l < pend; ++l) {
-        q.flag[slot(first + l)].store(pend - l, std::memory_order_relaxed);
-        jitter(rng);
-      }"""
-    assert fixed in text
-    exe = _build(tmp_path, text.replace(fixed, in_order), "ring_in_order")
+    assert old in text
+    exe = _build(tmp_path, text.replace(old, new), name)
     failures = 0
     for seed in range(1, 4):
         try:
-            r = subprocess.run([exe, "2", "1", "2", "48", "60", str(seed), "3"], capture_output=True, text=True, timeout=10)
+            r = subprocess.run([exe, "2", "1", "2", "16", "40", str(seed), "2"], capture_output=True, text=True,
+                               timeout=10)
             failures += r.returncode != 0
         except subprocess.TimeoutExpired:
-            failures += 1  # a stale full flag: the producer waits forever
-    assert failures > 0, "the model accepted group flags published first-record-first"
+            failures += 1  # deadlock
+    return failures > 0
+
+
+def test_ring_model_detects_missing_consumer_free(tmp_path):
+    assert _mutant_fails(tmp_path, "      w.store(0, std::memory_order_relaxed);  // free (same address: after the read)\n",
+                         "", "ring_nofree"), "the model accepted a consumer that never frees a slot"
+
+
+def test_ring_model_detects_producer_not_waiting(tmp_path):
+    assert _mutant_fails(tmp_path, "        while (w.load(std::memory_order_relaxed) != 0) std::this_thread::yield();",
+                         "        ;", "ring_nowait"), "the model accepted a producer that overwrites unconsumed records"
