@@ -54,6 +54,8 @@ def lib():
         L.orc_fwt_f64.argtypes = [P, I, P]
         L.orc_fwt_f32dag.argtypes = [P, I, P]
         L.orc_prefixsum_u32.argtypes = [P, I, P]
+        L.orc_prefixsum_u32_excl.argtypes = [P, I, P]
+        L.orc_prefixsum_f64.argtypes = [P, I, ctypes.c_int, P, P]
         L.orc_reduction_u32.argtypes = [P, I]
         L.orc_reduction_u32.restype = ctypes.c_uint64
         L.orc_transpose_u32.argtypes = [P, I, I, P]
@@ -139,11 +141,20 @@ def fwt_f32dag(x: np.ndarray) -> np.ndarray:
     return y
 
 
-def prefixsum_u32(x: np.ndarray) -> np.ndarray:
+def prefixsum_u32(x: np.ndarray, exclusive: bool = False) -> np.ndarray:
     x = np.ascontiguousarray(x, dtype=np.uint32)
     y = np.empty(x.size, np.uint32)
-    lib().orc_prefixsum_u32(_p(x), x.size, _p(y))
+    (lib().orc_prefixsum_u32_excl if exclusive else lib().orc_prefixsum_u32)(_p(x), x.size, _p(y))
     return y
+
+
+def prefixsum_f64(x: np.ndarray, exclusive: bool = False):
+    """fp64 scan of fp32 inputs and its conditioning bound sum |x_j| (oracle.c)."""
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    y = np.empty(x.size, np.float64)
+    b = np.empty(x.size, np.float64)
+    lib().orc_prefixsum_f64(_p(x), x.size, 1 if exclusive else 0, _p(y), _p(b))
+    return y, b
 
 
 def reduction_u32(x: np.ndarray) -> int:

@@ -178,6 +178,27 @@ void orc_prefixsum_u32(const uint32_t* x, int64_t n, uint32_t* y) {
     for (int64_t i = 0; i < n; ++i) { acc += x[i]; y[i] = acc; }
 }
 
+/* Exclusive form (SURVEY 8(c) PrefixSum reading (1): "inclusive, with an
+ * exclusive flag"; exclusive = shift): y_i = sum_{j<i} x_j mod 2^32. */
+void orc_prefixsum_u32_excl(const uint32_t* x, int64_t n, uint32_t* y) {
+    uint32_t acc = 0;
+    for (int64_t i = 0; i < n; ++i) { y[i] = acc; acc += x[i]; }
+}
+
+/* fp32 secondary (SURVEY 8(c) PrefixSum reading (2): the SDK scan is fp32): the
+ * definition in fp64, y_i = sum_{j<=i} x_j (exclusive: j < i), plus the
+ * conditioning bound b_i = sum |x_j| over the same range, against which the
+ * kernel's fixed-association fp32 scan is checked (|dy_i| <= 1e-5 b_i). */
+void orc_prefixsum_f64(const float* x, int64_t n, int exclusive, double* y, double* b) {
+    double acc = 0.0, abs_acc = 0.0;
+    for (int64_t i = 0; i < n; ++i) {
+        if (exclusive) { y[i] = acc; b[i] = abs_acc; }
+        acc += (double)x[i];
+        abs_acc += fabs((double)x[i]);
+        if (!exclusive) { y[i] = acc; b[i] = abs_acc; }
+    }
+}
+
 /* ------------------------------------------------------------------------ */
 /* Reduction ("R"; R-RED1 u32 inputs, exact u64 result)               */
 /* ------------------------------------------------------------------------ */

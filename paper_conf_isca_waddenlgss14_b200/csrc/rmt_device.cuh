@@ -52,7 +52,10 @@ constexpr unsigned long long WATCHDOG_CYCLES = 1ull << 32;  // default Ctx::wd: 
 constexpr int STRESS_TAGS = 1, STRESS_SKEW = 2, STRESS_DROP = 4;
 // ctrl[] words of the inter queue control block
 constexpr int CTRL_TICKET = 0, CTRL_DONE = 1, CTRL_WATCHDOG = 2;
-constexpr int INTER_SLOTS_MAX = 8;  // slots allocated per (region, warp); Ctx::S <= this
+#ifndef RMT_INTER_SLOTS
+#define RMT_INTER_SLOTS 8
+#endif
+constexpr int INTER_SLOTS_MAX = RMT_INTER_SLOTS;  // slots allocated per (region, warp); Ctx::S <= this
 // inter_cluster: record slots per warp in the consumer CTA's shared memory
 // (Ctx::S, a power of two chosen by the launcher): 8 lets the producer fill one
 // deferred batch (<= 4 records) while the consumer drains the previous one; 4

@@ -160,6 +160,11 @@ def prefixsum_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
     return (u32(seed, n, offset, stream=4) & np.uint32(0xFF)).astype(np.uint32)
 
 
+def prefixsum_f32(seed: int, n: int, offset: int = 0) -> np.ndarray:
+    """fp32 PrefixSum input (SURVEY 8(d) configs[1]: "+f32 U[0,1)")."""
+    return uniform_f32(seed + 1000, n, offset)
+
+
 def reduction_x(seed: int, n: int, offset: int = 0) -> np.ndarray:
     """u32 U{0..2^16-1}."""
     return (u32(seed, n, offset, stream=5) & np.uint32(0xFFFF)).astype(np.uint32)

@@ -230,6 +230,42 @@ def test_prefixsum_differencing_and_library():
     assert np.array_equal(y, np.cumsum(x, dtype=np.uint32))
 
 
+def test_prefixsum_exclusive_closed_forms():
+    """Exclusive scan (SURVEY 8(c) PrefixSum reading (1)): x = 1 -> y_i = i;
+    x_i = i -> i(i-1)/2 mod 2^32; y_0 = 0; differences recover the input."""
+    n = 1 << 17
+    assert np.array_equal(oracle.prefixsum_u32(np.ones(n, np.uint32), exclusive=True), np.arange(n, dtype=np.uint32))
+    i = np.arange(n, dtype=np.uint64)
+    y = oracle.prefixsum_u32(i.astype(np.uint32), exclusive=True)
+    assert np.array_equal(y, ((i * (i - 1) // 2) % 2**32).astype(np.uint32))
+    x = inputs.prefixsum_x(4, 50001)
+    y = oracle.prefixsum_u32(x, exclusive=True)
+    assert y[0] == 0 and np.array_equal(np.diff(y.astype(np.int64)) % 2**32, x[:-1].astype(np.int64))
+    assert oracle.prefixsum_u32(np.zeros(0, np.uint32), exclusive=True).size == 0
+
+
+def test_prefixsum_f64_closed_forms_and_library():
+    """fp64 oracle of the fp32 scan: integer-valued inputs are exact (x = 1 ->
+    i + 1; alternating +-1 -> 1, 0, 1, 0, ...), random inputs equal numpy's fp64
+    cumulative sum to the last bit of a few ulps, the bound is the cumulative sum
+    of |x|, exclusive is the shift with y_0 = b_0 = 0."""
+    n = 100003
+    y, b = oracle.prefixsum_f64(np.ones(n, np.float32))
+    assert np.array_equal(y, np.arange(1, n + 1, dtype=np.float64)) and np.array_equal(b, y)
+    alt = np.where(np.arange(n) % 2 == 0, 1.0, -1.0).astype(np.float32)
+    y, b = oracle.prefixsum_f64(alt)
+    assert np.array_equal(y, (np.arange(n) % 2 == 0).astype(np.float64))
+    assert np.array_equal(b, np.arange(1, n + 1, dtype=np.float64))
+    rng = np.random.default_rng(9)
+    x = rng.uniform(-1, 1, n).astype(np.float32)
+    y, b = oracle.prefixsum_f64(x)
+    ref = np.cumsum(x.astype(np.float64))
+    assert np.max(np.abs(y - ref)) <= 1e-9
+    assert np.allclose(b, np.cumsum(np.abs(x.astype(np.float64))), rtol=1e-12)
+    ye, be = oracle.prefixsum_f64(x, exclusive=True)
+    assert ye[0] == 0.0 and be[0] == 0.0 and np.array_equal(ye[1:], y[:-1]) and np.array_equal(be[1:], b[:-1])
+
+
 def test_reduction_closed_forms():
     n = (1 << 20) + 37
     assert oracle.reduction_u32(np.full(n, 7, np.uint32)) == 7 * n
