@@ -124,7 +124,11 @@ typedef struct {
  *   PREFIXSUM     buf {x:U32[n], y:U32[n]}  inclusive, mod 2^32     n, dims {carry_in} (u32 added
  *                 to every y: the exclusive prefix of earlier shards in a multi-GPU scan; 0 = none);
  *                 optional buf[2] totals:U64[G] (every rank's total, all-gathered on the device)
- *                 with dims {carry_in, rank}: totals[0 .. rank) are added too (no host round trip)
+ *                 with dims {carry_in, rank}: totals[0 .. rank) are added too (no host round trip);
+ *                 dims[2] flags: bit 0 EXCLUSIVE (y_i = sum_{j<i} x_j), bit 1 FP32 (x, y F32; a
+ *                 fixed association order identical in every variant: 16-element thread runs,
+ *                 16-lane Kogge-Stone segments, sequential tiles, reduce-then-scan chunks;
+ *                 SURVEY 8(c) PrefixSum readings (1)-(2); FP32 takes no carry_in / totals)
  *   REDUCTION     buf {x:U32[n], s:U64[1]}                          n
  *   TRANSPOSE     buf {A:U32|F32[H*W], B:same[W*H]}                 n = H*W, dims {H, W}, H%4 = W%4 = 0
  *   SOBEL         buf {I:U8X4[H*W], O:U8X4[H*W]}                    n = H*W, dims {H, W}, W%4 = 0

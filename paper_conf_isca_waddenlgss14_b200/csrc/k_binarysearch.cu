@@ -337,13 +337,61 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? BINS_MI
   rep.finish();
 }
 
+// ---- ghost mode (dims[2] = 1; SURVEY 8(c) BinarySearch reading (1)): the APP
+// SDK's single-key segment search, where "many work-items never execute a
+// global write".  Logical CTA j searches key q[j]: logical thread t owns
+// the segment [lo_t, hi_t) of A (256 near-equal segments) and checks whether
+// lower_bound(A, q[j]) falls in it -- (lo_t == 0 or A[lo_t - 1] < key) and
+// (hi_t == N or key <= A[hi_t - 1]), so exactly one thread (the last non-empty
+// segment for lower_bound = N; thread 0 when N = 0) qualifies -- and only that
+// thread binary-searches its segment and stores idx[j].  Every warp commits once
+// (warp-collective), all lanes but the writer with an empty predicate.
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_ghost_kernel(BsArgs a, Ctx c) {
+  __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  for (; rep.active(); rep.advance()) {
+    const unsigned jq = (unsigned)rep.lblock;
+    unsigned key = a.q[jq];
+    if constexpr (M == M_FAULT) key = rep.fault(SITE_LOAD, (long long)jq, key);
+    const unsigned t = (unsigned)rep.ltid;
+    const unsigned seg = (a.N + BL - 1) / BL;
+    const unsigned lo = min(a.N, t * seg), hi = min(a.N, lo + seg);
+    bool writer;
+    if (a.N == 0u) {
+      writer = t == 0u;
+    } else {
+      const bool ge_lo = lo == 0u || (lo < a.N && a.A[lo - 1] < key) || (lo == a.N && a.A[a.N - 1] < key);
+      const bool lt_hi = hi > lo && (hi == a.N || key <= a.A[hi - 1]);
+      writer = ge_lo && lt_hi;
+    }
+    unsigned pos = lo;
+    if (writer) {  // lower_bound inside [lo, hi]: binary search of the segment
+      unsigned l = lo, h = hi;
+      while (l < h) {
+        const unsigned m = l + (h - l) / 2;
+        if (a.A[m] < key) l = m + 1;
+        else h = m;
+      }
+      pos = l;
+    }
+    if constexpr (M == M_FAULT) pos = rep.fault(SITE_COMPUTE, (long long)jq, pos);
+    unsigned w[1] = {pos};
+    rep.template commit<1, 0, false, true>(writer ? 1u : 0u, jq, w, a.Q,
+                                           [&](unsigned i, unsigned, const unsigned* x) { a.idx[i] = x[0]; });
+  }
+  rep.finish();
+}
+
 }  // namespace
 
 int binarysearch_validate(const rmt_bufs_t* b, int64_t n) {
   int64_t N = b->dims[0], Q = b->dims[1];
   if (b->nbuf < 3 || N < 0 || N >= (1LL << 32) - 64 || Q < 0 || Q >= (1LL << 30) || n != Q ||
+      (b->dims[2] != 0 && b->dims[2] != 1) ||
       !buf_ok(b->buf[0], RMT_U32, N) || !buf_ok(b->buf[1], RMT_U32, Q) || !buf_ok(b->buf[2], RMT_U32, Q)) {
-    set_error("binarysearch: expected {A:U32[N], q:U32[Q], idx:U32[Q]}, dims {N,Q}, n = Q");
+    set_error("binarysearch: expected {A:U32[N], q:U32[Q], idx:U32[Q]}, dims {N, Q, mode}, n = Q, mode 0 batched | 1 ghost");
     return RMT_EINVAL;
   }
   return RMT_OK;
@@ -375,6 +423,12 @@ int binarysearch_run(Launch& L) {
   a.iters = (chunks + 148u * 8u - 1u) / (148u * 8u);
   if (a.iters == 0) a.iters = 1;
   const unsigned G = (chunks + a.iters - 1) / a.iters;
+  if (L.bufs->dims[2] == 1)  // ghost mode: one logical CTA per key, no index
+    return dispatch(L.variant, L.mode, [&](auto vm) {
+      constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+      return launch_std<V>(L, bins_ghost_kernel<V, M>, bins_ghost_kernel<V_NONE, M_NORMAL>, Q, BL, 0, a,
+                           "binarysearch/ghost");
+    });
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     int rc = RMT_OK;

@@ -35,6 +35,7 @@ struct PsArgs {
   unsigned v8;         // x is 32-B aligned: 256-bit loads where a thread's run allows
   const unsigned long long* totals;  // multi-GPU: every rank's total (all-gathered on the device), or null
   unsigned rank;       // totals[0 .. rank) are added to the carry (mod 2^32)
+  unsigned excl;       // exclusive scan (y_i = sum_{j<i} x_j)
 };
 
 // u32 sum over the logical CTA (logical warps + duplicated smem)
@@ -247,7 +248,10 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_k
         unsigned mask = 0;
 #pragma unroll
         for (int k = 0; k < 4; ++k) {
-          w[k] = prefix + v[4 * i + k];
+          // exclusive: the run's inclusive value one element back (0 at a run start)
+          const int ii = 4 * i + k;
+          const unsigned vx = (ii % RUN == 0) ? 0u : v[ii > 0 ? ii - 1 : 0];
+          w[k] = prefix + (a.excl ? vx : v[ii]);
           mask |= (e0 + k < hi ? 1u : 0u) << k;
         }
         rep.template commit<4, 0>(mask, mask ? e0 : 0u, w, a.n, [&](unsigned idx, unsigned m, const unsigned* x) {
@@ -263,11 +267,180 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_k
   rep.finish();
 }
 
+// ---------------------------------------------------------------- fp32 scan
+// The fp32 secondary (reading R-PS3): one FIXED association order, identical in
+// every variant, so the replicas (and none) are bitwise equal and the result is
+// deterministic -- a thread scans its RUN = 16 consecutive elements sequentially,
+// segments of 16 logical lanes scan the thread totals Kogge-Stone (d = 1, 2, 4,
+// 8), the 16 segment totals of a tile are scanned the same way, tiles chain
+// sequentially inside a chunk, and a chunk's carry-in is the sum of the earlier
+// chunks' partials (lane l of a segment sums partials l, l + 16, ... in order,
+// then a 16-lane xor tree -- IEEE addition commutes, so every lane holds the
+// same bits).  A 32-lane (none / inter) warp is two 16-lane segments doing the
+// same work as a 16-lane intra logical warp.  No look-back: its order would
+// depend on timing.
+constexpr int FSEG = 16;
+
+template <class R>
+__device__ __forceinline__ float fadd_seg_scan(const R& rep, float x) {  // inclusive, 16-lane segments
+#pragma unroll
+  for (int d = 1; d < FSEG; d <<= 1) {
+    const float u = __uint_as_float(rep.lshfl_up(__float_as_uint(x), d));
+    if ((rep.llane & (FSEG - 1)) >= d) x = __fadd_rn(u, x);
+  }
+  return x;
+}
+template <class R>
+__device__ __forceinline__ float fadd_seg_all(const R& rep, float x) {  // the same total in every lane
+#pragma unroll
+  for (int m = FSEG / 2; m >= 1; m >>= 1) x = __fadd_rn(x, __uint_as_float(rep.lshfl_xor(__float_as_uint(x), m)));
+  return x;
+}
+// Fixed-order fp32 sum over the logical CTA's 256 logical threads: segment xor
+// trees, then the 16 segment totals (shared memory) by the same tree.
+template <class R>
+__device__ __forceinline__ float block_sum_f32(const R& rep, float s, unsigned* sw) {
+  s = fadd_seg_all(rep, s);
+  const unsigned seg = (unsigned)rep.ltid / FSEG;
+  if ((rep.llane & (FSEG - 1)) == 0 && rep.sts_ok1(__float_as_uint(s), seg)) rep.sm(sw, seg) = __float_as_uint(s);
+  __syncthreads();
+  float t = __uint_as_float(rep.sm(sw, rep.llane & (FSEG - 1)));
+  t = fadd_seg_all(rep, t);
+  __syncthreads();
+  return t;
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_reduce_f32_kernel(PsArgs a, Ctx c) {
+  __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  __shared__ unsigned sw[FSEG * Geom<V>::SMDUP];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const float* x = reinterpret_cast<const float*>(a.x);
+  for (; rep.active(); rep.advance()) {
+    const unsigned ch = (unsigned)rep.lblock;
+    const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
+    float s = 0.0f;
+    // thread t sums elements lo + TILE b + 16 t .. + 15 of every tile b, in order
+#pragma unroll 1
+    for (unsigned t0 = lo; t0 < hi; t0 += TILE) {
+      const unsigned e = t0 + ITEMS * (unsigned)rep.ltid;
+      float v[ITEMS];
+      if (e + ITEMS <= hi) {
+#pragma unroll
+        for (int j = 0; j < ITEMS / 4; ++j) {
+          const float4 w = __ldg(reinterpret_cast<const float4*>(x + e) + j);
+          v[4 * j] = w.x; v[4 * j + 1] = w.y; v[4 * j + 2] = w.z; v[4 * j + 3] = w.w;
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < ITEMS; ++k) v[k] = e + k < hi ? x[e + k] : 0.0f;
+      }
+#pragma unroll
+      for (int k = 0; k < ITEMS; ++k) {
+        if constexpr (M == M_FAULT) v[k] = rep.faultf(SITE_LOAD, (long long)e + k, v[k]);
+        s = __fadd_rn(s, v[k]);
+      }
+    }
+    s = rep.faultf(SITE_COMPUTE, (long long)ch * BL + rep.ltid, s);
+    const float t = block_sum_f32(rep, s, sw);
+    if (rep.warp == 0) {  // one store per CTA leaves the SoR ("ghost" warps)
+      unsigned w[1] = {__float_as_uint(t)};
+      rep.template commit<1, 2>(rep.llane == 0 ? 1u : 0u, ch, w, a.nch,
+                                [&](unsigned i, unsigned, const unsigned* xx) { a.partial[i] = xx[0]; });
+    }
+  }
+  rep.finish();
+}
+
+template <int V, int M>
+__global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_scan_f32_kernel(PsArgs a, Ctx c) {
+  __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
+  __shared__ unsigned sw[FSEG * Geom<V>::SMDUP];
+  Rep<V, M> rep(c);
+  rep.init(mb);
+  const float* x = reinterpret_cast<const float*>(a.x);
+  for (; rep.active(); rep.advance()) {
+    const unsigned ch = a.nch - 1u - (unsigned)rep.lblock;  // reverse order: L2-hot chunks first
+    // carry-in: the earlier chunks' partials, lane l of every segment summing
+    // partials l, l + 16, ... in order, then the segment's xor tree
+    float cs = 0.0f;
+    for (unsigned i = rep.llane & (FSEG - 1); i < ch; i += FSEG) cs = __fadd_rn(cs, __uint_as_float(__ldcg(a.partial + i)));
+    float carry = fadd_seg_all(rep, cs);
+    const unsigned lo = ch * a.chunk, hi = min(a.n, lo + a.chunk);
+    const unsigned seg = (unsigned)rep.ltid / FSEG;
+#pragma unroll 1
+    for (unsigned t0 = lo; t0 < hi; t0 += TILE) {  // uniform trip count per CTA
+      const unsigned e = t0 + ITEMS * (unsigned)rep.ltid;
+      float v[ITEMS];
+      if (e + ITEMS <= hi) {
+#pragma unroll
+        for (int j = 0; j < ITEMS / 4; ++j) {
+          const float4 w = __ldcs(reinterpret_cast<const float4*>(x + e) + j);
+          v[4 * j] = w.x; v[4 * j + 1] = w.y; v[4 * j + 2] = w.z; v[4 * j + 3] = w.w;
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < ITEMS; ++k) v[k] = e + k < hi ? x[e + k] : 0.0f;
+      }
+      if constexpr (M == M_FAULT) {
+#pragma unroll
+        for (int k = 0; k < ITEMS; ++k) v[k] = rep.faultf(SITE_LOAD, (long long)e + k, v[k]);
+      }
+#pragma unroll
+      for (int k = 1; k < ITEMS; ++k) v[k] = __fadd_rn(v[k - 1], v[k]);  // the thread's run, in order
+      const float ws = fadd_seg_scan(rep, v[ITEMS - 1]);               // segment-inclusive thread totals
+      float ex = __uint_as_float(rep.lshfl_up(__float_as_uint(ws), 1));
+      if ((rep.llane & (FSEG - 1)) == 0) ex = 0.0f;                    // segment-exclusive
+      if ((rep.llane & (FSEG - 1)) == FSEG - 1 && rep.sts_ok1(__float_as_uint(ws), seg))
+        rep.sm(sw, seg) = __float_as_uint(ws);
+      __syncthreads();
+      float wt = __uint_as_float(rep.sm(sw, rep.llane & (FSEG - 1)));  // the tile's 16 segment totals
+      if constexpr (M == M_FAULT) wt = rep.faultf(SITE_SMEM, (long long)ch * BL + (rep.llane & (FSEG - 1)), wt);
+      const float winc = fadd_seg_scan(rep, wt);
+      const int g0 = rep.llane & ~(FSEG - 1);
+      // (the shuffle runs in every lane -- warp-collective -- and segment 0 discards it)
+      const unsigned segw = rep.lshfl_idx(__float_as_uint(winc), g0 + (seg == 0u ? 0 : (int)seg - 1));
+      const float segpre = seg == 0u ? 0.0f : __uint_as_float(segw);
+      const float total = __uint_as_float(rep.lshfl_idx(__float_as_uint(winc), g0 + FSEG - 1));
+      __syncthreads();  // sw is reused by the next tile
+      const float base = __fadd_rn(__fadd_rn(carry, segpre), ex);
+#pragma unroll
+      for (int i = 0; i < ITEMS / 4; ++i) {
+        const unsigned e0 = e + 4 * i;
+        unsigned w[4];
+        unsigned mask = 0;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int ii = 4 * i + k;
+          const float yi = a.excl ? (ii == 0 ? base : __fadd_rn(base, v[ii > 0 ? ii - 1 : 0])) : __fadd_rn(base, v[ii]);
+          w[k] = __float_as_uint(yi);
+          mask |= (e0 + k < hi ? 1u : 0u) << k;
+        }
+        rep.template commit<4, 0>(mask, mask ? e0 : 0u, w, a.n, [&](unsigned idx, unsigned m, const unsigned* xx) {
+          if (m == 0xFu) __stcs(reinterpret_cast<uint4*>(a.y + idx), make_uint4(xx[0], xx[1], xx[2], xx[3]));
+          else
+            for (int k = 0; k < 4; ++k)
+              if ((m >> k) & 1u) a.y[idx + k] = xx[k];
+        }, /*defer=*/i < ITEMS / 4 - 1);
+      }
+      carry = __fadd_rn(carry, total);
+    }
+  }
+  rep.finish();
+}
+
 }  // namespace
 
 int prefixsum_validate(const rmt_bufs_t* b, int64_t n) {
   const bool tot = b->nbuf >= 3 && b->buf[2].ptr != nullptr;
-  if (b->nbuf < 2 || n < 0 || n >= (1LL << 30) || !buf_ok(b->buf[0], RMT_U32, n) || !buf_ok(b->buf[1], RMT_U32, n) ||
+  const int64_t flags = b->dims[2];
+  const int dt = (flags & 2) ? RMT_F32 : RMT_U32;
+  if ((flags & ~3LL) != 0 || ((flags & 2) && (tot || b->dims[0] != 0))) {
+    set_error("prefixsum: dims[2] flags are bit 0 exclusive, bit 1 fp32 (fp32: no carry_in, no totals)");
+    return RMT_EINVAL;
+  }
+  if (b->nbuf < 2 || n < 0 || n >= (1LL << 30) || !buf_ok(b->buf[0], dt, n) || !buf_ok(b->buf[1], dt, n) ||
       (tot && (b->buf[2].dtype != RMT_U64 || ((uintptr_t)b->buf[2].ptr % 16) != 0 || b->dims[1] < 0 ||
                b->dims[1] > b->buf[2].numel))) {
     set_error("prefixsum: expected {x,y} U32[n], n < 2^30, dims {carry_in}; optionally totals:U64[G] with dims "
@@ -288,9 +461,18 @@ int prefixsum_run(Launch& L) {
   const unsigned nch = (n + chunk - 1) / chunk;
   PsArgs a{(const unsigned*)L.bufs->buf[0].ptr, (unsigned*)L.bufs->buf[1].ptr, (unsigned*)L.scratch, n, chunk, nch,
            (unsigned)(L.bufs->dims[0] & 0xFFFFFFFFu), ((uintptr_t)L.bufs->buf[0].ptr % 32) == 0 ? 1u : 0u,
-           L.bufs->nbuf >= 3 ? (const unsigned long long*)L.bufs->buf[2].ptr : nullptr, (unsigned)L.bufs->dims[1]};
+           L.bufs->nbuf >= 3 ? (const unsigned long long*)L.bufs->buf[2].ptr : nullptr, (unsigned)L.bufs->dims[1],
+           (unsigned)(L.bufs->dims[2] & 1)};
+  const bool f32 = (L.bufs->dims[2] & 2) != 0;
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
+    if (f32) {
+      int rc = launch_std<V>(L, ps_reduce_f32_kernel<V, M>, ps_reduce_f32_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a,
+                             "prefixsum/reduce_f32");
+      if (rc) return rc;
+      return launch_std<V>(L, ps_scan_f32_kernel<V, M>, ps_scan_f32_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a,
+                           "prefixsum/scan_f32");
+    }
     int rc = launch_std<V>(L, ps_reduce_kernel<V, M>, ps_reduce_kernel<V_NONE, M_NORMAL>, nch, BL, 0, a,
                            "prefixsum/reduce");
     if (rc) return rc;

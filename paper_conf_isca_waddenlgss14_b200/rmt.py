@@ -33,7 +33,7 @@ SCHEMA = {
     "blackscholes": (F32, F32, F32),
     "binarysearch": (U32, U32, U32),
     "fwt": (F32, F32),
-    "prefixsum": (U32, U32),
+    "prefixsum": (None, None),  # U32, or F32 with dims[2] bit 1 (include/rmt.h)
     "reduction": (U32, U64),
     "transpose": (None, None),
     "sobel": (U8X4, U8X4),

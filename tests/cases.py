@@ -225,23 +225,34 @@ class Transpose(Case):
 class PrefixSum(Case):
     kernel = "prefixsum"
 
-    def __init__(self, n, seed=4, x=None):
+    def __init__(self, n, seed=4, x=None, exclusive=False, f32=False):
         self.n = n
-        self.x = inputs.prefixsum_x(seed, n) if x is None else x
+        self.exclusive, self.f32 = exclusive, f32
+        self.dims = (0, 0, (1 if exclusive else 0) | (2 if f32 else 0))
+        self.tag = ("-excl" if exclusive else "") + ("-f32" if f32 else "")
+        if x is None:
+            x = inputs.prefixsum_f32(seed, n) if f32 else inputs.prefixsum_x(seed, n)
+        self.x = x
 
     @functools.cached_property
     def x_d(self):
-        return dev(self.x if self.n else np.zeros(4, np.uint32))
+        return dev(self.x if self.n else np.zeros(4, self.x.dtype))
 
     def buffers(self):
-        return [self.x_d[: self.n], out_like(4 * max(self.n, 1))[: self.n]]
+        y = out_like(4 * max(self.n, 1))[: self.n]
+        return [self.x_d[: self.n], y.view(torch.float32) if self.f32 else y]
 
     def outputs(self, b):
         return [host(b[1], np.uint32)]
 
     def check(self, outs, x=None):
         x = self.x if x is None else x
-        assert np.array_equal(outs[0], oracle.prefixsum_u32(x))
+        if self.f32:  # fp64 definition, |dy_i| <= 1e-5 sum |x_j| (SURVEY 8(c) PrefixSum fp32 parity rule)
+            ref, bound = oracle.prefixsum_f64(x, exclusive=self.exclusive)
+            got = outs[0].view(np.float32).astype(np.float64)
+            assert np.all(np.abs(got - ref) <= 1e-5 * bound + 1e-30), np.max(np.abs(got - ref) / (bound + 1e-30))
+        else:
+            assert np.array_equal(outs[0], oracle.prefixsum_u32(x, exclusive=self.exclusive))
 
     def flipped_oracle(self, elem, bit):
         return [oracle.prefixsum_u32(_flip(self.x, elem, bit))]
@@ -314,10 +325,12 @@ class FWT(Case):
 class BinarySearch(Case):
     kernel = "binarysearch"
 
-    def __init__(self, N, Q, seed=6, odd=False, dups=False):
+    def __init__(self, N, Q, seed=6, odd=False, dups=False, ghost=False):
         self.N, self.Q = N, Q
         self.n = Q
-        self.dims = (N, Q)
+        # ghost: the single-key segment search, one writer per key (dims[2] = 1)
+        self.dims = (N, Q, 1) if ghost else (N, Q)
+        self.ghost = ghost
         if dups:  # runs of equal keys, 0 and 0xFFFFFFFF in A and in the queries
             self.A, self.q = inputs.binarysearch_dups(seed, N, Q)
             self.tag = "-dups"
@@ -327,6 +340,8 @@ class BinarySearch(Case):
         else:
             self.A, self.q = inputs.binarysearch_inputs(seed, max(N, 1), Q)
             self.A = self.A[:N]
+        if ghost:
+            self.tag += "-ghost"
 
     @functools.cached_property
     def A_d(self):
@@ -352,7 +367,9 @@ class BinarySearch(Case):
 
     def commit_group(self, e):
         # a logical thread searches 2 interleaved queries and commits them as one
-        # 8-B vector (k_binarysearch.cu)
+        # 8-B vector (k_binarysearch.cu); ghost mode commits one word per key
+        if self.ghost:
+            return np.array([e])
         lo = e - e % 2
         return np.arange(lo, min(lo + 2, self.Q))
 
@@ -645,6 +662,10 @@ def small_cases():
         Reduction(0), Reduction(3), Reduction(1000003), Reduction(1 << 22),
         Transpose(4, 4), Transpose(68, 132), Transpose(256, 512, index_coded=True), Transpose(1000, 764),
         PrefixSum(1), PrefixSum(4095), PrefixSum(4096 * 37 + 11), PrefixSum(1 << 22), PrefixSum((1 << 25) + 12347),
+        # the exclusive flag and the fixed-association fp32 scan (SURVEY 8(c) PrefixSum readings (1)-(2))
+        PrefixSum(1, exclusive=True), PrefixSum(4096 * 37 + 11, exclusive=True), PrefixSum((1 << 22) + 5, exclusive=True),
+        PrefixSum(1, f32=True), PrefixSum(4095, f32=True), PrefixSum(4096 * 37 + 11, f32=True),
+        PrefixSum((1 << 22) + 3, f32=True, exclusive=True), PrefixSum(1 << 24, f32=True),
         FWT(1), FWT(2), FWT(64), FWT(4096), FWT(1 << 13), FWT(1 << 19), FWT(1 << 20), FWT(1 << 16, ternary=True),
         FWT(1 << 15, specials=True), FWT(64, specials=True),
         BinarySearch(0, 16), BinarySearch(1, 7), BinarySearch(1000, 1003), BinarySearch(1 << 16, 50000, odd=True),
@@ -655,6 +676,9 @@ def small_cases():
         # shared-memory table edges (k_binarysearch.cu): n_T = 8192 = P exactly
         # (no padding entry: the final compare), and three sample levels (T = 3)
         BinarySearch(1 << 18, 3001), BinarySearch((8 << 20) + 7, 40000),
+        # ghost (single-key segment search): empty A, N < 256 (empty segments), keys past the end, duplicates
+        BinarySearch(0, 16, ghost=True), BinarySearch(17, 999, ghost=True), BinarySearch(1000, 1003, ghost=True),
+        BinarySearch(1 << 16, 3000, odd=True, ghost=True), BinarySearch(4096 * 3 + 7, 2001, dups=True, ghost=True),
         Sobel(3, 4), Sobel(37, 100), Sobel(100, 1028, noise=True), Sobel(256, 2048),
         DCT(8, 8), DCT(24, 264), DCT(512, 2048 + 8), DCT(64, 512, specials=True),
         FloydWarshall(4), FloydWarshall(52), FloydWarshall(256),

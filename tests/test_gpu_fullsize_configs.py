@@ -106,6 +106,36 @@ def test_suite28_fullsize(kernel):
     _release(j)
 
 
+def test_prefixsum_f32_fullsize():
+    """The fp32 PrefixSum (fixed association, dims[2] bit 1) at the suite size
+    2^26, inclusive and exclusive: within 1e-5 of the fp64 definition scaled by
+    sum |x_j|, every variant bitwise equal to none."""
+    n = 1 << 26
+    x = inputs.prefixsum_f32(4, n)
+    xd = torch.from_numpy(x).cuda()
+    y = torch.empty(n, dtype=torch.float32, device="cuda")
+    for excl in (False, True):
+        dims = (0, 0, 2 | (1 if excl else 0))
+        ref = None
+        for v in ["none", *VARIANTS]:
+            y.fill_(float("nan"))
+            err = torch.zeros(1, dtype=torch.int64, device="cuda")
+            ws = rmt.make_workspace("prefixsum", v, n, dims)
+            rmt.launch("prefixsum", v, [xd, y], n, err, dims=dims, workspace=ws)
+            torch.cuda.synchronize()
+            got = y.cpu().numpy().view(np.uint32).copy()
+            assert int(err.item()) == 0, f"prefixsum f32/{v}: false alarms"
+            if ref is None:
+                ref = got
+                yo, bo = oracle.prefixsum_f64(x, exclusive=excl)
+                d = np.abs(got.view(np.float32).astype(np.float64) - yo)
+                assert np.all(d <= 1e-5 * bo + 1e-30), float(np.max(d / (bo + 1e-30)))
+            else:
+                assert np.array_equal(got, ref), f"prefixsum f32/{v} differs from none"
+    del xd, y
+    torch.cuda.empty_cache()
+
+
 # ---------------------------------------------------------------- configs[3]
 def test_floydwarshall_4096_fullsize():
     j = workloads.job_floydwarshall(4096)
