@@ -14,7 +14,9 @@ from cases import (DCT, DWT, FWT, BinarySearch, BinomialOption, BitonicSort, Bla
                    FloydWarshall, MatMul, PrefixSum, Reduction, Sobel, Transpose)
 from helpers import run  # noqa: E402
 
-cases = [BlackScholes(3000), BlackScholesIndep(1024), BinarySearch(5000, 1000), FWT(1 << 13), PrefixSum(4096 * 3 + 7),
+cases = [BlackScholes(3000), BlackScholesIndep(1024), BinarySearch(5000, 1000), BinarySearch(300000, 1000),
+         BinarySearch(5000, 300, ghost=True), FWT(1 << 13), PrefixSum(4096 * 3 + 7),
+         PrefixSum(4096 * 3 + 7, exclusive=True), PrefixSum(4096 * 3 + 7, f32=True),
          Reduction(100003), Transpose(68, 132), Sobel(37, 100), DCT(24, 264), FloydWarshall(52),
          MatMul(128, 256, 128), DWT(1 << 13), BitonicSort(1 << 13), BinomialOption(300)]
 variants = ("none",) + rmt.RMT_VARIANTS
