@@ -91,28 +91,28 @@ Levels make_levels(unsigned N) {
 // (sub.cc: carry = no borrow = w >= k), summed with addc -- two integer-pipe
 // instructions per word instead of a compare, a select and a bit-combine.
 __device__ __forceinline__ unsigned count_ge8(const unsigned (&w)[8], unsigned k) {
-  unsigned c, t;
+  unsigned c;
   asm("{\n\t"
-      "sub.cc.u32 %1, %2, %10;\n\t"
+      ".reg .u32 t;\n\t"  // scratch: the differences are not needed
+      "sub.cc.u32 t, %1, %9;\n\t"
       "addc.u32 %0, 0, 0;\n\t"
-      "sub.cc.u32 %1, %3, %10;\n\t"
+      "sub.cc.u32 t, %2, %9;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %4, %10;\n\t"
+      "sub.cc.u32 t, %3, %9;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %5, %10;\n\t"
+      "sub.cc.u32 t, %4, %9;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %6, %10;\n\t"
+      "sub.cc.u32 t, %5, %9;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %7, %10;\n\t"
+      "sub.cc.u32 t, %6, %9;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %8, %10;\n\t"
+      "sub.cc.u32 t, %7, %9;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
-      "sub.cc.u32 %1, %9, %10;\n\t"
+      "sub.cc.u32 t, %8, %9;\n\t"
       "addc.u32 %0, %0, 0;\n\t"
       "}"
-      : "=r"(c), "=&r"(t)
+      : "=r"(c)
       : "r"(w[0]), "r"(w[1]), "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7]), "r"(k));
-  (void)t;  // scratch register of the asm (the differences are not needed)
   return c;
 }
 
