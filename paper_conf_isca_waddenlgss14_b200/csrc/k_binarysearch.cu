@@ -181,6 +181,9 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
 #ifndef BINS_MINB
 #define BINS_MINB 4
 #endif
+#ifndef BINS_WAVES
+#define BINS_WAVES 8u  // logical CTAs per SM (the table copy is amortised over the rest)
+#endif
 #ifndef BINS_GROUP
 #define BINS_GROUP 1
 #endif
@@ -420,7 +423,7 @@ int binarysearch_run(Launch& L) {
   const unsigned Gi = (a.L.vecs_before[a.L.T + 1] + FAN / 4 + BL - 1) / BL;
   const unsigned chunks = (Q + CHUNK - 1) / CHUNK;
   // about 8 waves of logical CTAs: the table copy is amortised over a.iters chunks
-  a.iters = (chunks + 148u * 8u - 1u) / (148u * 8u);
+  a.iters = (chunks + 148u * BINS_WAVES - 1u) / (148u * BINS_WAVES);
   if (a.iters == 0) a.iters = 1;
   const unsigned G = (chunks + a.iters - 1) / a.iters;
   if (L.bufs->dims[2] == 1)  // ghost mode: one logical CTA per key, no index
