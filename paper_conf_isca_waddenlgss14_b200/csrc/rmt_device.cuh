@@ -795,6 +795,14 @@ struct Rep {
           return;
         }
       }
+      if constexpr (INTRA && COND) {
+        // A conditional store site where no lane of the warp stores -- in EITHER
+        // replica: both sit in this warp -- has nothing to exchange: every
+        // predicate already agrees.  One vote instead of the key
+        // exchange and compare (a fault that turns a predicate on makes the vote
+        // true and takes the full path).
+        if (!__any_sync(FULL, mask != 0u)) return;
+      }
       unsigned pk = 0, pv[NW];
       bool have = true;  // consumer got the producer's record
       if constexpr (V == V_INTRA_REG || V == V_INTRA_NOLDS) {
