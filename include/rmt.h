@@ -116,7 +116,10 @@ typedef struct {
  *   BLACKSCHOLES  buf {r:F32[n], call:F32[n], put:F32[n]}           n = options, dims {mode}
  *                 mode 0: one draw r per option, (S,K,T,R,sigma) from r with S == K (DESIGN.md R-BS1)
  *                 mode 1: buf[0] = params:F32[5n], planes S | K | T | R | sigma, n%4 = 0 (R-BS4)
- *   BINARYSEARCH  buf {A:U32[N] sorted, q:U32[Q], idx:U32[Q]}       n = Q, dims {N, Q}
+ *   BINARYSEARCH  buf {A:U32[N] sorted, q:U32[Q], idx:U32[Q]}       n = Q, dims {N, Q, mode}
+ *                 idx[j] = lower_bound(A, q[j]) = #{i : A[i] < q[j]}; mode 0 = batched (every
+ *                 query stores), mode 1 = ghost: the APP SDK single-key segment search, one
+ *                 logical CTA per key and one writing work-item per key
  *   FWT           buf {x:F32[N], y:F32[N]}                          n = N = 2^m, dims {0}
  *                 dims {1, upper}: one cross-shard butterfly stage of a multi-GPU FWT,
  *                 buf {x: this shard, y: out, p: the partner shard} F32[N]; y = x + p (lower
