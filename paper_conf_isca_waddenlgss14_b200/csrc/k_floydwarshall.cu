@@ -151,6 +151,9 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) fw_pass_kernel(FwArgs a, Ct
 // barrier orders every consumer's committed D stores of pass k before any
 // replica's loads of pass k + 1.  Fault builds see per-pass fault descriptors
 // (the host encodes the pass: elem = k0 n^2 + e).
+#ifndef FW_BAR_NS
+#define FW_BAR_NS 32  // grid-barrier poll back-off (ns)
+#endif
 __device__ __forceinline__ void grid_barrier(unsigned* bar, unsigned nctas) {
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -160,7 +163,8 @@ __device__ __forceinline__ void grid_barrier(unsigned* bar, unsigned nctas) {
       bar[0] = 0u;
       st_release(bar + 1, gen + 1u);
     } else {
-      while (ld_acquire(bar + 1) == gen) __nanosleep(32);
+      while (ld_acquire(bar + 1) == gen)
+        if (FW_BAR_NS) __nanosleep(FW_BAR_NS);
     }
   }
   __syncthreads();

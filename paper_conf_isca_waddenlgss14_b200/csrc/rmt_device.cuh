@@ -203,7 +203,7 @@ __device__ __forceinline__ void cluster_sync_all() {
 // single-bit fault of the fault model -- always changes the digest; changes in
 // several words alias with probability ~2^-32.
 template <int NW>
-__device__ __forceinline__ unsigned rec_digest(unsigned key, unsigned mask, const unsigned (&v)[NW]) {
+__host__ __device__ __forceinline__ unsigned rec_digest(unsigned key, unsigned mask, const unsigned (&v)[NW]) {
   unsigned h = key * 0x9E3779B1u;
   h ^= h >> 15;
 #pragma unroll
