@@ -15,6 +15,9 @@
 // digest records: inter_group 3.10 -> 2.89x)
 #define RMT_SPIN_NS0 0
 #include "rmt_host.cuh"
+#ifndef FWT_INTER_MINB
+#define FWT_INTER_MINB 10  // inter_group: 10 CTAs of 128 per SM (51 registers; measured 3.05 -> 2.73x vs 72 registers)
+#endif
 
 namespace rmt {
 namespace {
@@ -351,7 +354,7 @@ __device__ __forceinline__ int p1x(int e) { return e ^ ((e >> 5) & 31); }
 
 
 template <int V, int M>
-__global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, Ctx c) {
+__global__ void __launch_bounds__(BLS * Geom<V>::DUP, V == V_INTER ? FWT_INTER_MINB : 0) fwt_p1_kernel(FwtArgs a, Ctx c) {
   using R = Rep<V, M, true>;  // group flags: 8 records per warp
   constexpr bool DUPL = R::SMDUP;
   constexpr bool PAD = V != V_NONE;  // layout choice (see p1_phys / p1x): measured per variant
@@ -440,7 +443,7 @@ __global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_p1_kernel(FwtArgs a, C
 // x 32 contiguous columns.  Layout e = col | row << 5 (bank = col), replica
 // planes XOR bank bit 4 (a warp's 16 logical lanes share it).
 template <int V, int M>
-__global__ void __launch_bounds__(BLS * Geom<V>::DUP) fwt_ps_kernel(FwtArgs a, Ctx c) {
+__global__ void __launch_bounds__(BLS * Geom<V>::DUP, V == V_INTER ? FWT_INTER_MINB : 0) fwt_ps_kernel(FwtArgs a, Ctx c) {
   using R = Rep<V, M, true>;  // group flags: 8 records per warp
   constexpr bool DUPL = R::SMDUP;
   __shared__ unsigned mb[mbox_words<V>(BLS * Geom<V>::DUP)];
