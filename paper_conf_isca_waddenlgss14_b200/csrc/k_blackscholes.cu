@@ -11,6 +11,9 @@
 // parameters, five F32 planes S | K | T | R | sigma of n options each (SURVEY
 // 8(c) "bs_indep": moneyness ln(S/K) != 0, negative d1/d2, deep ITM / OTM).
 #include "rmt_host.cuh"
+#ifndef BLKSCH_INTER_MINB
+#define BLKSCH_INTER_MINB 8  // inter_group: 8 CTAs of 256 per SM (32 registers): 4.01 -> 3.75x at 2^30
+#endif
 
 namespace rmt {
 namespace {
@@ -86,7 +89,7 @@ __device__ __forceinline__ void load4(const float* p, unsigned i0, unsigned n, f
 }
 
 template <int V, int M, bool IND>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP) bs_kernel(BsArgs a, Ctx c) {
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, V == V_INTER ? BLKSCH_INTER_MINB : 0) bs_kernel(BsArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M> rep(c);
   rep.init(mb);

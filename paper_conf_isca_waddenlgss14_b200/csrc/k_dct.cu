@@ -14,6 +14,9 @@
 #include <math.h>
 
 #include "rmt_host.cuh"
+#ifndef DCT_INTER_MINB
+#define DCT_INTER_MINB 0  // inter_group: minimum resident CTAs per SM (0: unspecified)
+#endif
 
 namespace rmt {
 namespace {
@@ -39,7 +42,7 @@ struct DctArgs {
 };
 
 template <int V, int M>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP) dct_kernel(DctArgs a, Ctx c) {
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, V == V_INTER ? DCT_INTER_MINB : 0) dct_kernel(DctArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   __shared__ unsigned mb[mbox_words<V>(BL * DUP)];
   __shared__ __align__(16) float Zs[Geom<V>::SMDUP == 2 ? PLANE + ZWORDS : ZWORDS];

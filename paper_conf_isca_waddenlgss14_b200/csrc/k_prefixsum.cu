@@ -15,6 +15,9 @@
 //           still L2-resident.
 // Integer addition is associative: every variant produces the identical result.
 #include "rmt_host.cuh"
+#ifndef PS_INTER_MINB
+#define PS_INTER_MINB 0  // inter_group: minimum resident CTAs per SM (0: unspecified)
+#endif
 
 namespace rmt {
 namespace {
@@ -109,7 +112,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) ps_reduce_kernel(PsArgs a, 
 }
 
 template <int V, int M>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP, 4 / Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ctx c) {
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, V == V_INTER && PS_INTER_MINB ? PS_INTER_MINB : 4 / Geom<V>::DUP) ps_scan_kernel(PsArgs a, Ctx c) {
   constexpr int DUP = Geom<V>::DUP;
   constexpr int LW = 32 / DUP;
   constexpr int NLW = BL / LW;
