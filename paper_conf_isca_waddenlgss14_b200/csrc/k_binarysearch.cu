@@ -181,6 +181,9 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
 #ifndef BINS_MINB
 #define BINS_MINB 4
 #endif
+#ifndef BINS_INTER_MINB
+#define BINS_INTER_MINB BINS_MINB
+#endif
 #ifndef BINS_WAVES
 #define BINS_WAVES 8u  // logical CTAs per SM (the table copy is amortised over the rest)
 #endif
@@ -189,7 +192,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_index_kernel(BsArgs a,
 #endif
 template <int V, int M>
 // Registers capped at 64 (4 CTAs of 256 / 2 of 512 threads per SM).
-__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? BINS_MINB / 2 : BINS_MINB) bins_kernel(BsArgs a, Ctx c) {
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? BINS_MINB / 2 : V == V_INTER ? BINS_INTER_MINB : BINS_MINB) bins_kernel(BsArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   extern __shared__ __align__(16) unsigned char bins_dyn[];
   // inter: group flags, the commits of BINS_GROUP consecutive chunks published

@@ -29,6 +29,9 @@ constexpr int BL = 256;
 #ifndef SOBEL_GROUP
 #define SOBEL_GROUP 3
 #endif
+#ifndef SOBEL_INTER_MINB
+#define SOBEL_INTER_MINB 4
+#endif
 #ifndef SOBEL_MULT_INTER
 #define SOBEL_MULT_INTER 0
 #endif
@@ -152,7 +155,7 @@ struct BoolC {
 };
 
 template <int V, int M>
-__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : 4) sobel_kernel(SobArgs a, Ctx c) {
+__global__ void __launch_bounds__(BL * Geom<V>::DUP, Geom<V>::DUP == 2 ? 2 : V == V_INTER ? SOBEL_INTER_MINB : 4) sobel_kernel(SobArgs a, Ctx c) {
   __shared__ unsigned mb[mbox_words<V>(BL * Geom<V>::DUP)];
   Rep<V, M, (SOBEL_GROUP > 1 && V == V_INTER)> rep(c);
   rep.init(mb);
