@@ -220,6 +220,25 @@ int rmt_run_host_variants(int kernel, int nvar, const int* variants, const rmt_b
                           void* const* workspaces, const size_t* ws_bytes, void* stream, int64_t* h2d_bytes,
                           int64_t* d2h_bytes);
 
+/*
+ * rmt_run_host_variants_pipelined -- rmt_run_host_variants without the host
+ * synchronisation, on three caller-owned streams so that consecutive calls
+ * overlap: the INPUT copies go on stream_h2d, the launches (and FloydWarshall's
+ * per-variant D re-copy) on stream_compute after the inputs landed, the OUTPUT
+ * and error-count copies on stream_d2h after the last launch.  Keep every call's
+ * launches on ONE compute stream (inter-group pairs assume their kernel is not
+ * co-scheduled with another queue kernel).  err_host (u64[nvar]) and the host
+ * output buffers must be pinned and are valid only after the caller
+ * synchronises stream_d2h; host inputs must stay untouched until stream_h2d
+ * completes.  Returns RMT_OK if everything was enqueued (errors of the
+ * asynchronous work surface at the caller's synchronisation).
+ */
+int rmt_run_host_variants_pipelined(int kernel, int nvar, const int* variants, const rmt_bufs_t* host,
+                                    const rmt_bufs_t* dev, int64_t n, unsigned long long* err_host,
+                                    unsigned long long* err_dev, void* const* workspaces, const size_t* ws_bytes,
+                                    void* stream_h2d, void* stream_compute, void* stream_d2h, int64_t* h2d_bytes,
+                                    int64_t* d2h_bytes);
+
 /* Fault injection (BASELINE.json north_star item (4)): arm ONE single-bit flip
  * for subsequent launches until rmt_clear_faults().
  *   replica  0|1 (intra: 0 = even lane = consumer, 1 = odd lane = producer;

@@ -355,6 +355,75 @@ int rmt_run_host_variants(int kernel, int nvar, const int* variants, const rmt_b
   return RMT_OK;
 }
 
+int rmt_run_host_variants_pipelined(int kernel, int nvar, const int* variants, const rmt_bufs_t* host,
+                                    const rmt_bufs_t* dev, int64_t n, unsigned long long* err_host,
+                                    unsigned long long* err_dev, void* const* workspaces, const size_t* ws_bytes,
+                                    void* stream_h2d, void* stream_compute, void* stream_d2h, int64_t* h2d_bytes,
+                                    int64_t* d2h_bytes) {
+  if (kernel < 0 || kernel >= RMT_K_COUNT || nvar < 1 || !variants || !host || !dev || !err_host || !err_dev ||
+      !workspaces || !ws_bytes) {
+    set_error("rmt_run_host_variants_pipelined: bad arguments");
+    return RMT_EINVAL;
+  }
+  const KEntry& e = kTable[kernel];
+  cudaStream_t s1 = (cudaStream_t)stream_h2d, sc = (cudaStream_t)stream_compute, s3 = (cudaStream_t)stream_d2h;
+  int64_t hb = 0, db = 0;
+  int rc;
+  auto is_out = [&](int bi) {
+    for (int k = 0; k < e.nout; ++k)
+      if (e.out[k] == bi) return true;
+    return false;
+  };
+  cudaEvent_t ev_in, ev_done;
+  if ((rc = cuda_check(cudaEventCreateWithFlags(&ev_in, cudaEventDisableTiming), "event"))) return rc;
+  if ((rc = cuda_check(cudaEventCreateWithFlags(&ev_done, cudaEventDisableTiming), "event"))) return rc;
+  // inputs on the H2D stream (they overlap the previous call's compute and D2H)
+  for (int i = 0; i < e.nin; ++i) {
+    const int bi = e.in[i];
+    const rmt_buf_t& h = host->buf[bi];
+    const rmt_buf_t& d = dev->buf[bi];
+    if (!h.ptr || h.numel != d.numel || h.dtype != d.dtype) { set_error("host/dev schema mismatch"); return RMT_EINVAL; }
+    size_t bytes = (size_t)h.numel * dtype_bytes(h.dtype);
+    if ((rc = cuda_check(cudaMemcpyAsync(d.ptr, h.ptr, bytes, cudaMemcpyHostToDevice, s1), "H2D"))) return rc;
+    hb += (int64_t)bytes;
+  }
+  cudaEventRecord(ev_in, s1);
+  cudaStreamWaitEvent(sc, ev_in, 0);
+  for (int v = 0; v < nvar; ++v) {
+    // an in/out buffer (FloydWarshall's D) again before every later variant, in compute order
+    for (int i = 0; v > 0 && i < e.nin; ++i) {
+      const int bi = e.in[i];
+      if (!is_out(bi)) continue;
+      const rmt_buf_t& h = host->buf[bi];
+      const rmt_buf_t& d = dev->buf[bi];
+      size_t bytes = (size_t)h.numel * dtype_bytes(h.dtype);
+      if ((rc = cuda_check(cudaMemcpyAsync(d.ptr, h.ptr, bytes, cudaMemcpyHostToDevice, sc), "H2D"))) return rc;
+      hb += (int64_t)bytes;
+    }
+    if ((rc = cuda_check(cudaMemsetAsync(err_dev + v, 0, sizeof(unsigned long long), sc), "memset err"))) return rc;
+    rc = rmt_launch(kernel, variants[v], dev, n, err_dev + v, workspaces[v], ws_bytes[v], stream_compute);
+    if (rc) return rc;
+  }
+  cudaEventRecord(ev_done, sc);
+  cudaStreamWaitEvent(s3, ev_done, 0);
+  for (int i = 0; i < e.nout; ++i) {
+    const rmt_buf_t& h = host->buf[e.out[i]];
+    const rmt_buf_t& d = dev->buf[e.out[i]];
+    if (!h.ptr || h.numel != d.numel) { set_error("host/dev schema mismatch"); return RMT_EINVAL; }
+    size_t bytes = (size_t)h.numel * dtype_bytes(h.dtype);
+    if ((rc = cuda_check(cudaMemcpyAsync(h.ptr, d.ptr, bytes, cudaMemcpyDeviceToHost, s3), "D2H"))) return rc;
+    db += (int64_t)bytes;
+  }
+  if ((rc = cuda_check(cudaMemcpyAsync(err_host, err_dev, 8 * (size_t)nvar, cudaMemcpyDeviceToHost, s3), "D2H err")))
+    return rc;
+  db += 8 * nvar;
+  cudaEventDestroy(ev_in);  // released once the recorded work completes
+  cudaEventDestroy(ev_done);
+  if (h2d_bytes) *h2d_bytes = hb;
+  if (d2h_bytes) *d2h_bytes = db;
+  return cuda_check(cudaGetLastError(), "pipelined launch");
+}
+
 int rmt_inject_fault(int replica, int site, int bit, int64_t elem) {
   if (replica < 0 || replica > 1 || site < RMT_SITE_LOAD || site > RMT_SITE_STORE_ADDR || bit < 0 || bit > 31 ||
       elem < 0) {

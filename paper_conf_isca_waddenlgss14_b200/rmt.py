@@ -84,6 +84,11 @@ def lib() -> ctypes.CDLL:
                                             ctypes.POINTER(SZ), P, ctypes.POINTER(ctypes.c_int64),
                                             ctypes.POINTER(ctypes.c_int64)]
         L.rmt_run_host_variants.restype = I32
+        L.rmt_run_host_variants_pipelined.argtypes = [I32, I32, ctypes.POINTER(I32), ctypes.POINTER(_Bufs),
+                                                      ctypes.POINTER(_Bufs), I64, P, P, ctypes.POINTER(P),
+                                                      ctypes.POINTER(SZ), P, P, P, ctypes.POINTER(ctypes.c_int64),
+                                                      ctypes.POINTER(ctypes.c_int64)]
+        L.rmt_run_host_variants_pipelined.restype = I32
         L.rmt_inject_fault.argtypes = [I32, I32, I32, I64]
         L.rmt_inject_fault.restype = I32
         L.rmt_clear_faults.restype = I32
@@ -244,6 +249,28 @@ def run_host_variants(kernel: str, variants, host, dev, n: int, err_dev, workspa
                                        errs, err_dev.data_ptr(), wsp, wsb, stream, ctypes.byref(h2d),
                                        ctypes.byref(d2h)), f"rmt_run_host_variants({kernel})")
     return list(errs), h2d.value, d2h.value
+
+
+def run_host_variants_pipelined(kernel: str, variants, host, dev, n: int, err_dev, workspaces, err_host,
+                                streams, dims=()):
+    """rmt_run_host_variants_pipelined: enqueue the inputs on streams[0], the
+    launches on streams[1], the outputs and error counts on streams[2]; no
+    synchronisation.  err_host: a pinned int64 CPU tensor [len(variants)], valid
+    after streams[2] is synchronised (as are the host outputs).  Keep the host
+    buffer lists alive until then.  Returns (h2d_bytes, d2h_bytes)."""
+    nv = len(variants)
+    hb = make_bufs(kernel, host, dims)
+    db = make_bufs(kernel, dev, dims)
+    vids = (ctypes.c_int * nv)(*[VARIANTS[v] for v in variants])
+    wsp = (ctypes.c_void_p * nv)(*[w.data_ptr() if w is not None else None for w in workspaces])
+    wsb = (ctypes.c_size_t * nv)(*[w.numel() if w is not None else 0 for w in workspaces])
+    h2d = ctypes.c_int64(0)
+    d2h = ctypes.c_int64(0)
+    _check(lib().rmt_run_host_variants_pipelined(KERNELS[kernel], nv, vids, ctypes.byref(hb), ctypes.byref(db),
+                                                 int(n), err_host.data_ptr(), err_dev.data_ptr(), wsp, wsb,
+                                                 *[s.cuda_stream for s in streams], ctypes.byref(h2d),
+                                                 ctypes.byref(d2h)), f"rmt_run_host_variants_pipelined({kernel})")
+    return h2d.value, d2h.value
 
 
 def inject_fault(replica: int, site, bit: int, elem: int):

@@ -139,3 +139,32 @@ def test_input_only_16byte_aligned(make, variant):
     err = run(case.kernel, variant, b, case.n, case.dims)
     assert err == 0
     case.check(case.outputs(b))
+
+
+def test_pipelined_host_path_matches_oracle():
+    """rmt_run_host_variants_pipelined (bench.py's e2e leg): several kernels in a
+    row, inputs / launches / outputs on three streams, no host sync until the
+    end -- every output equals the oracle and every error count is 0."""
+    import oracle
+    from cases import BinarySearch, FloydWarshall, PrefixSum
+    variants = ["none", "intra_reg", "inter_group", "inter_cluster"]
+    cases = [BinarySearch(70001, 5003), PrefixSum(4096 * 7 + 3), FloydWarshall(64)]
+    streams = (torch.cuda.Stream(), torch.cuda.Stream(), torch.cuda.Stream())
+    runs = []
+    for c in cases:
+        dev = c.buffers()
+        host = [t.cpu().pin_memory() for t in dev]
+        errd = torch.zeros(len(variants), dtype=torch.int64, device="cuda")
+        errh = torch.zeros(len(variants), dtype=torch.int64).pin_memory()
+        wsl = [rmt.make_workspace(c.kernel, v, c.n, c.dims) for v in variants]
+        torch.cuda.synchronize()
+        rmt.run_host_variants_pipelined(c.kernel, variants, host, dev, c.n, errd, wsl, errh, streams, dims=c.dims)
+        runs.append((c, host, errh, dev, wsl))
+    for s in streams:
+        s.synchronize()
+    for c, host, errh, dev, wsl in runs:
+        assert errh.tolist() == [0] * len(variants), f"{c.kernel}: {errh.tolist()}"
+        if c.kernel == "floydwarshall":  # D in/out (the last variant's result), P out
+            c.check([host[0].numpy().view(np.uint32).reshape(c.n, c.n), host[1].numpy().view(np.uint32).reshape(c.n, c.n)])
+        else:
+            c.check([host[-1].numpy().view(np.uint32).reshape(-1)])
