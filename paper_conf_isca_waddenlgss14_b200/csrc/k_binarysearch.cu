@@ -362,7 +362,7 @@ __global__ void __launch_bounds__(BL * Geom<V>::DUP) bins_ghost_kernel(BsArgs a,
     unsigned key = a.q[jq];
     if constexpr (M == M_FAULT) key = rep.fault(SITE_LOAD, (long long)jq, key);
     const unsigned t = (unsigned)rep.ltid;
-    const unsigned seg = (a.N + BL - 1) / BL;
+    const unsigned seg = (unsigned)(((unsigned long long)a.N + BL - 1) / BL);  // N may be near 2^32
     const unsigned lo = min(a.N, t * seg), hi = min(a.N, lo + seg);
     bool writer;
     if (a.N == 0u) {

@@ -374,9 +374,16 @@ int rmt_run_host_variants_pipelined(int kernel, int nvar, const int* variants, c
       if (e.out[k] == bi) return true;
     return false;
   };
-  cudaEvent_t ev_in, ev_done;
-  if ((rc = cuda_check(cudaEventCreateWithFlags(&ev_in, cudaEventDisableTiming), "event"))) return rc;
-  if ((rc = cuda_check(cudaEventCreateWithFlags(&ev_done, cudaEventDisableTiming), "event"))) return rc;
+  struct Events {  // destroyed on every return (released once the recorded work completes)
+    cudaEvent_t in = nullptr, done = nullptr;
+    ~Events() {
+      if (in) cudaEventDestroy(in);
+      if (done) cudaEventDestroy(done);
+    }
+  } ev;
+  if ((rc = cuda_check(cudaEventCreateWithFlags(&ev.in, cudaEventDisableTiming), "event"))) return rc;
+  if ((rc = cuda_check(cudaEventCreateWithFlags(&ev.done, cudaEventDisableTiming), "event"))) return rc;
+  cudaEvent_t ev_in = ev.in, ev_done = ev.done;
   // inputs on the H2D stream (they overlap the previous call's compute and D2H)
   for (int i = 0; i < e.nin; ++i) {
     const int bi = e.in[i];
@@ -417,8 +424,6 @@ int rmt_run_host_variants_pipelined(int kernel, int nvar, const int* variants, c
   if ((rc = cuda_check(cudaMemcpyAsync(err_host, err_dev, 8 * (size_t)nvar, cudaMemcpyDeviceToHost, s3), "D2H err")))
     return rc;
   db += 8 * nvar;
-  cudaEventDestroy(ev_in);  // released once the recorded work completes
-  cudaEventDestroy(ev_done);
   if (h2d_bytes) *h2d_bytes = hb;
   if (d2h_bytes) *d2h_bytes = db;
   return cuda_check(cudaGetLastError(), "pipelined launch");
