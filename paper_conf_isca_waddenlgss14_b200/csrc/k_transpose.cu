@@ -109,7 +109,7 @@ int transpose_run(Launch& L) {
   return dispatch(L.variant, L.mode, [&](auto vm) {
     constexpr int V = decltype(vm)::V, M = decltype(vm)::M;
     return launch_std<V>(L, tr_kernel<V, M>, tr_kernel<V_NONE, M_NORMAL>, nsx * nty, BL, 0, a, "transpose",
-                         /*mult_inter=*/2);
+                         /*mult_inter=*/4);  // digest records: 4x the resident pairs 2.21 -> 2.10x
   });
 }
 
